@@ -1,0 +1,319 @@
+#!/usr/bin/env python
+"""bench.py — stimulus·gate·cycle evaluations per second of the gsim hot path on B200.
+
+Contract:
+  python bench.py --gpus N --steps K --warmup W           (N > 1: under torch.distributed.run)
+  python bench.py --impl reference ...                     (the CPU oracle arm, rank 0 only)
+
+A *step* is ``--cycles-per-step`` clock cycles (default 100) of the whole hot path —
+stimulus generation, every level of gates with the fused register latch, the remaining
+latches and the output MISR — over one batch of stimuli.  The default workload is
+BASELINE.json configs[3] (C4: RISC-V-core-scale synthetic, 1M gates + 50k registers,
+65,536 stimuli per GPU), the largest configuration that fits one GPU; its 1,000-cycle
+run is 10 steps.  Multi-GPU is weak scaling: every rank simulates its own 65,536 global
+lanes (lane_offset = rank * lanes) of the same netlist; the only collective is the
+all-reduce of the per-rank signatures.
+
+value = G_eval * lanes_total * cycles / max-over-ranks device time of the K timed steps.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "stimulus-gate-cycle evals/s at 1/2/4/8 B200; HBM GB/s vs roofline"
+UNIT = "sgc/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C4")
+    ap.add_argument("--cycles-per-step", type=int, default=100)
+    ap.add_argument("--lanes", type=int, default=0, help="override lanes per GPU")
+    ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-roofline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle CPU time")
+    ap.add_argument("--quick", action="store_true", help="ncu mode: no e2e/cpu/roofline/clocks")
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled DURING the timed region (200 ms)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm = [float(r[1]) for r in self.rows if len(r) > 2 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) > 2 and r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for i, n in enumerate(names):
+                if len(r) > 5 + i and r[5 + i].lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": sorted(reasons),
+                "samples": len(self.rows)}
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0}, "fallback"
+
+
+# ------------------------------------------------------------------ CPU oracle
+def oracle_rate(nl, cfg, lane_offset, seconds: float, cycles_cap: int | None = None):
+    """Time the oracle (as it stands) on a bounded sample: n_threads lanes x c cycles."""
+    import numpy as np
+    import oracle
+    threads = oracle.max_threads()
+    G = int((nl.gate_k > 0).sum())
+    lanes_total = cfg.lanes
+    # calibration: one lane per thread, 2 cycles
+    sample = np.linspace(0, lanes_total - 1, threads).astype(np.int64) + lane_offset
+    t = time.perf_counter()
+    oracle.simulate(nl, sample, 2, seed=cfg.stim_seed, threads=threads, want=("sig",))
+    dt = max(time.perf_counter() - t, 1e-3)
+    per_cycle = dt / 2
+    cycles = max(2, int(seconds / per_cycle))
+    if cycles_cap:
+        cycles = min(cycles, cycles_cap)
+    t = time.perf_counter()
+    oracle.simulate(nl, sample, cycles, seed=cfg.stim_seed, threads=threads, want=("sig",))
+    dt = time.perf_counter() - t
+    return {"value": G * len(sample) * cycles / dt, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "sample": f"{len(sample)} lanes (one per thread, spread over the batch) x {cycles} cycles "
+                      f"of {cfg.name}, generated stimuli seed {cfg.stim_seed}; {dt:.1f} s wall"}, dt
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as it stands, rank 0 only, same metric/config."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import numpy as np
+    import oracle
+    import workloads
+    cfg = workloads.CONFIGS[args.config]
+    nl = cfg.netlist()
+    G = int((nl.gate_k > 0).sum())
+    threads = oracle.max_threads()
+    sample = np.linspace(0, cfg.lanes - 1, threads).astype(np.int64)
+    # per step: every thread simulates one lane for c cycles; size c so the run is minutes
+    t = time.perf_counter()
+    oracle.simulate(nl, sample, 2, seed=cfg.stim_seed, threads=threads, want=("sig",))
+    per_cycle = max((time.perf_counter() - t) / 2, 1e-4)
+    budget = 150.0 / max(args.steps + args.warmup, 1)
+    c = max(1, min(args.cycles_per_step, int(budget / per_cycle)))
+    for _ in range(args.warmup):
+        oracle.simulate(nl, sample, c, seed=cfg.stim_seed, threads=threads, want=("sig",))
+    t = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.simulate(nl, sample, c, seed=cfg.stim_seed, threads=threads, want=("sig",))
+    dt = time.perf_counter() - t
+    val = G * len(sample) * c * args.steps / dt
+    line = {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": dt * 1e3 / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+            "impl": "reference",
+            "config": {"workload": f"{cfg.name}: {cfg.label}", "gates": G, "lanes_per_step": len(sample),
+                       "cycles_per_step": c},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": threads, "kind": "oracle",
+                             "sample": f"{len(sample)} lanes x {c} cycles per step of {cfg.name}"},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ GPU arm
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    import workloads
+    import paper_conf_ipps_gavierrprs23_b200 as gs
+    from paper_conf_ipps_gavierrprs23_b200 import dist as gdist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        print(f"warning: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    cfg = workloads.CONFIGS[args.config]
+    nl = cfg.netlist()
+    lanes = args.lanes or (cfg.lanes // cfg.shards if cfg.shards > 1 else cfg.lanes)
+    lane_offset = rank * lanes
+    t0 = time.perf_counter()
+    prog = gs.Netlist.from_arrays(nl).compile(balance=True)
+    compile_s = time.perf_counter() - t0
+    info = prog.info
+    G = info["n_eval_gates"]
+    if world > 1:
+        gdist.check_same_program(info["program_hash"])
+    stream = torch.cuda.Stream(device=local)
+    sim = gs.Sim(prog, lanes, lane_offset=lane_offset, kernel=args.kernel, device=local, stream=stream)
+    sim.bind_generated(cfg.stim_seed)
+    C = args.cycles_per_step
+    launches_per_cycle = sim.launches_per_cycle()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    for _ in range(args.warmup):
+        sim.step(C)
+    sim.sync()
+    torch.cuda.synchronize()
+    barrier()
+    clocks = ClockSampler(local)
+    if not args.quick:
+        clocks.start()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record(stream)
+    for _ in range(args.steps):
+        sim.step(C)
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    clk = clocks.stop() if not args.quick else None
+    ms = ev0.elapsed_time(ev1)
+    barrier()
+    ms_max = gdist.max_over_ranks(ms) if world > 1 else ms
+    sig = sim.signature()
+    red = gdist.reduce_signature(sig) if world > 1 else sig
+
+    total_sgc = float(G) * lanes * world * C * args.steps
+    value = total_sgc / (ms_max / 1e3)
+
+    # ---------------------------------------------------------------- roofline
+    roof = None
+    pk, pk_src = peaks()
+    if not args.no_roofline and not args.quick:
+        pr = sim.profile_step(min(C, 10))
+        achieved = pr["level_bytes"] / (pr["level_ms"] / 1e3) / 1e9
+        per_launch_bytes = pr["level_bytes"] / max(pr["level_launches"], 1)
+        roof = {"bound": "hbm", "kernel": "k_level_lut (kernel A, one launch per level)",
+                "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
+                "frac": achieved / pk["hbm_gbs"], "traffic": None,
+                "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({pk_src})",
+                "algorithmic_bytes_per_launch": per_launch_bytes,
+                "level_share_of_step": pr["level_ms"] / pr["total_ms"],
+                "avg_level_launch_us": pr["level_ms"] * 1e3 / max(pr["level_launches"], 1),
+                "measured": f"CUDA events around every level launch on the sim stream, "
+                            f"{min(C, 10)} un-graphed cycles after the timed region"}
+
+    # ---------------------------------------------------------------- e2e
+    e2e = None
+    if not args.no_e2e and not args.quick:
+        n_pi = info["n_pi"]
+        words = lanes // 64
+        K2 = max(1, min(args.steps, 3))
+        host = torch.empty((C, n_pi, words), dtype=torch.int64).pin_memory()
+        host.random_()
+        h_np = host.numpy().view(np.uint64)
+        out_buf = torch.empty((info["n_po"], words), dtype=torch.int64).pin_memory()
+        o_np = out_buf.numpy().view(np.uint64)
+        sim2 = sim
+        sim2.reset()
+        sim2.bind_host(h_np)            # warm-up: allocate the staging buffer
+        sim2.step(C)
+        sim2.read_outputs(o_np)
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(K2):
+            sim2.bind_host(h_np)        # H2D of this step's stimuli (pinned host -> device)
+            sim2.step(C)
+            sim2.read_outputs(o_np)     # D2H of this step's outputs
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ems = e0.elapsed_time(e1)
+        ems = gdist.max_over_ranks(ems) if world > 1 else ems
+        e2e = {"value": float(G) * lanes * world * C * K2 / (ems / 1e3), "unit": UNIT,
+               "h2d_bytes_per_step": int(host.numel() * 8), "d2h_bytes_per_step": int(out_buf.numel() * 8),
+               "steps": K2, "path": "gs_sim_bind_stimulus_host + gs_sim_step + gs_sim_read_outputs"}
+
+    # ---------------------------------------------------------------- cpu baseline
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.quick:
+        cpu, _ = oracle_rate(nl, cfg, lane_offset, args.cpu_seconds, cycles_cap=None)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+            "config": {"workload": f"{cfg.name}: {cfg.label}", "gates": G, "registers": info["n_reg"],
+                       "levels": info["n_levels"], "lanes_per_gpu": lanes, "lanes_total": lanes * world,
+                       "cycles_per_step": C, "kernel": args.kernel, "balance": True,
+                       "l2": "inputs larger than L2 (state %.1f GB per GPU)" % (info["n_rows"] * lanes / 8 / 1e9),
+                       "parallelism": f"dp{world} (stimulus sharding)", "compile_s": round(compile_s, 2),
+                       "paper_style_gcps": value * (G + info["n_reg"]) / G},
+            "gpu_launches": int(launches_per_cycle * C * args.steps),
+            "signature": {k: str(v) for k, v in red.items()},
+            "clocks": clk,
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+        }
+        print(json.dumps(line), flush=True)
+    sim.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,263 @@
+/*
+ * gsim.h — C-ABI of the B200-native batched, levelized circuit simulator.
+ *
+ * The calls follow the statement of the problem in PAPER.md (Gavier et al.,
+ * "Neural Network Compiler for Parallel High-Throughput Simulation of Digital
+ * Circuits"); "P:N" is PAPER.md line N.
+ *
+ *   netlist  : a digital circuit f:{0,1}^n -> {0,1}^m (§II-B) split into
+ *              LUTs of at most L inputs forming a DAG (§III-B1), with
+ *              D flip-flops on one global clock cut into pseudo-inputs
+ *              (Q) and pseudo-outputs (D) joined by a recurrent connection
+ *              (§III-C).
+ *   compile  : levelize the DAG (the merged NN layers, §III-D) with
+ *              level balancing, and compile every truth table to the
+ *              coefficients of its multilinear polynomial (Eq. 1 P:115,
+ *              Algorithm 1).
+ *   simulate : bind a batch of stimuli, step N clock cycles on the GPU, read the
+ *              outputs and register state back ("transfer the binary inputs
+ *              ... binary outputs obtained"); verify by comparing outputs.
+ *
+ * Conventions (all calls):
+ *   - Every call returns gs_status; GS_OK == 0, errors are negative.  The
+ *     thread-local message of the last failure is gs_last_error().  No C++
+ *     exception ever crosses this boundary.
+ *   - Arrays passed in are COPIED; the library never keeps a caller pointer.
+ *   - Device memory is CALLER-OWNED: the simulator works in one caller-provided
+ *     device workspace (e.g. a torch uint8 CUDA tensor) sized by
+ *     gs_sim_workspace_bytes; the hot path (gs_sim_step) never allocates.
+ *     The single exception is gs_sim_bind_stimulus_host, which keeps a
+ *     library-owned device staging buffer (grown on demand, freed by
+ *     gs_sim_destroy) for the paper-style host->device stimulus transfer.
+ *   - Handles are freed by their _destroy call; a gs_program must outlive every
+ *     gs_sim created from it.  One gs_sim is used from one host thread / stream.
+ *   - Lane s of a word is bit (s mod 64) of uint64 word floor(s/64) (little-endian:
+ *     also correct when the same memory is viewed as 32-bit words).
+ */
+#ifndef GSIM_H
+#define GSIM_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GSIM_VERSION "0.1.0"
+#define GS_MAX_K 6   /* largest LUT fan-in L supported by both kernels ("4, 6 or 8") */
+
+typedef int32_t gs_status;
+enum {
+    GS_OK = 0,
+    GS_ERR_ARG = -1,              /* bad argument / net id / truth-table bits >= 2^k   */
+    GS_ERR_ARITY = -2,            /* k > GS_MAX_K (or > opts.max_k)                    */
+    GS_ERR_UNDRIVEN = -3,         /* a register without D (gs_set_register_d)          */
+    GS_ERR_COMB_LOOP = -4,        /* the gate graph is not a DAG (reading R8)   */
+    GS_ERR_BUFFER_TOO_SMALL = -5, /* required size written back where documented       */
+    GS_ERR_CUDA = -6,             /* a CUDA runtime error (message in gs_last_error)   */
+    GS_ERR_STATE = -7,            /* call not valid in the current state               */
+    GS_ERR_NOMEM = -8             /* host allocation failure                           */
+};
+
+typedef uint32_t gs_net;          /* net id; see the numbering rules below */
+typedef struct gs_netlist gs_netlist;
+typedef struct gs_program gs_program;
+typedef struct gs_sim gs_sim;
+
+/* Thread-local text of the last error (never NULL; "" after success). */
+const char* gs_last_error(void);
+const char* gs_version(void);
+
+/* ======================================================================= netlist
+ * Nets are numbered in creation order by the incremental calls.  Every add_*
+ * call returns the new net id in *out.  A gate may reference any existing or
+ * later net (the compiler sorts); the gate graph must be acyclic once registers
+ * are cut (Q is a source, D a sink).
+ */
+gs_status gs_netlist_create(gs_netlist** out);
+gs_status gs_netlist_destroy(gs_netlist* nl);
+
+/* New primary input.  PIs are numbered 0,1,... in creation order (the "pi"
+ * index used by stimulus layouts). */
+gs_status gs_add_input(gs_netlist* nl, gs_net* out);
+
+/* Constant net (a 0-input LUT, "LUTs smaller than L"); value must be 0 or 1. */
+gs_status gs_add_const(gs_netlist* nl, int value, gs_net* out);
+
+/* k-input LUT (0 <= k <= GS_MAX_K).  in[0..k-1] are net ids (repeats are
+ * legal, reading R9).  tt is the truth table LSB-first: bit m = f(x) where x_i =
+ * bit i of m (reading R1; the paper's Algorithm 1 nests x_1 outermost, which is
+ * the same table under k-bit index reversal).  Bits >= 2^k must be zero. */
+gs_status gs_add_gate(gs_netlist* nl, uint32_t k, const gs_net* in, uint64_t tt, gs_net* out);
+
+/* D flip-flop on the global clock.  *q_out is its Q net (pseudo-input);
+ * init (0/1) is Q at cycle 0 (reading R3).  Registers are numbered 0,1,... in
+ * creation order (the "reg" index of register read/write layouts). */
+gs_status gs_add_register(gs_netlist* nl, int init, gs_net* q_out);
+
+/* Connect D of register q to net d (pseudo-output); separate from
+ * creation so that feedback through registers can be built.  Re-setting is
+ * allowed (last call wins). */
+gs_status gs_set_register_d(gs_netlist* nl, gs_net q, gs_net d);
+
+/* Mark net as a primary output; *po_index (may be NULL) receives its output
+ * index (0,1,... in call order).  A net may be marked more than once. */
+gs_status gs_mark_output(gs_netlist* nl, gs_net net, uint32_t* po_index);
+
+/* Bulk load (10M-gate netlists).  Only valid on an EMPTY netlist.  Net ids:
+ *   [0, n_pi)                  primary inputs 0..n_pi-1
+ *   [n_pi, n_pi+n_reg)         register Q nets 0..n_reg-1
+ *   [n_pi+n_reg, +n_gates)     gate g output
+ * gate g has k = gate_k[g] inputs gate_in[gate_in_off[g] .. gate_in_off[g+1]),
+ * truth table gate_tt[g]; register r has init reg_init[r] and D = reg_d[r];
+ * outputs are po[0..n_po).  Same validity rules as the incremental calls. */
+typedef struct {
+    uint32_t n_pi, n_reg, n_gates, n_po;
+    const uint8_t* reg_init;      /* [n_reg]     0/1                         */
+    const uint32_t* reg_d;        /* [n_reg]     net ids                     */
+    const uint8_t* gate_k;        /* [n_gates]                               */
+    const uint32_t* gate_in_off;  /* [n_gates+1] CSR offsets, gate_in_off[0]=0 */
+    const uint32_t* gate_in;      /* [gate_in_off[n_gates]] net ids          */
+    const uint64_t* gate_tt;      /* [n_gates]   LSB-first truth tables      */
+    const uint32_t* po;           /* [n_po]      net ids                     */
+} gs_netlist_arrays;
+gs_status gs_netlist_load_arrays(gs_netlist* nl, const gs_netlist_arrays* a);
+
+typedef struct {
+    uint32_t n_nets, n_pi, n_reg, n_gates, n_po;
+    uint64_t n_edges;
+} gs_netlist_counts;
+gs_status gs_netlist_get_counts(const gs_netlist* nl, gs_netlist_counts* out);
+
+/* ======================================================================= compile */
+typedef struct {
+    int balance;      /* 0: ASAP levels.  1: slack-based balancing within [ASAP, ALAP]
+                         (same depth; flattens the unbalanced level widths) */
+    uint32_t max_k;   /* reject gates wider than this (0 = GS_MAX_K)                  */
+} gs_compile_opts;
+
+/* Validate (GS_ERR_UNDRIVEN, GS_ERR_COMB_LOOP, GS_ERR_ARITY), levelize (level(g) =
+ * 1 + max level of its gate inputs; PIs, Qs, constants are level 0; optional
+ * balancing), compile every TT to multilinear coefficients, lay out state rows and
+ * pack per-level device descriptors.  opts may be NULL (balance=1). */
+gs_status gs_compile(const gs_netlist* nl, const gs_compile_opts* opts, gs_program** out);
+gs_status gs_program_destroy(gs_program* prog);
+
+typedef struct {
+    uint32_t n_pi, n_reg, n_po;
+    uint32_t n_gates;          /* all gates of the netlist                               */
+    uint32_t n_eval_gates;     /* gates evaluated per cycle (k >= 1) = G of the metric   */
+    uint32_t n_levels;         /* depth D = number of merged NN layers           */
+    uint32_t max_width, min_width;
+    uint32_t k_hist[GS_MAX_K + 1];
+    uint64_t n_edges;          /* sum of k over evaluated gates                          */
+    uint64_t nnz_coeffs;       /* nonzero w_S over all gates ("connections" of the merged
+                                  hidden->output layer)                    */
+    uint64_t hidden_neurons;   /* sum 2^k (worst-case hidden neurons)             */
+    uint64_t n_rows;           /* state rows                */
+    uint64_t program_hash;     /* hash of the compiled program (multi-rank consistency)  */
+} gs_program_info;
+gs_status gs_program_get_info(const gs_program* prog, gs_program_info* out);
+
+/* widths[l] = gates on level l+1 (l < n_levels).  n must be >= n_levels. */
+gs_status gs_program_level_widths(const gs_program* prog, uint32_t* widths, uint32_t n);
+
+/* level[g] for every gate in netlist order (0 for constants).  n >= n_gates. */
+gs_status gs_program_gate_levels(const gs_program* prog, uint32_t* level, uint32_t n);
+
+/* Multilinear coefficients w_S (LSB-first subset index) of gate g (netlist order),
+ * as compiled by the Möbius butterfly (Algorithm 1 in iterative form).  n >= 2^k. */
+gs_status gs_program_coeffs(const gs_program* prog, uint32_t gate, int32_t* w, uint32_t n);
+
+/* ======================================================================= simulate */
+enum {
+    GS_KERNEL_AUTO = 0,   /* = GS_KERNEL_LUT                                               */
+    GS_KERNEL_LUT = 1,    /* kernel A: bit-sliced LUT evaluation, 64 stimuli per word      */
+    GS_KERNEL_POLY = 2,   /* kernel B: the paper's network, sum_S w_S Theta(sum x - |S| + 1)
+                             per stimulus in int32, ballot-packed (Eq. 1-3)                */
+    GS_KERNEL_AB = 3      /* A writes, B recomputes every level and counts mismatches      */
+};
+
+typedef struct {
+    int device;                   /* CUDA device ordinal                                   */
+    void* stream;                 /* cudaStream_t all work is queued on (NULL = legacy)    */
+    uint64_t lanes;               /* stimuli in this shard, multiple of 64                 */
+    uint64_t lane_offset;         /* global index of local lane 0, multiple of 64          */
+    int kernel;                   /* GS_KERNEL_*                                           */
+    uint32_t n_trace_words;       /* local words whose outputs are recorded every cycle    */
+    const uint32_t* trace_words;  /* [n_trace_words] local word indices (copied)           */
+    uint32_t trace_cycles;        /* capacity of the trace, in cycles                      */
+    int use_graphs;               /* 1: replay each cycle as a CUDA graph (default)        */
+} gs_sim_opts;
+
+/* Device workspace bytes required for (prog, opts). */
+gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts, size_t* bytes);
+
+/* Create a simulator in the caller's device workspace (256-byte aligned, >= the
+ * size above, else GS_ERR_BUFFER_TOO_SMALL).  Uploads the program, then resets. */
+gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts, void* dev_workspace,
+                        size_t workspace_bytes, gs_sim** out);
+gs_status gs_sim_destroy(gs_sim* sim);
+
+/* Stimulus binding.  Generated: PI p of global lane s at cycle c is bit
+ * (s mod 64) of H(seed, p, c, s/64), the counter-based hash of reading R2
+ * (computed on the device every cycle; identical across shards).  Host: words
+ * laid out [cycle][pi][local word], `cycles` cycles starting at the NEXT cycle
+ * stepped; copied host->device on the stream (pinned memory recommended).
+ * Device: the same layout already in caller-owned device memory (not copied;
+ * must stay valid while stepping). */
+gs_status gs_sim_bind_stimulus_generated(gs_sim* sim, uint64_t seed);
+gs_status gs_sim_bind_stimulus_host(gs_sim* sim, const uint64_t* words, uint32_t cycles);
+gs_status gs_sim_bind_stimulus_device(gs_sim* sim, const uint64_t* dev_words, uint32_t cycles);
+
+/* Q := init, cycle := 0, MISR := 0, counters := 0, trace cleared. */
+gs_status gs_sim_reset(gs_sim* sim);
+
+/* Advance ncycles clock cycles (asynchronous on the stream).  Per cycle: stimulus
+ * rows, every level in order (gates + fused register latch into the other Q bank),
+ * remaining latches, output MISR/trace.  GS_ERR_STATE if no stimulus is bound or a
+ * host/device stimulus would run past its bound cycles. */
+gs_status gs_sim_step(gs_sim* sim, uint32_t ncycles);
+gs_status gs_sim_sync(gs_sim* sim);
+gs_status gs_sim_get_cycle(const gs_sim* sim, uint64_t* cycle);
+
+/* Readback (synchronous).  Layouts, with W = lanes/64 local words:
+ *   outputs   [po][W]  outputs of the last stepped cycle (before its latch, R4)
+ *   registers [reg][W] Q after the last clock edge
+ *   trace     [cycle][po][n_trace_words] for the first trace_cycles cycles
+ *   lane sigs [lanes]  per-lane 64-bit MISR over all outputs of all cycles (R5)
+ * nwords is the capacity of the host buffer in uint64 (GS_ERR_BUFFER_TOO_SMALL). */
+gs_status gs_sim_read_outputs(gs_sim* sim, uint64_t* host, size_t nwords);
+gs_status gs_sim_read_registers(gs_sim* sim, uint64_t* host, size_t nwords);
+gs_status gs_sim_write_registers(gs_sim* sim, const uint64_t* host, size_t nwords);
+gs_status gs_sim_read_trace(gs_sim* sim, uint64_t* host, size_t nwords, uint32_t* cycles_recorded);
+gs_status gs_sim_read_lane_signatures(gs_sim* sim, uint64_t* host, size_t nlanes);
+
+typedef struct {
+    uint64_t lane_sig_sum;          /* sum_s mix64(sig_s ^ mix64(s)) mod 2^64 (R6)     */
+    uint64_t out_popcount;          /* ones over all outputs, lanes and cycles        */
+    uint64_t ab_mismatch;           /* GS_KERNEL_AB: words where B != A               */
+    uint64_t invariant_violations;  /* kernel B outputs outside {0,1}         */
+    uint64_t cycles;                /* cycles stepped since reset                     */
+} gs_signature;
+gs_status gs_sim_read_signature(gs_sim* sim, gs_signature* out);
+
+/* Measurement support (bench.py roofline): step ncycles WITHOUT graphs, bracketing
+ * every level launch with CUDA events on the sim's stream.  Writes the summed
+ * device time of the level kernels, of the whole cycles, the number of level
+ * launches and the algorithmic bytes the level kernels moved. */
+typedef struct {
+    double level_ms, total_ms;
+    uint64_t level_launches, total_launches;
+    double level_bytes;
+} gs_profile;
+gs_status gs_sim_profile_step(gs_sim* sim, uint32_t ncycles, gs_profile* out);
+
+/* Number of kernel launches one gs_sim_step(1) issues (bench "gpu_launches"). */
+gs_status gs_sim_launches_per_cycle(const gs_sim* sim, uint64_t* launches);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GSIM_H */

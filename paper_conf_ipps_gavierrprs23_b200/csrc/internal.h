@@ -1,0 +1,85 @@
+// internal.h — host-side data structures of the gsim library (not part of the ABI).
+//
+// See DESIGN.md §"HBM layout" for the row map and descriptor formats.
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/gsim.h"
+
+namespace gs {
+
+// ---------------------------------------------------------------- errors
+void set_error(const std::string& msg);
+void clear_error();
+gs_status fail(gs_status code, const std::string& msg);
+
+// ---------------------------------------------------------------- netlist
+enum NetKind : uint8_t { NET_PI = 0, NET_REG = 1, NET_GATE = 2 };
+
+struct Netlist {
+    std::vector<uint8_t> net_kind;      // per net
+    std::vector<uint32_t> net_index;    // index within its kind
+    std::vector<uint32_t> pi_net;       // net id of PI p
+    std::vector<uint32_t> reg_net;      // net id of register r (its Q)
+    std::vector<uint8_t> reg_init;
+    std::vector<uint32_t> reg_d;        // net id, UINT32_MAX = unset
+    std::vector<uint32_t> gate_net;
+    std::vector<uint8_t> gate_k;
+    std::vector<uint32_t> gate_in_off{0};
+    std::vector<uint32_t> gate_in;      // net ids
+    std::vector<uint64_t> gate_tt;
+    std::vector<uint32_t> po_net;
+    uint32_t n_nets() const { return (uint32_t)net_kind.size(); }
+};
+
+// ---------------------------------------------------------------- program
+constexpr uint32_t QFLAG = 0x80000000u;   // row ref is a Q row: add the current bank offset
+constexpr uint32_t NONE32 = 0xFFFFFFFFu;
+
+// 16-byte per-gate auxiliary descriptor (device layout, see kernels.cu)
+struct GateAux {
+    uint64_t tt;      // LSB-first truth table
+    uint32_t qdst;    // bank-0 row of the register this gate's output also latches into, or NONE32
+    uint32_t k;       // fan-in
+};
+static_assert(sizeof(GateAux) == 16, "GateAux layout");
+
+struct Program {
+    uint32_t n_pi = 0, n_reg = 0, n_po = 0, n_gates = 0, n_eval = 0, n_levels = 0;
+    uint32_t row_pi0 = 2, row_q0 = 0, row_gate0 = 0;
+    uint64_t n_rows = 0;
+    bool any_wide = false;                    // some gate has k > 4
+
+    // execution order = level by level, k-grouped within a level
+    std::vector<uint32_t> level_off;          // [n_levels + 1] into exec order
+    std::vector<uint32_t> in_lo;              // [n_eval * 4] row refs (QFLAG for Q rows)
+    std::vector<uint32_t> in_hi;              // [n_eval * 2] (inputs 4, 5) if any_wide
+    std::vector<GateAux> aux;                 // [n_eval]
+    std::vector<uint32_t> term_off;           // [n_eval + 1] kernel B nonzero terms
+    std::vector<uint32_t> terms;              // S | (|S|-1)<<8 | (w & 0xffff)<<16
+    std::vector<uint32_t> po_rows;            // [n_po]  row refs
+    std::vector<uint32_t> latch_src;          // row refs
+    std::vector<uint32_t> latch_dst;          // register index r
+    std::vector<uint8_t> reg_init;
+
+    // queries
+    std::vector<uint32_t> gate_level;         // per netlist gate (0 for constants)
+    std::vector<uint32_t> coeff_off;          // per netlist gate into coeffs
+    std::vector<int32_t> coeffs;
+    std::vector<uint32_t> exec_gate;          // exec index -> netlist gate (for G count / debug)
+    gs_program_info info{};
+};
+
+gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out);
+
+// Möbius transform of one LSB-first truth table (Algorithm 1 as an iterative butterfly)
+void mobius_butterfly(uint64_t tt, uint32_t k, int32_t* w);
+
+}  // namespace gs
+
+struct gs_program {
+    gs::Program* p;
+};

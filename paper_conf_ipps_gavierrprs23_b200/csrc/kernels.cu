@@ -1,0 +1,462 @@
+// kernels.cu — the sm_100a hot path of gsim.
+//
+// One cycle of the simulated circuit = stimulus rows, then one launch per level
+// (the merged NN layers of PAPER.md §III-D), then the end-of-cycle kernel
+// (remaining register latches of the recurrent connection P:241, output MISR /
+// trace).  State is bit-packed and stimulus-major: row r holds one signal for all
+// lanes, 64 stimuli per uint64 word.
+//
+// Kernel A (k_level_lut): a level is a gather + Boolean evaluation, not a dense
+// contraction, so there are no tensor cores here: every thread loads 16 B of each
+// input row (coalesced: a warp reads 512 B contiguous per row), evaluates the gate's
+// truth table bit-sliced as a Shannon mux tree (2^k - 1 LOP3 per 32 lanes) and
+// stores 16 B of the output row (plus the fused latch store into the other Q bank).
+//
+// Kernel B (k_level_poly): the paper's two-layer network per gate (Fig. 2, P:130;
+// Eq. 1-3) evaluated per stimulus in int32: hidden neuron h_S = Theta(sum_{s in S}
+// x_s - |S| + 1), output sum_S w_S h_S (only the nonzero w_S, sparse as in P:187),
+// then ballot-packed back to 32 stimuli per word.  Outputs outside {0,1} are counted
+// (P:224 says they cannot happen).  Used standalone or as a cross-check of A.
+#include <cuda_runtime.h>
+
+#include "kernels.h"
+
+namespace gs {
+
+#define FULL 0xFFFFFFFFu
+
+__device__ __forceinline__ uint32_t resolve(uint32_t ref, uint32_t qcur) {
+    // Q rows are referenced bank-0 relative with QFLAG; add the current bank offset
+    return (ref & 0x7FFFFFFFu) + ((ref >> 31) ? qcur : 0u);
+}
+
+// ----------------------------------------------------------------------------- hash
+// splitmix64 finaliser + the counter-based stimulus hash of DESIGN.md reading R2.
+__device__ __forceinline__ unsigned long long dmix64(unsigned long long z) {
+    z += 0x9E3779B97F4A7C15ULL;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+    return z ^ (z >> 31);
+}
+
+// ------------------------------------------------------------------ kernel A: LUT
+// Bit-sliced Shannon expansion of an LSB-first truth table: stage 0 selects between
+// the minterm constants with x_0, stage i muxes pairs with x_i.  All operands are
+// 32-bit so every mux is one LOP3.
+template <int K>
+__device__ __forceinline__ uint32_t lut_eval(uint64_t tt, const uint32_t* x);
+
+// K = 5, 6: Shannon-expand on the top variables over 16-entry sub-tables, one at a
+// time, so the register footprint stays that of K = 4 (keeps occupancy up).
+template <int K>
+__device__ __forceinline__ uint32_t lut_eval_wide(uint64_t tt, const uint32_t* x) {
+    uint32_t y[4];
+#pragma unroll 1
+    for (int j = 0; j < (1 << (K - 4)); ++j) y[j] = lut_eval<4>(tt >> (16 * j), x);
+    if (K == 5) return (x[4] & y[1]) | (~x[4] & y[0]);
+    const uint32_t lo = (x[4] & y[1]) | (~x[4] & y[0]);
+    const uint32_t hi = (x[4] & y[3]) | (~x[4] & y[2]);
+    return (x[5] & hi) | (~x[5] & lo);
+}
+
+template <int K>
+__device__ __forceinline__ uint32_t lut_eval(uint64_t tt, const uint32_t* x) {
+    if (K > 4) return lut_eval_wide<K>(tt, x);
+    constexpr int KK = K > 4 ? 4 : K;
+    uint32_t v[1 << (KK - 1)];
+#pragma unroll
+    for (int j = 0; j < (1 << (KK - 1)); ++j) {
+        const uint32_t c0 = 0u - (uint32_t)((tt >> (2 * j)) & 1u);
+        const uint32_t c1 = 0u - (uint32_t)((tt >> (2 * j + 1)) & 1u);
+        v[j] = (x[0] & c1) | (~x[0] & c0);
+    }
+#pragma unroll
+    for (int i = 1; i < KK; ++i) {
+#pragma unroll
+        for (int j = 0; j < (1 << (KK - 1 - i)); ++j) v[j] = (x[i] & v[2 * j + 1]) | (~x[i] & v[2 * j]);
+    }
+    return v[0];
+}
+
+// evaluate 4 x 32-bit lanes-words (one 16-byte vector) of a K-input gate
+template <int K>
+__device__ __forceinline__ uint4 lut_eval4(uint64_t tt, const uint4* xv) {
+    uint4 y;
+    uint32_t x[K];
+#pragma unroll
+    for (int i = 0; i < K; ++i) x[i] = xv[i].x;
+    y.x = lut_eval<K>(tt, x);
+#pragma unroll
+    for (int i = 0; i < K; ++i) x[i] = xv[i].y;
+    y.y = lut_eval<K>(tt, x);
+#pragma unroll
+    for (int i = 0; i < K; ++i) x[i] = xv[i].z;
+    y.z = lut_eval<K>(tt, x);
+#pragma unroll
+    for (int i = 0; i < K; ++i) x[i] = xv[i].w;
+    y.w = lut_eval<K>(tt, x);
+    return y;
+}
+
+template <int K>
+__device__ __forceinline__ void lut_gate_vec16(const LevelArgs& a, uint32_t gate, uint4 in, uint32_t v,
+                                               uint64_t tt, uint32_t qdst) {
+    uint32_t r[6];
+    r[0] = in.x; r[1] = in.y; r[2] = in.z; r[3] = in.w;
+    if (K > 4) {
+        const uint2 hi = __ldg(a.dhi + gate);
+        r[4] = hi.x; r[5] = hi.y;
+    }
+    uint4 x[K];
+#pragma unroll
+    for (int i = 0; i < K; ++i) {
+        const uint32_t row = resolve(r[i], a.qcur);
+        x[i] = __ldg(reinterpret_cast<const uint4*>(a.state + (uint64_t)row * a.stride) + v);
+    }
+    const uint4 y = lut_eval4<K>(tt, x);
+    *(reinterpret_cast<uint4*>(a.state + (uint64_t)(a.row_gate0 + gate) * a.stride) + v) = y;
+    if (qdst != 0xFFFFFFFFu)
+        *(reinterpret_cast<uint4*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride) + v) = y;
+}
+
+template <int K>
+__device__ __forceinline__ void lut_gate_vec8(const LevelArgs& a, uint32_t gate, uint4 in, uint32_t v,
+                                              uint64_t tt, uint32_t qdst) {
+    uint32_t r[6];
+    r[0] = in.x; r[1] = in.y; r[2] = in.z; r[3] = in.w;
+    if (K > 4) {
+        const uint2 hi = __ldg(a.dhi + gate);
+        r[4] = hi.x; r[5] = hi.y;
+    }
+    uint2 x[K];
+#pragma unroll
+    for (int i = 0; i < K; ++i) {
+        const uint32_t row = resolve(r[i], a.qcur);
+        x[i] = __ldg(reinterpret_cast<const uint2*>(a.state + (uint64_t)row * a.stride) + v);
+    }
+    uint32_t xs[K];
+    uint2 y;
+#pragma unroll
+    for (int i = 0; i < K; ++i) xs[i] = x[i].x;
+    y.x = lut_eval<K>(tt, xs);
+#pragma unroll
+    for (int i = 0; i < K; ++i) xs[i] = x[i].y;
+    y.y = lut_eval<K>(tt, xs);
+    *(reinterpret_cast<uint2*>(a.state + (uint64_t)(a.row_gate0 + gate) * a.stride) + v) = y;
+    if (qdst != 0xFFFFFFFFu)
+        *(reinterpret_cast<uint2*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride) + v) = y;
+}
+
+// One thread = one gate x one vector (16 B = 128 stimuli, or 8 B = 64 when a row has an
+// odd number of words).  vpr = vectors per row; when vpr >= 32 every warp works on a
+// single gate (k is warp-uniform, loads are 512 B contiguous per input row).
+template <bool VEC16, bool POW2>
+__global__ void __launch_bounds__(256) k_level_lut(LevelArgs a, uint32_t vpr, uint32_t vshift) {
+    const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+    const uint32_t gi = POW2 ? (t >> vshift) : (t / vpr);
+    if (gi >= a.ng) return;
+    const uint32_t v = POW2 ? (t & (vpr - 1)) : (t - gi * vpr);
+    const uint32_t gate = a.g0 + gi;
+    const uint4 in = __ldg(a.din + gate);
+    const uint4 au = __ldg(reinterpret_cast<const uint4*>(a.aux) + gate);
+    const uint64_t tt = ((uint64_t)au.y << 32) | au.x;
+    const uint32_t qdst = au.z, k = au.w;
+    if (VEC16) {
+        switch (k) {
+            case 1: lut_gate_vec16<1>(a, gate, in, v, tt, qdst); break;
+            case 2: lut_gate_vec16<2>(a, gate, in, v, tt, qdst); break;
+            case 3: lut_gate_vec16<3>(a, gate, in, v, tt, qdst); break;
+            case 4: lut_gate_vec16<4>(a, gate, in, v, tt, qdst); break;
+            case 5: lut_gate_vec16<5>(a, gate, in, v, tt, qdst); break;
+            default: lut_gate_vec16<6>(a, gate, in, v, tt, qdst); break;
+        }
+    } else {
+        switch (k) {
+            case 1: lut_gate_vec8<1>(a, gate, in, v, tt, qdst); break;
+            case 2: lut_gate_vec8<2>(a, gate, in, v, tt, qdst); break;
+            case 3: lut_gate_vec8<3>(a, gate, in, v, tt, qdst); break;
+            case 4: lut_gate_vec8<4>(a, gate, in, v, tt, qdst); break;
+            case 5: lut_gate_vec8<5>(a, gate, in, v, tt, qdst); break;
+            default: lut_gate_vec8<6>(a, gate, in, v, tt, qdst); break;
+        }
+    }
+}
+
+cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s) {
+    if (a.ng == 0) return cudaSuccess;
+    const bool vec16 = (a.words % 2) == 0;
+    const uint32_t vpr = vec16 ? a.words / 2 : a.words;
+    const bool pow2 = (vpr & (vpr - 1)) == 0;
+    uint32_t vshift = 0;
+    while ((1u << vshift) < vpr) ++vshift;
+    const uint64_t threads = (uint64_t)a.ng * vpr;
+    if (threads >= (1ull << 31)) return cudaErrorInvalidValue;
+    const uint32_t blocks = (uint32_t)((threads + 255) / 256);
+    if (vec16) {
+        if (pow2) k_level_lut<true, true><<<blocks, 256, 0, s>>>(a, vpr, vshift);
+        else k_level_lut<true, false><<<blocks, 256, 0, s>>>(a, vpr, vshift);
+    } else {
+        if (pow2) k_level_lut<false, true><<<blocks, 256, 0, s>>>(a, vpr, vshift);
+        else k_level_lut<false, false><<<blocks, 256, 0, s>>>(a, vpr, vshift);
+    }
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------ kernel B: polynomial
+// One warp = one gate x 32 consecutive 32-bit words (1,024 stimuli).  Lane t owns
+// stimulus t of every word b; the words are transposed with shuffles so each lane
+// builds its own input point idx[b] (bit i = x_i), then evaluates the network.
+__global__ void __launch_bounds__(256) k_level_poly(LevelArgs a, uint32_t words32, uint32_t wpg, int check_only) {
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t gi = warp / wpg;
+    if (gi >= a.ng) return;                                   // warp-uniform
+    const uint32_t chunk = warp - gi * wpg;
+    const uint32_t gate = a.g0 + gi;
+    const uint32_t j = chunk * 32 + lane;                     // this lane's 32-bit word
+    const bool valid = j < words32;
+    const uint4 in = __ldg(a.din + gate);
+    const uint4 au = __ldg(reinterpret_cast<const uint4*>(a.aux) + gate);
+    const uint32_t qdst = au.z, k = au.w;
+    uint32_t r[6] = {in.x, in.y, in.z, in.w, 0u, 0u};
+    if (k > 4) {
+        const uint2 hi = __ldg(a.dhi + gate);
+        r[4] = hi.x; r[5] = hi.y;
+    }
+    uint32_t x[6];
+#pragma unroll
+    for (int i = 0; i < 6; ++i) {
+        x[i] = 0u;
+        if (i < (int)k && valid)
+            x[i] = __ldg(reinterpret_cast<const uint32_t*>(a.state + (uint64_t)resolve(r[i], a.qcur) * a.stride) + j);
+    }
+    // idx[b]: input point of stimulus `lane` in word b
+    uint32_t idx[32];
+#pragma unroll
+    for (int b = 0; b < 32; ++b) idx[b] = 0u;
+#pragma unroll
+    for (int i = 0; i < 6; ++i) {
+        if (i < (int)k) {
+#pragma unroll
+            for (int b = 0; b < 32; ++b) idx[b] |= ((__shfl_sync(FULL, x[i], b) >> lane) & 1u) << i;
+        }
+    }
+    // nonzero terms of this gate: lane t holds terms t and t + 32 (k <= 6 -> <= 64)
+    const uint32_t t0 = __ldg(a.term_off + gate), nt = __ldg(a.term_off + gate + 1) - t0;
+    const uint32_t myterm0 = lane < nt ? __ldg(a.terms + t0 + lane) : 0u;
+    const uint32_t myterm1 = lane + 32 < nt ? __ldg(a.terms + t0 + 32 + lane) : 0u;
+    int acc[32];
+#pragma unroll
+    for (int b = 0; b < 32; ++b) acc[b] = 0;
+    for (uint32_t i = 0; i < nt; ++i) {
+        const uint32_t tm = __shfl_sync(FULL, i < 32 ? myterm0 : myterm1, i & 31);
+        const uint32_t S = tm & 0xFFu;                         // monomial S (bit s <-> x_s)
+        const int bias = (int)(int8_t)((tm >> 8) & 0xFFu);     // |S| - 1   (Eq. 3)
+        const int w = (int)(int16_t)(tm >> 16);                // w_S       (Eq. 1)
+#pragma unroll
+        for (int b = 0; b < 32; ++b) {
+            // hidden neuron: Theta(sum_{s in S} x_s - |S| + 1) = [popc(idx & S) > |S| - 1]
+            const int h = __popc(idx[b] & S) > bias ? 1 : 0;
+            acc[b] += w * h;
+        }
+    }
+    uint32_t y = 0u, bad = 0u;
+#pragma unroll
+    for (int b = 0; b < 32; ++b) {
+        const uint32_t bal = __ballot_sync(FULL, acc[b] == 1);
+        if (lane == (uint32_t)b) y = bal;
+        bad += (acc[b] != 0 && acc[b] != 1) ? 1u : 0u;
+    }
+    // counts only the stimuli this warp really owns
+    if (!valid) bad = 0u;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) bad += __shfl_xor_sync(FULL, bad, o);
+    if (lane == 0 && bad) atomicAdd(&a.ctl->violations, (unsigned long long)bad);
+    if (!valid) return;
+    uint32_t* out = reinterpret_cast<uint32_t*>(a.state + (uint64_t)(a.row_gate0 + gate) * a.stride) + j;
+    if (check_only) {
+        const uint32_t ref = *out;
+        const uint32_t mism = __ballot_sync(__activemask(), ref != y);
+        if (mism && lane == __ffs(__activemask()) - 1) atomicAdd(&a.ctl->ab_mismatch, (unsigned long long)__popc(mism));
+    } else {
+        *out = y;
+        if (qdst != 0xFFFFFFFFu)
+            reinterpret_cast<uint32_t*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride)[j] = y;
+    }
+}
+
+cudaError_t launch_level_poly(const LevelArgs& a, int check_only, cudaStream_t s) {
+    if (a.ng == 0) return cudaSuccess;
+    const uint32_t words32 = a.words * 2;
+    const uint32_t wpg = (words32 + 31) / 32;
+    const uint64_t warps = (uint64_t)a.ng * wpg;
+    if (warps * 32 >= (1ull << 31)) return cudaErrorInvalidValue;
+    const uint32_t blocks = (uint32_t)((warps * 32 + 255) / 256);
+    k_level_poly<<<blocks, 256, 0, s>>>(a, words32, wpg, check_only);
+    return cudaGetLastError();
+}
+
+// --------------------------------------------------------------------- stimulus
+__global__ void __launch_bounds__(256) k_stim(Ctl* ctl, uint8_t* state, uint64_t stride, uint32_t words,
+                                              uint32_t row_pi0, uint32_t n_pi, uint64_t word_off) {
+    const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= (uint64_t)n_pi * words) return;
+    const uint32_t p = (uint32_t)(t / words), w = (uint32_t)(t - (uint64_t)p * words);
+    const unsigned long long c = ctl->cycle;
+    unsigned long long v;
+    if (ctl->stim_mode == 0) {
+        v = dmix64(dmix64(dmix64(ctl->seed ^ p) ^ c) ^ (word_off + w));
+    } else {
+        const unsigned long long* src = reinterpret_cast<const unsigned long long*>(ctl->stim_ptr);
+        v = src[((c - ctl->stim_base) * n_pi + p) * words + w];
+    }
+    reinterpret_cast<unsigned long long*>(state + (uint64_t)(row_pi0 + p) * stride)[w] = v;
+}
+
+cudaError_t launch_stim(Ctl* ctl, uint8_t* state, uint64_t stride, uint32_t words, uint32_t row_pi0,
+                        uint32_t n_pi, uint64_t word_off, cudaStream_t s) {
+    const uint64_t n = (uint64_t)n_pi * words;
+    if (n == 0) return cudaSuccess;
+    k_stim<<<(uint32_t)((n + 255) / 256), 256, 0, s>>>(ctl, state, stride, words, row_pi0, n_pi, word_off);
+    return cudaGetLastError();
+}
+
+// --------------------------------------------------------------- end of cycle
+// Blocks [0, latch_blocks): remaining register latches Q_next[r] = src (reads the
+// current bank / gate rows, writes the other bank, so order does not matter).
+// Blocks [latch_blocks, ...): one warp per word: output MISR (64 bit-planes per word,
+// DESIGN.md reading R5), output popcount and the per-cycle trace of sampled words.
+// The last block to finish advances the device cycle counter.
+constexpr unsigned long long MISR_POLY = 0x42F0E1EBA9EA3693ULL;   // CRC-64/ECMA-182
+
+__global__ void __launch_bounds__(256) k_end_cycle(EndArgs a, uint32_t latch_blocks) {
+    const unsigned long long c = a.ctl->cycle;
+    if (blockIdx.x < latch_blocks) {
+        const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+        if (t < (uint64_t)a.n_latch * a.words) {
+            const uint32_t e = (uint32_t)(t / a.words), w = (uint32_t)(t - (uint64_t)e * a.words);
+            const uint32_t src = resolve(__ldg(a.latch_src + e), a.qcur);
+            const uint32_t dst = a.row_q0 + __ldg(a.latch_dst + e) + a.qnext;
+            reinterpret_cast<unsigned long long*>(a.state + (uint64_t)dst * a.stride)[w] =
+                reinterpret_cast<const unsigned long long*>(a.state + (uint64_t)src * a.stride)[w];
+        }
+    } else {
+        const uint32_t warp = ((blockIdx.x - latch_blocks) * blockDim.x + threadIdx.x) >> 5;
+        const uint32_t lane = threadIdx.x & 31;
+        if (warp < a.words) {
+            const uint32_t w = warp;
+            unsigned long long v0 = 0, v1 = 0;
+            uint32_t pop = 0;
+            for (uint32_t o = lane; o < a.n_po; o += 32) {
+                const uint32_t row = resolve(__ldg(a.po_rows + o), a.qcur);
+                const unsigned long long x = reinterpret_cast<const unsigned long long*>(a.state + (uint64_t)row * a.stride)[w];
+                pop += __popcll(x);
+                if ((o & 63) < 32) v0 ^= x; else v1 ^= x;   // o mod 64 = lane or lane + 32
+            }
+            unsigned long long* m0 = a.misr + (uint64_t)lane * a.words + w;
+            unsigned long long* m1 = a.misr + (uint64_t)(lane + 32) * a.words + w;
+            const unsigned long long p0 = *m0, p1 = *m1;
+            const unsigned long long up0 = __shfl_up_sync(FULL, p0, 1);
+            const unsigned long long up1 = __shfl_up_sync(FULL, p1, 1);
+            const unsigned long long p31 = __shfl_sync(FULL, p0, 31);
+            const unsigned long long p63 = __shfl_sync(FULL, p1, 31);
+            const unsigned long long prev0 = lane == 0 ? 0ULL : up0;      // plane j-1 for j = lane
+            const unsigned long long prev1 = lane == 0 ? p31 : up1;       // plane j-1 for j = lane + 32
+            const unsigned long long fb0 = ((MISR_POLY >> lane) & 1ULL) ? p63 : 0ULL;
+            const unsigned long long fb1 = ((MISR_POLY >> (lane + 32)) & 1ULL) ? p63 : 0ULL;
+            *m0 = prev0 ^ fb0 ^ v0;
+            *m1 = prev1 ^ fb1 ^ v1;
+            const int32_t slot = a.trace ? __ldg(a.trace_slot + w) : -1;
+            if (slot >= 0 && c < a.trace_cap) {
+                for (uint32_t o = lane; o < a.n_po; o += 32) {
+                    const uint32_t row = resolve(__ldg(a.po_rows + o), a.qcur);
+                    a.trace[((uint64_t)c * a.n_po + o) * a.ntw + slot] =
+                        reinterpret_cast<const unsigned long long*>(a.state + (uint64_t)row * a.stride)[w];
+                }
+            }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) pop += __shfl_xor_sync(FULL, pop, o);
+            if (lane == 0 && pop) atomicAdd(&a.ctl->popcount, (unsigned long long)pop);
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        const unsigned int prev = atomicAdd(&a.ctl->done, 1u);
+        if (prev == gridDim.x - 1) {
+            a.ctl->done = 0u;
+            a.ctl->cycle = c + 1;
+            __threadfence();
+        }
+    }
+}
+
+cudaError_t launch_end_cycle(const EndArgs& a, cudaStream_t s) {
+    const uint64_t lt = (uint64_t)a.n_latch * a.words;
+    const uint32_t latch_blocks = (uint32_t)((lt + 255) / 256);
+    const uint32_t misr_blocks = (a.words * 32 + 255) / 256;
+    k_end_cycle<<<latch_blocks + misr_blocks, 256, 0, s>>>(a, latch_blocks);
+    return cudaGetLastError();
+}
+
+// --------------------------------------------------------------------- utilities
+__global__ void k_fill_rows(uint8_t* state, uint64_t stride, uint32_t words, uint32_t row0, uint32_t nrows,
+                            const uint8_t* init, int value) {
+    const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= (uint64_t)nrows * words) return;
+    const uint32_t r = (uint32_t)(t / words), w = (uint32_t)(t - (uint64_t)r * words);
+    const int bit = init ? init[r] : value;
+    reinterpret_cast<unsigned long long*>(state + (uint64_t)(row0 + r) * stride)[w] = bit ? ~0ULL : 0ULL;
+}
+
+cudaError_t launch_fill_rows(uint8_t* state, uint64_t stride, uint32_t words, uint32_t row0, uint32_t nrows,
+                             const uint8_t* init, int value, cudaStream_t s) {
+    const uint64_t n = (uint64_t)nrows * words;
+    if (n == 0) return cudaSuccess;
+    k_fill_rows<<<(uint32_t)((n + 255) / 256), 256, 0, s>>>(state, stride, words, row0, nrows, init, value);
+    return cudaGetLastError();
+}
+
+__global__ void k_gather_rows(const uint8_t* state, uint64_t stride, uint32_t words, const uint32_t* rows,
+                              uint32_t n, uint32_t qcur, unsigned long long* out) {
+    const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= (uint64_t)n * words) return;
+    const uint32_t o = (uint32_t)(t / words), w = (uint32_t)(t - (uint64_t)o * words);
+    out[t] = reinterpret_cast<const unsigned long long*>(state + (uint64_t)resolve(rows[o], qcur) * stride)[w];
+}
+
+cudaError_t launch_gather_rows(const uint8_t* state, uint64_t stride, uint32_t words, const uint32_t* rows,
+                               uint32_t n, uint32_t qcur, unsigned long long* out, cudaStream_t s) {
+    const uint64_t t = (uint64_t)n * words;
+    if (t == 0) return cudaSuccess;
+    k_gather_rows<<<(uint32_t)((t + 255) / 256), 256, 0, s>>>(state, stride, words, rows, n, qcur, out);
+    return cudaGetLastError();
+}
+
+// per-lane signature: transpose the 64 bit-planes of the lane's word (R5), then the
+// job signature term mix64(sig ^ mix64(global lane)) summed mod 2^64 (R6).
+__global__ void __launch_bounds__(256) k_lane_sigs(Ctl* ctl, const unsigned long long* misr, uint32_t words,
+                                                   uint64_t lane_offset, unsigned long long* lane_sigs) {
+    const uint64_t s = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    unsigned long long term = 0;
+    if (s < (uint64_t)words * 64) {
+        const uint32_t w = (uint32_t)(s >> 6), b = (uint32_t)(s & 63);
+        unsigned long long sig = 0;
+        for (int j = 0; j < 64; ++j) sig |= ((misr[(uint64_t)j * words + w] >> b) & 1ULL) << j;
+        lane_sigs[s] = sig;
+        term = dmix64(sig ^ dmix64(lane_offset + s));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) term += __shfl_xor_sync(FULL, term, o);
+    if ((threadIdx.x & 31) == 0 && term) atomicAdd(&ctl->sig_sum, term);
+}
+
+cudaError_t launch_lane_sigs(Ctl* ctl, const unsigned long long* misr, uint32_t words, uint64_t lane_offset,
+                             unsigned long long* lane_sigs, cudaStream_t s) {
+    const uint64_t n = (uint64_t)words * 64;
+    if (n == 0) return cudaSuccess;
+    k_lane_sigs<<<(uint32_t)((n + 255) / 256), 256, 0, s>>>(ctl, misr, words, lane_offset, lane_sigs);
+    return cudaGetLastError();
+}
+
+}  // namespace gs

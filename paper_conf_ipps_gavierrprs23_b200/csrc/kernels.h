@@ -1,0 +1,69 @@
+// kernels.h — launch wrappers of the sm_100a kernels (kernels.cu).  Internal.
+#pragma once
+
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "internal.h"
+
+namespace gs {
+
+// Device control block (first 256 B of the workspace).
+struct Ctl {
+    unsigned long long cycle;        // cycles stepped since reset (device-side clock)
+    unsigned long long seed;         // generated-stimulus seed
+    unsigned long long stim_ptr;     // host/device-bound stimulus [cycle][pi][word]
+    unsigned long long stim_base;    // cycle index of stim_ptr's first cycle
+    unsigned long long popcount;     // ones over all outputs of all cycles
+    unsigned long long ab_mismatch;  // kernel B != kernel A (GS_KERNEL_AB)
+    unsigned long long violations;   // kernel B outputs outside {0,1}
+    unsigned long long sig_sum;      // scratch for gs_sim_read_signature
+    unsigned int stim_mode;          // 0 generated, 1 bound buffer
+    unsigned int done;               // last-block counter of the end-of-cycle kernel
+};
+
+struct LevelArgs {
+    const uint4* din;
+    const GateAux* aux;
+    const uint2* dhi;
+    const uint32_t* term_off;
+    const uint32_t* terms;
+    uint32_t g0, ng;                  // exec-order gate range of the level
+    uint8_t* state;
+    uint64_t stride;                  // bytes per state row (= lanes / 8)
+    uint32_t words;                   // 64-bit words per row
+    uint32_t row_gate0;
+    uint32_t qcur, qnext;             // bank offsets (0 or n_reg) for Q refs / latch stores
+    Ctl* ctl;
+};
+
+struct EndArgs {
+    Ctl* ctl;
+    uint8_t* state;
+    uint64_t stride;
+    uint32_t words;
+    const uint32_t* latch_src;
+    const uint32_t* latch_dst;
+    uint32_t n_latch;
+    uint32_t row_q0, qcur, qnext;
+    const uint32_t* po_rows;
+    uint32_t n_po;
+    unsigned long long* misr;         // [64][words]
+    const int32_t* trace_slot;        // [words]
+    unsigned long long* trace;        // [trace_cap][n_po][ntw]
+    uint32_t ntw, trace_cap;
+};
+
+cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s);
+cudaError_t launch_level_poly(const LevelArgs& a, int check_only, cudaStream_t s);
+cudaError_t launch_stim(Ctl* ctl, uint8_t* state, uint64_t stride, uint32_t words, uint32_t row_pi0,
+                        uint32_t n_pi, uint64_t word_off, cudaStream_t s);
+cudaError_t launch_end_cycle(const EndArgs& a, cudaStream_t s);
+cudaError_t launch_fill_rows(uint8_t* state, uint64_t stride, uint32_t words, uint32_t row0, uint32_t nrows,
+                             const uint8_t* init, int value, cudaStream_t s);
+cudaError_t launch_gather_rows(const uint8_t* state, uint64_t stride, uint32_t words, const uint32_t* rows,
+                               uint32_t n, uint32_t qcur, unsigned long long* out, cudaStream_t s);
+cudaError_t launch_lane_sigs(Ctl* ctl, const unsigned long long* misr, uint32_t words, uint64_t lane_offset,
+                             unsigned long long* lane_sigs, cudaStream_t s);
+
+}  // namespace gs

@@ -1,0 +1,556 @@
+// sim.cpp — the simulation engine half of the C-ABI (include/gsim.h).
+//
+// Per clock cycle (P:241 recurrent connection, P:271 stimulus in / outputs out):
+//   stim kernel -> one level kernel per level (A, B or A+B) -> end-of-cycle kernel.
+// The per-cycle launch sequence only depends on the Q-bank parity, so it is captured
+// once per parity as a CUDA graph and replayed; the cycle index lives on the device
+// (Ctl::cycle) and is advanced by the end-of-cycle kernel.
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+#include "internal.h"
+#include "kernels.h"
+
+using namespace gs;
+
+namespace {
+
+size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+struct Layout {
+    size_t ctl, state, din, aux, dhi, term_off, terms, po_rows, latch_src, latch_dst, reg_init,
+        trace_slot, misr, trace, lane_sigs, scratch, total;
+};
+
+Layout make_layout(const Program& p, const gs_sim_opts& o) {
+    Layout L{};
+    const uint64_t words = o.lanes / 64;
+    const uint64_t stride = words * 8;
+    const bool poly = o.kernel == GS_KERNEL_POLY || o.kernel == GS_KERNEL_AB;
+    size_t off = 0;
+    auto take = [&](size_t bytes) {
+        size_t at = off;
+        off = align256(off + bytes);
+        return at;
+    };
+    L.ctl = take(sizeof(Ctl));
+    L.state = take((size_t)p.n_rows * stride);
+    L.din = take((size_t)p.n_eval * 16);
+    L.aux = take((size_t)p.n_eval * 16);
+    L.dhi = take(p.any_wide ? (size_t)p.n_eval * 8 : 0);
+    L.term_off = take(poly ? ((size_t)p.n_eval + 1) * 4 : 0);
+    L.terms = take(poly ? p.terms.size() * 4 : 0);
+    L.po_rows = take((size_t)p.n_po * 4);
+    L.latch_src = take(p.latch_src.size() * 4);
+    L.latch_dst = take(p.latch_dst.size() * 4);
+    L.reg_init = take(p.reg_init.size());
+    L.trace_slot = take((size_t)words * 4);
+    L.misr = take((size_t)64 * words * 8);
+    L.trace = take((size_t)o.trace_cycles * p.n_po * o.n_trace_words * 8);
+    L.lane_sigs = take((size_t)o.lanes * 8);
+    L.scratch = take((size_t)p.n_po * words * 8);
+    L.total = off;
+    return L;
+}
+
+}  // namespace
+
+struct gs_sim {
+    const Program* prog = nullptr;
+    gs_sim_opts opts{};
+    std::vector<uint32_t> trace_words;
+    Layout L{};
+    uint8_t* ws = nullptr;
+    cudaStream_t stream = nullptr, cap = nullptr;
+    uint32_t words = 0;
+    uint64_t stride = 0;
+    uint64_t cycle = 0;               // host mirror of Ctl::cycle
+    int bound = 0;                    // 0 none, 1 generated, 2 host/device buffer
+    uint64_t bound_seed = 0, bound_ptr = 0, bound_base = 0, bound_cycles = 0;
+    uint64_t bind_stage[3] = {0, 0, 0};
+    uint32_t bind_mode = 0;
+    void* host_stage = nullptr;       // library-owned device copy of host stimulus
+    size_t host_stage_bytes = 0;
+    cudaGraphExec_t exec[2] = {nullptr, nullptr};
+
+    Ctl* ctl() const { return reinterpret_cast<Ctl*>(ws + L.ctl); }
+    uint8_t* state() const { return ws + L.state; }
+    template <class T> T* at(size_t off) const { return reinterpret_cast<T*>(ws + off); }
+};
+
+#define CU(call)                                                                           \
+    do {                                                                                   \
+        cudaError_t e_ = (call);                                                           \
+        if (e_ != cudaSuccess)                                                             \
+            return fail(GS_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_));  \
+    } while (0)
+
+static LevelArgs level_args(const gs_sim* s, uint32_t l, uint32_t parity) {
+    const Program& p = *s->prog;
+    LevelArgs a{};
+    a.din = s->at<const uint4>(s->L.din);
+    a.aux = s->at<const GateAux>(s->L.aux);
+    a.dhi = p.any_wide ? s->at<const uint2>(s->L.dhi) : nullptr;
+    a.term_off = s->at<const uint32_t>(s->L.term_off);
+    a.terms = s->at<const uint32_t>(s->L.terms);
+    a.g0 = p.level_off[l];
+    a.ng = p.level_off[l + 1] - p.level_off[l];
+    a.state = s->state();
+    a.stride = s->stride;
+    a.words = s->words;
+    a.row_gate0 = p.row_gate0;
+    a.qcur = parity ? p.n_reg : 0;
+    a.qnext = parity ? 0 : p.n_reg;
+    a.ctl = s->ctl();
+    return a;
+}
+
+static EndArgs end_args(const gs_sim* s, uint32_t parity) {
+    const Program& p = *s->prog;
+    EndArgs e{};
+    e.ctl = s->ctl();
+    e.state = s->state();
+    e.stride = s->stride;
+    e.words = s->words;
+    e.latch_src = s->at<const uint32_t>(s->L.latch_src);
+    e.latch_dst = s->at<const uint32_t>(s->L.latch_dst);
+    e.n_latch = (uint32_t)p.latch_src.size();
+    e.row_q0 = p.row_q0;
+    e.qcur = parity ? p.n_reg : 0;
+    e.qnext = parity ? 0 : p.n_reg;
+    e.po_rows = s->at<const uint32_t>(s->L.po_rows);
+    e.n_po = p.n_po;
+    e.misr = s->at<unsigned long long>(s->L.misr);
+    e.trace_slot = s->at<const int32_t>(s->L.trace_slot);
+    e.trace = (s->opts.n_trace_words && s->opts.trace_cycles) ? s->at<unsigned long long>(s->L.trace) : nullptr;
+    e.ntw = s->opts.n_trace_words;
+    e.trace_cap = s->opts.trace_cycles;
+    return e;
+}
+
+static cudaError_t level_launch(const gs_sim* s, uint32_t l, uint32_t parity, cudaStream_t st) {
+    const LevelArgs a = level_args(s, l, parity);
+    switch (s->opts.kernel) {
+        case GS_KERNEL_POLY: return launch_level_poly(a, 0, st);
+        case GS_KERNEL_AB: {
+            cudaError_t e = launch_level_lut(a, st);
+            if (e != cudaSuccess) return e;
+            return launch_level_poly(a, 1, st);
+        }
+        default: return launch_level_lut(a, st);
+    }
+}
+
+static cudaError_t cycle_launches(const gs_sim* s, uint32_t parity, cudaStream_t st,
+                                  std::vector<cudaEvent_t>* evs = nullptr) {
+    const Program& p = *s->prog;
+    cudaError_t e = launch_stim(s->ctl(), s->state(), s->stride, s->words, p.row_pi0, p.n_pi,
+                                s->opts.lane_offset / 64, st);
+    if (e != cudaSuccess) return e;
+    for (uint32_t l = 0; l < p.n_levels; ++l) {
+        if (evs) cudaEventRecord((*evs)[2 * l], st);
+        e = level_launch(s, l, parity, st);
+        if (e != cudaSuccess) return e;
+        if (evs) cudaEventRecord((*evs)[2 * l + 1], st);
+    }
+    return launch_end_cycle(end_args(s, parity), st);
+}
+
+static gs_status ensure_graph(gs_sim* s, uint32_t parity) {
+    if (s->exec[parity]) return GS_OK;
+    cudaGraph_t g = nullptr;
+    CU(cudaStreamBeginCapture(s->cap, cudaStreamCaptureModeThreadLocal));
+    cudaError_t e = cycle_launches(s, parity, s->cap);
+    cudaError_t e2 = cudaStreamEndCapture(s->cap, &g);
+    if (e != cudaSuccess) {
+        if (g) cudaGraphDestroy(g);
+        return fail(GS_ERR_CUDA, std::string("graph capture: ") + cudaGetErrorString(e));
+    }
+    CU(e2);
+    cudaError_t e3 = cudaGraphInstantiate(&s->exec[parity], g, 0);
+    cudaGraphDestroy(g);
+    CU(e3);
+    return GS_OK;
+}
+
+static gs_status check_sim(const gs_sim* s, const char* fn) {
+    if (!s) return fail(GS_ERR_ARG, std::string(fn) + ": NULL sim");
+    return GS_OK;
+}
+
+// Ctl fields seed, stim_ptr, stim_base are contiguous, stim_mode follows later
+static gs_status write_binding(gs_sim* s) {
+    static_assert(offsetof(Ctl, stim_ptr) == offsetof(Ctl, seed) + 8, "Ctl layout");
+    static_assert(offsetof(Ctl, stim_base) == offsetof(Ctl, seed) + 16, "Ctl layout");
+    s->bind_stage[0] = s->bound_seed;
+    s->bind_stage[1] = s->bound_ptr;
+    s->bind_stage[2] = s->bound_base;
+    s->bind_mode = s->bound == 2 ? 1u : 0u;
+    CU(cudaMemcpyAsync(s->ws + s->L.ctl + offsetof(Ctl, seed), s->bind_stage, 24, cudaMemcpyHostToDevice, s->stream));
+    CU(cudaMemcpyAsync(s->ws + s->L.ctl + offsetof(Ctl, stim_mode), &s->bind_mode, 4, cudaMemcpyHostToDevice, s->stream));
+    CU(cudaStreamSynchronize(s->stream));   // the staging fields may be rewritten by the next bind
+    return GS_OK;
+}
+
+extern "C" {
+
+gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts, size_t* bytes) {
+    if (!prog || !opts || !bytes) return fail(GS_ERR_ARG, "gs_sim_workspace_bytes: NULL argument");
+    if (opts->lanes == 0 || opts->lanes % 64) return fail(GS_ERR_ARG, "lanes must be a positive multiple of 64");
+    if (opts->lanes / 64 >= (1ull << 31)) return fail(GS_ERR_ARG, "too many lanes");
+    *bytes = make_layout(*prog->p, *opts).total;
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts, void* dev_ws, size_t bytes, gs_sim** out) {
+    if (!prog || !opts || !out || !dev_ws) return fail(GS_ERR_ARG, "gs_sim_create: NULL argument");
+    if (opts->lanes == 0 || opts->lanes % 64) return fail(GS_ERR_ARG, "gs_sim_create: lanes must be a positive multiple of 64");
+    if (opts->lane_offset % 64) return fail(GS_ERR_ARG, "gs_sim_create: lane_offset must be a multiple of 64");
+    if (opts->kernel < GS_KERNEL_AUTO || opts->kernel > GS_KERNEL_AB) return fail(GS_ERR_ARG, "gs_sim_create: bad kernel");
+    if (opts->n_trace_words && !opts->trace_words) return fail(GS_ERR_ARG, "gs_sim_create: trace_words is NULL");
+    if ((reinterpret_cast<uintptr_t>(dev_ws) & 255) != 0) return fail(GS_ERR_ARG, "gs_sim_create: workspace must be 256-byte aligned");
+    const Program& p = *prog->p;
+    const uint32_t words = (uint32_t)(opts->lanes / 64);
+    for (uint32_t i = 0; i < opts->n_trace_words; ++i)
+        if (opts->trace_words[i] >= words) return fail(GS_ERR_ARG, "gs_sim_create: trace word out of range");
+    Layout L = make_layout(p, *opts);
+    if (bytes < L.total) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_create: workspace smaller than gs_sim_workspace_bytes");
+    CU(cudaSetDevice(opts->device));
+    gs_sim* s = new gs_sim();
+    s->prog = &p;
+    s->opts = *opts;
+    if (s->opts.kernel == GS_KERNEL_AUTO) s->opts.kernel = GS_KERNEL_LUT;
+    s->trace_words.assign(opts->trace_words, opts->trace_words + opts->n_trace_words);
+    s->opts.trace_words = s->trace_words.data();
+    s->L = L;
+    s->ws = static_cast<uint8_t*>(dev_ws);
+    s->stream = static_cast<cudaStream_t>(opts->stream);
+    s->words = words;
+    s->stride = (uint64_t)words * 8;
+    auto cleanup = [&](gs_status st) {
+        if (s->cap) cudaStreamDestroy(s->cap);
+        delete s;
+        return st;
+    };
+    cudaError_t e = cudaStreamCreateWithFlags(&s->cap, cudaStreamNonBlocking);
+    if (e != cudaSuccess) return cleanup(fail(GS_ERR_CUDA, std::string("cudaStreamCreate: ") + cudaGetErrorString(e)));
+    // upload the program (descriptors are device-resident for the sim's lifetime)
+    struct Up { size_t off; const void* src; size_t n; };
+    std::vector<int32_t> slot(words, -1);
+    for (uint32_t i = 0; i < opts->n_trace_words; ++i) slot[opts->trace_words[i]] = (int32_t)i;
+    const bool poly = s->opts.kernel != GS_KERNEL_LUT;
+    std::vector<Up> ups = {
+        {L.din, p.in_lo.data(), p.in_lo.size() * 4},
+        {L.aux, p.aux.data(), p.aux.size() * sizeof(GateAux)},
+        {L.dhi, p.in_hi.data(), p.any_wide ? p.in_hi.size() * 4 : 0},
+        {L.term_off, p.term_off.data(), poly ? p.term_off.size() * 4 : 0},
+        {L.terms, p.terms.data(), poly ? p.terms.size() * 4 : 0},
+        {L.po_rows, p.po_rows.data(), p.po_rows.size() * 4},
+        {L.latch_src, p.latch_src.data(), p.latch_src.size() * 4},
+        {L.latch_dst, p.latch_dst.data(), p.latch_dst.size() * 4},
+        {L.reg_init, p.reg_init.data(), p.reg_init.size()},
+        {L.trace_slot, slot.data(), slot.size() * 4},
+    };
+    for (const Up& u : ups) {
+        if (!u.n) continue;
+        e = cudaMemcpyAsync(s->ws + u.off, u.src, u.n, cudaMemcpyHostToDevice, s->stream);
+        if (e != cudaSuccess) return cleanup(fail(GS_ERR_CUDA, std::string("upload: ") + cudaGetErrorString(e)));
+    }
+    e = cudaStreamSynchronize(s->stream);   // host vectors above are temporaries
+    if (e != cudaSuccess) return cleanup(fail(GS_ERR_CUDA, std::string("upload sync: ") + cudaGetErrorString(e)));
+    gs_status st = gs_sim_reset(s);
+    if (st != GS_OK) return cleanup(st);
+    *out = s;
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_destroy(gs_sim* s) {
+    if (!s) return GS_OK;
+    cudaSetDevice(s->opts.device);
+    cudaStreamSynchronize(s->stream);
+    for (auto& x : s->exec)
+        if (x) cudaGraphExecDestroy(x);
+    if (s->cap) cudaStreamDestroy(s->cap);
+    if (s->host_stage) cudaFree(s->host_stage);
+    delete s;
+    return GS_OK;
+}
+
+gs_status gs_sim_reset(gs_sim* s) {
+    if (gs_status st = check_sim(s, "gs_sim_reset")) return st;
+    const Program& p = *s->prog;
+    CU(cudaSetDevice(s->opts.device));
+    CU(cudaMemsetAsync(s->ws + s->L.ctl, 0, sizeof(Ctl), s->stream));
+    CU(cudaMemsetAsync(s->ws + s->L.misr, 0, (size_t)64 * s->words * 8, s->stream));
+    if (s->L.lane_sigs != s->L.scratch) CU(cudaMemsetAsync(s->ws + s->L.lane_sigs, 0, (size_t)s->opts.lanes * 8, s->stream));
+    size_t tbytes = (size_t)s->opts.trace_cycles * p.n_po * s->opts.n_trace_words * 8;
+    if (tbytes) CU(cudaMemsetAsync(s->ws + s->L.trace, 0, tbytes, s->stream));
+    CU(launch_fill_rows(s->state(), s->stride, s->words, 0, 1, nullptr, 0, s->stream));          // const0
+    CU(launch_fill_rows(s->state(), s->stride, s->words, 1, 1, nullptr, 1, s->stream));          // const1
+    CU(launch_fill_rows(s->state(), s->stride, s->words, p.row_q0, p.n_reg, s->at<const uint8_t>(s->L.reg_init), 0, s->stream));
+    s->cycle = 0;
+    // keep the binding; a bound buffer restarts at its first cycle
+    s->bound_base = 0;
+    if (s->bound)
+        if (gs_status st = write_binding(s)) return st;
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_bind_stimulus_generated(gs_sim* s, uint64_t seed) {
+    if (gs_status st = check_sim(s, "gs_sim_bind_stimulus_generated")) return st;
+    CU(cudaSetDevice(s->opts.device));
+    s->bound = 1;
+    s->bound_seed = seed;
+    s->bound_ptr = 0;
+    s->bound_base = s->cycle;
+    s->bound_cycles = 0;
+    if (gs_status st = write_binding(s)) return st;
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_bind_stimulus_device(gs_sim* s, const uint64_t* dev_words, uint32_t cycles) {
+    if (gs_status st = check_sim(s, "gs_sim_bind_stimulus_device")) return st;
+    if (!dev_words && cycles) return fail(GS_ERR_ARG, "gs_sim_bind_stimulus_device: NULL words");
+    CU(cudaSetDevice(s->opts.device));
+    s->bound = 2;
+    s->bound_seed = 0;
+    s->bound_ptr = reinterpret_cast<uint64_t>(dev_words);
+    s->bound_base = s->cycle;
+    s->bound_cycles = cycles;
+    if (gs_status st = write_binding(s)) return st;
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_bind_stimulus_host(gs_sim* s, const uint64_t* words, uint32_t cycles) {
+    if (gs_status st = check_sim(s, "gs_sim_bind_stimulus_host")) return st;
+    if (!words && cycles) return fail(GS_ERR_ARG, "gs_sim_bind_stimulus_host: NULL words");
+    CU(cudaSetDevice(s->opts.device));
+    const size_t bytes = (size_t)cycles * s->prog->n_pi * s->words * 8;
+    if (bytes > s->host_stage_bytes) {
+        CU(cudaStreamSynchronize(s->stream));
+        if (s->host_stage) cudaFree(s->host_stage);
+        s->host_stage = nullptr;
+        s->host_stage_bytes = 0;
+        CU(cudaMalloc(&s->host_stage, bytes));
+        s->host_stage_bytes = bytes;
+    }
+    if (bytes) CU(cudaMemcpyAsync(s->host_stage, words, bytes, cudaMemcpyHostToDevice, s->stream));
+    s->bound = 2;
+    s->bound_seed = 0;
+    s->bound_ptr = reinterpret_cast<uint64_t>(s->host_stage);
+    s->bound_base = s->cycle;
+    s->bound_cycles = cycles;
+    if (gs_status st = write_binding(s)) return st;
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_step(gs_sim* s, uint32_t n) {
+    if (gs_status st = check_sim(s, "gs_sim_step")) return st;
+    if (!s->bound) return fail(GS_ERR_STATE, "gs_sim_step: no stimulus bound");
+    if (s->bound == 2 && s->cycle + n > s->bound_base + s->bound_cycles)
+        return fail(GS_ERR_STATE, "gs_sim_step: stepping past the bound stimulus cycles");
+    CU(cudaSetDevice(s->opts.device));
+    for (uint32_t i = 0; i < n; ++i) {
+        const uint32_t parity = (uint32_t)(s->cycle & 1);
+        if (s->opts.use_graphs) {
+            if (gs_status st = ensure_graph(s, parity)) return st;
+            CU(cudaGraphLaunch(s->exec[parity], s->stream));
+        } else {
+            CU(cycle_launches(s, parity, s->stream));
+        }
+        s->cycle++;
+    }
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_sync(gs_sim* s) {
+    if (gs_status st = check_sim(s, "gs_sim_sync")) return st;
+    CU(cudaSetDevice(s->opts.device));
+    CU(cudaStreamSynchronize(s->stream));
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_get_cycle(const gs_sim* s, uint64_t* cycle) {
+    if (!s || !cycle) return fail(GS_ERR_ARG, "gs_sim_get_cycle: NULL argument");
+    *cycle = s->cycle;
+    return GS_OK;
+}
+
+gs_status gs_sim_read_outputs(gs_sim* s, uint64_t* host, size_t nwords) {
+    if (gs_status st = check_sim(s, "gs_sim_read_outputs")) return st;
+    const Program& p = *s->prog;
+    const size_t need = (size_t)p.n_po * s->words;
+    if (!host && need) return fail(GS_ERR_ARG, "gs_sim_read_outputs: NULL buffer");
+    if (nwords < need) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_read_outputs: need n_po * lanes/64 words");
+    if (s->cycle == 0) return fail(GS_ERR_STATE, "gs_sim_read_outputs: no cycle stepped yet");
+    CU(cudaSetDevice(s->opts.device));
+    const uint32_t last_parity = (uint32_t)((s->cycle - 1) & 1);
+    CU(launch_gather_rows(s->state(), s->stride, s->words, s->at<const uint32_t>(s->L.po_rows), p.n_po,
+                          last_parity ? p.n_reg : 0, s->at<unsigned long long>(s->L.scratch), s->stream));
+    if (need) CU(cudaMemcpyAsync(host, s->ws + s->L.scratch, need * 8, cudaMemcpyDeviceToHost, s->stream));
+    CU(cudaStreamSynchronize(s->stream));
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_read_registers(gs_sim* s, uint64_t* host, size_t nwords) {
+    if (gs_status st = check_sim(s, "gs_sim_read_registers")) return st;
+    const Program& p = *s->prog;
+    const size_t need = (size_t)p.n_reg * s->words;
+    if (!host && need) return fail(GS_ERR_ARG, "gs_sim_read_registers: NULL buffer");
+    if (nwords < need) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_read_registers: need n_reg * lanes/64 words");
+    CU(cudaSetDevice(s->opts.device));
+    const uint32_t bank = (uint32_t)(s->cycle & 1);     // the bank the next cycle reads = Q(cycle)
+    const uint8_t* src = s->state() + (uint64_t)(p.row_q0 + bank * p.n_reg) * s->stride;
+    if (need) CU(cudaMemcpyAsync(host, src, need * 8, cudaMemcpyDeviceToHost, s->stream));
+    CU(cudaStreamSynchronize(s->stream));
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_write_registers(gs_sim* s, const uint64_t* host, size_t nwords) {
+    if (gs_status st = check_sim(s, "gs_sim_write_registers")) return st;
+    const Program& p = *s->prog;
+    const size_t need = (size_t)p.n_reg * s->words;
+    if (!host && need) return fail(GS_ERR_ARG, "gs_sim_write_registers: NULL buffer");
+    if (nwords < need) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_write_registers: need n_reg * lanes/64 words");
+    CU(cudaSetDevice(s->opts.device));
+    const uint32_t bank = (uint32_t)(s->cycle & 1);
+    uint8_t* dst = s->state() + (uint64_t)(p.row_q0 + bank * p.n_reg) * s->stride;
+    if (need) CU(cudaMemcpyAsync(dst, host, need * 8, cudaMemcpyHostToDevice, s->stream));
+    CU(cudaStreamSynchronize(s->stream));
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_read_trace(gs_sim* s, uint64_t* host, size_t nwords, uint32_t* cycles_recorded) {
+    if (gs_status st = check_sim(s, "gs_sim_read_trace")) return st;
+    const Program& p = *s->prog;
+    const uint64_t rec = s->cycle < s->opts.trace_cycles ? s->cycle : s->opts.trace_cycles;
+    const size_t need = (size_t)rec * p.n_po * s->opts.n_trace_words;
+    if (!host && need) return fail(GS_ERR_ARG, "gs_sim_read_trace: NULL buffer");
+    if (nwords < need) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_read_trace: buffer too small");
+    CU(cudaSetDevice(s->opts.device));
+    if (need) CU(cudaMemcpyAsync(host, s->ws + s->L.trace, need * 8, cudaMemcpyDeviceToHost, s->stream));
+    CU(cudaStreamSynchronize(s->stream));
+    if (cycles_recorded) *cycles_recorded = (uint32_t)rec;
+    clear_error();
+    return GS_OK;
+}
+
+static gs_status compute_lane_sigs(gs_sim* s) {
+    CU(cudaMemsetAsync(s->ws + s->L.ctl + offsetof(Ctl, sig_sum), 0, 8, s->stream));
+    CU(launch_lane_sigs(s->ctl(), s->at<const unsigned long long>(s->L.misr), s->words, s->opts.lane_offset,
+                        s->at<unsigned long long>(s->L.lane_sigs), s->stream));
+    return GS_OK;
+}
+
+gs_status gs_sim_read_lane_signatures(gs_sim* s, uint64_t* host, size_t nlanes) {
+    if (gs_status st = check_sim(s, "gs_sim_read_lane_signatures")) return st;
+    if (!host) return fail(GS_ERR_ARG, "gs_sim_read_lane_signatures: NULL buffer");
+    if (nlanes < s->opts.lanes) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_read_lane_signatures: need `lanes` entries");
+    CU(cudaSetDevice(s->opts.device));
+    if (gs_status st = compute_lane_sigs(s)) return st;
+    CU(cudaMemcpyAsync(host, s->ws + s->L.lane_sigs, (size_t)s->opts.lanes * 8, cudaMemcpyDeviceToHost, s->stream));
+    CU(cudaStreamSynchronize(s->stream));
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_read_signature(gs_sim* s, gs_signature* out) {
+    if (gs_status st = check_sim(s, "gs_sim_read_signature")) return st;
+    if (!out) return fail(GS_ERR_ARG, "gs_sim_read_signature: NULL out");
+    CU(cudaSetDevice(s->opts.device));
+    if (gs_status st = compute_lane_sigs(s)) return st;
+    Ctl h{};
+    CU(cudaMemcpyAsync(&h, s->ctl(), sizeof(Ctl), cudaMemcpyDeviceToHost, s->stream));
+    CU(cudaStreamSynchronize(s->stream));
+    out->lane_sig_sum = h.sig_sum;
+    out->out_popcount = h.popcount;
+    out->ab_mismatch = h.ab_mismatch;
+    out->invariant_violations = h.violations;
+    out->cycles = h.cycle;
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_launches_per_cycle(const gs_sim* s, uint64_t* launches) {
+    if (!s || !launches) return fail(GS_ERR_ARG, "gs_sim_launches_per_cycle: NULL argument");
+    const Program& p = *s->prog;
+    uint64_t lv = 0;
+    for (uint32_t l = 0; l < p.n_levels; ++l)
+        if (p.level_off[l + 1] > p.level_off[l]) lv++;
+    const uint64_t per_level = s->opts.kernel == GS_KERNEL_AB ? 2 : 1;
+    *launches = (p.n_pi ? 1 : 0) + lv * per_level + 1;
+    return GS_OK;
+}
+
+gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
+    if (gs_status st = check_sim(s, "gs_sim_profile_step")) return st;
+    if (!out) return fail(GS_ERR_ARG, "gs_sim_profile_step: NULL out");
+    if (!s->bound) return fail(GS_ERR_STATE, "gs_sim_profile_step: no stimulus bound");
+    if (s->bound == 2 && s->cycle + n > s->bound_base + s->bound_cycles)
+        return fail(GS_ERR_STATE, "gs_sim_profile_step: stepping past the bound stimulus cycles");
+    const Program& p = *s->prog;
+    CU(cudaSetDevice(s->opts.device));
+    std::vector<cudaEvent_t> evs(2 * (size_t)p.n_levels);
+    cudaEvent_t e0, e1;
+    for (auto& e : evs) CU(cudaEventCreate(&e));
+    CU(cudaEventCreate(&e0));
+    CU(cudaEventCreate(&e1));
+    double level_ms = 0, total_ms = 0, level_bytes = 0;
+    uint64_t lvl_launches = 0, launches = 0, per = 0;
+    gs_sim_launches_per_cycle(s, &per);
+    // algorithmic bytes of one level launch: every gate reads k input rows, writes its
+    // output row, plus the fused latch store
+    std::vector<double> lb(p.n_levels, 0.0);
+    for (uint32_t l = 0; l < p.n_levels; ++l)
+        for (uint32_t g = p.level_off[l]; g < p.level_off[l + 1]; ++g)
+            lb[l] += (double)(p.aux[g].k + 1 + (p.aux[g].qdst != NONE32 ? 1 : 0)) * (double)s->stride;
+    gs_status rc = GS_OK;
+    for (uint32_t i = 0; i < n && rc == GS_OK; ++i) {
+        const uint32_t parity = (uint32_t)(s->cycle & 1);
+        cudaEventRecord(e0, s->stream);
+        cudaError_t e = cycle_launches(s, parity, s->stream, &evs);
+        cudaEventRecord(e1, s->stream);
+        if (e != cudaSuccess) { rc = fail(GS_ERR_CUDA, cudaGetErrorString(e)); break; }
+        s->cycle++;
+        e = cudaEventSynchronize(e1);
+        if (e != cudaSuccess) { rc = fail(GS_ERR_CUDA, cudaGetErrorString(e)); break; }
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e0, e1);
+        total_ms += ms;
+        for (uint32_t l = 0; l < p.n_levels; ++l) {
+            if (p.level_off[l + 1] == p.level_off[l]) continue;
+            cudaEventElapsedTime(&ms, evs[2 * l], evs[2 * l + 1]);
+            level_ms += ms;
+            level_bytes += lb[l];
+            lvl_launches++;
+        }
+        launches += per;
+    }
+    for (auto& e : evs) cudaEventDestroy(e);
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    if (rc != GS_OK) return rc;
+    out->level_ms = level_ms;
+    out->total_ms = total_ms;
+    out->level_launches = lvl_launches;
+    out->total_launches = launches;
+    out->level_bytes = level_bytes;
+    clear_error();
+    return GS_OK;
+}
+
+}  // extern "C"

@@ -47,3 +47,29 @@ def bits_to_int(bits):
     for i in range(bits.shape[-1]):
         acc = acc + (bits[..., i].astype(object) << i)
     return acc
+
+
+def mix64_np(z):
+    z = np.asarray(z, dtype=np.uint64)
+    with np.errstate(over="ignore"):
+        z = z + np.uint64(0x9E3779B97F4A7C15)
+        z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+        z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+    return z ^ (z >> np.uint64(31))
+
+
+def stim_words_np(seed, p, c, words):
+    """Vectorised H(seed, p, c, w) over an array of global word indices (reading R2)."""
+    a = mix64_np(np.uint64(seed) ^ np.uint64(p))
+    b = mix64_np(a ^ np.uint64(c))
+    return mix64_np(b ^ np.asarray(words, dtype=np.uint64))
+
+
+def pi_lanes_np(seed, n_pi, cycle, n_lanes, lane_offset=0):
+    """PI bits [n_pi][n_lanes] for consecutive lanes starting at lane_offset (multiple of 64)."""
+    words = np.arange(lane_offset // 64, lane_offset // 64 + n_lanes // 64, dtype=np.uint64)
+    out = np.empty((n_pi, n_lanes), dtype=np.uint8)
+    for p in range(n_pi):
+        w = stim_words_np(seed, p, cycle, words)
+        out[p] = np.unpackbits(w.view(np.uint8), bitorder="little")
+    return out

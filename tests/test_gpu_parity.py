@@ -1,0 +1,303 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the CPU oracle, bit-exact.
+
+Every comparison is element by element on the same seeded inputs; the oracle never
+sees anything the GPU produced.  Closed forms (a+b, a*b, LFSR, counters) are checked
+on ALL lanes where the oracle would be too slow.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import workloads
+from workloads import netlists as W
+import paper_conf_ipps_gavierrprs23_b200 as gs
+from tests import _ref
+from tests._build import ensure_built
+
+pytestmark = pytest.mark.gpu
+ensure_built()
+
+
+def compile_nl(nl, balance=True):
+    return gs.Netlist.from_arrays(nl).compile(balance=balance)
+
+
+def gpu_trace_bits(tr, words_sel):
+    """GPU trace [cycles][po][ntw] -> bits [lanes_of_traced_words][cycles][po]."""
+    bits = gs.unpack_lanes(tr)                         # [c][po][ntw*64]
+    return np.transpose(bits, (2, 0, 1))
+
+
+def run_gpu(nl, lanes, cycles, kernel="lut", seed=None, host_stim=None, trace_words=(),
+            lane_offset=0, balance=True, use_graphs=True, prog=None):
+    prog = prog or compile_nl(nl, balance)
+    sim = gs.Sim(prog, lanes, lane_offset=lane_offset, kernel=kernel, trace_words=trace_words,
+                 trace_cycles=cycles if len(trace_words) else 0, use_graphs=use_graphs)
+    if host_stim is not None:
+        sim.bind_host(host_stim)
+    else:
+        sim.bind_generated(seed)
+    sim.step(cycles)
+    sim.sync()
+    out = dict(outputs=sim.read_outputs(), regs=sim.read_registers(),
+               sigs=sim.read_lane_signatures(), signature=sim.signature())
+    if len(trace_words):
+        out["trace"] = sim.read_trace()
+    sim.close()
+    return out
+
+
+def lane_bits(words_2d, lanes_idx):
+    """[rows][W] words -> [len(lanes_idx)][rows] bits for the given local lanes."""
+    b = gs.unpack_lanes(words_2d)
+    return b[:, lanes_idx].T
+
+
+KERNELS = ["lut", "poly", "ab"]
+
+
+# ------------------------------------------------------------------ C1: adder
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_c1_adder_generated_equals_a_plus_b_and_oracle(kernel):
+    cfg = workloads.CONFIGS["C1"]
+    nl = cfg.netlist()
+    r = run_gpu(nl, cfg.lanes, 1, kernel, seed=cfg.stim_seed, trace_words=range(cfg.lanes // 64))
+    lanes = np.arange(cfg.lanes)
+    got = lane_bits(r["outputs"], lanes)                                # [lanes][9]
+    pi = _ref.pi_lanes_np(cfg.stim_seed, 16, 0, cfg.lanes).astype(np.int64)
+    a = (pi[:8] << np.arange(8)[:, None]).sum(0)
+    b = (pi[8:] << np.arange(8)[:, None]).sum(0)
+    assert np.array_equal((got.astype(np.int64) << np.arange(9)).sum(1), a + b)
+    o = oracle.simulate(nl, lanes, 1, seed=cfg.stim_seed)
+    assert np.array_equal(got, o["last"])
+    assert np.array_equal(gpu_trace_bits(r["trace"], None), o["trace"])
+    assert np.array_equal(r["sigs"], o["sig"])
+    assert r["signature"]["lane_sig_sum"] == oracle.lane_sig_sum(o["sig"], lanes)
+    assert r["signature"]["ab_mismatch"] == 0 and r["signature"]["invariant_violations"] == 0
+    assert r["signature"]["out_popcount"] == int(o["trace"].sum())
+
+
+def test_c1_adder_exhaustive_host_stimulus():
+    nl = workloads.adder(8)
+    lanes = 1 << 16
+    s = np.arange(lanes, dtype=np.uint64)
+    stim = np.zeros((1, 16, lanes // 64), dtype=np.uint64)
+    for p in range(16):
+        bits = ((s >> np.uint64(p)) & np.uint64(1)).astype(np.uint8)
+        stim[0, p] = np.packbits(bits, bitorder="little").view(np.uint64)
+    for kernel in KERNELS:
+        r = run_gpu(nl, lanes, 1, kernel, host_stim=stim)
+        got = lane_bits(r["outputs"], np.arange(lanes)).astype(np.int64)
+        assert np.array_equal((got << np.arange(9)).sum(1), ((s & np.uint64(0xFF)) + (s >> np.uint64(8))).astype(np.int64))
+        assert r["signature"]["ab_mismatch"] == 0
+
+
+# ------------------------------------------------------------------ tiny brute force
+@pytest.mark.parametrize("seed", range(10))
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_tiny_random_netlists_all_lanes_all_cycles(seed, kernel):
+    nl = workloads.random_tiny(seed, n_pi=5, n_reg=4, n_gates=40, n_po=7, max_k=4 if seed % 3 else 6)
+    lanes, cycles = 256, 7
+    stim = workloads.random_host_stimulus(1000 + seed, cycles, nl.n_pi, lanes // 64)
+    r = run_gpu(nl, lanes, cycles, kernel, host_stim=stim, trace_words=range(lanes // 64),
+                use_graphs=bool(seed % 2))
+    o = oracle.simulate(nl, np.arange(lanes), cycles, host_stim=stim)
+    assert np.array_equal(gpu_trace_bits(r["trace"], None), o["trace"])
+    assert np.array_equal(lane_bits(r["regs"], np.arange(lanes)), o["regs"])
+    assert np.array_equal(lane_bits(r["outputs"], np.arange(lanes)), o["last"])
+    assert np.array_equal(r["sigs"], o["sig"])
+    assert r["signature"]["ab_mismatch"] == 0 and r["signature"]["invariant_violations"] == 0
+
+
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_register_edge_cases_and_probes(kernel):
+    for nl in (workloads.register_edge_cases(), workloads.probes_circuit()):
+        lanes, cycles = 192, 300            # 3 words: exercises the 8-byte vector path
+        r = run_gpu(nl, lanes, cycles, kernel, seed=77, trace_words=range(3))
+        o = oracle.simulate(nl, np.arange(lanes), cycles, seed=77)
+        assert np.array_equal(gpu_trace_bits(r["trace"], None), o["trace"])
+        assert np.array_equal(lane_bits(r["regs"], np.arange(lanes)), o["regs"])
+        assert np.array_equal(r["sigs"], o["sig"])
+
+
+# ------------------------------------------------------------------ C2: multiplier
+def test_c2_multiplier_all_lanes_equal_a_times_b():
+    cfg = workloads.CONFIGS["C2"]
+    nl = cfg.netlist()
+    r = run_gpu(nl, cfg.lanes, 1, "lut", seed=cfg.stim_seed)
+    bits = gs.unpack_lanes(r["outputs"]).astype(np.uint64)             # [64][lanes]
+    prod = np.zeros(cfg.lanes, dtype=np.uint64)
+    for o in range(64):
+        prod |= bits[o] << np.uint64(o)
+    pi = _ref.pi_lanes_np(cfg.stim_seed, 64, 0, cfg.lanes).astype(np.uint64)
+    a = np.zeros(cfg.lanes, dtype=np.uint64)
+    b = np.zeros(cfg.lanes, dtype=np.uint64)
+    for i in range(32):
+        a |= pi[i] << np.uint64(i)
+        b |= pi[32 + i] << np.uint64(i)
+    with np.errstate(over="ignore"):
+        assert np.array_equal(prod, a * b)
+    sample = np.concatenate([np.arange(0, 128), np.arange(cfg.lanes - 128, cfg.lanes),
+                             np.random.default_rng(0).integers(0, cfg.lanes, 1792)])
+    o = oracle.simulate(nl, sample, 1, seed=cfg.stim_seed, want=("last",))
+    assert np.array_equal(lane_bits(r["outputs"], sample), o["last"])
+
+
+def test_c2_kernels_agree():
+    cfg = workloads.CONFIGS["C2"]
+    r = run_gpu(cfg.netlist(), 1 << 16, 1, "ab", seed=cfg.stim_seed)
+    assert r["signature"]["ab_mismatch"] == 0 and r["signature"]["invariant_violations"] == 0
+
+
+# ------------------------------------------------------------------ sequential synthetic
+def probe_closed_forms(nl, outputs_bits, last_cycle, seed, n_lanes, lane_offset=0):
+    """LFSR16 / 8-bit counter / enabled 6-bit counter at the last cycle, all lanes."""
+    pp = nl.meta["probe_po"]
+    lf = outputs_bits[:, pp["lfsr16"][0]:pp["lfsr16"][1]]
+    s = [1] + [0] * 15
+    for _ in range(last_cycle):
+        s = [s[15] ^ s[14] ^ s[12] ^ s[3]] + s[:15]
+    assert (lf == np.array(s, dtype=np.uint8)[None, :]).all()
+    c8 = (outputs_bits[:, 16:24].astype(np.int64) << np.arange(8)).sum(1)
+    assert (c8 == last_cycle % 256).all()
+    en = np.zeros(n_lanes, dtype=np.int64)
+    for c in range(last_cycle):
+        en += _ref.pi_lanes_np(seed, 1, c, n_lanes, lane_offset)[0]
+    c6 = (outputs_bits[:, 24:30].astype(np.int64) << np.arange(6)).sum(1)
+    assert (c6 == en % 64).all()
+
+
+def sampled_lane_check(nl, r, sample_local, lane_offset, cycles, seed, trace_words):
+    o = oracle.simulate(nl, sample_local + lane_offset, cycles, seed=seed)
+    tb = gpu_trace_bits(r["trace"], None)                  # [ntw*64][c][po]
+    pos = {w: i for i, w in enumerate(trace_words)}
+    rows = np.array([pos[s // 64] * 64 + s % 64 for s in sample_local])
+    assert np.array_equal(tb[rows], o["trace"])
+    assert np.array_equal(lane_bits(r["regs"], sample_local), o["regs"])
+    assert np.array_equal(r["sigs"][sample_local], o["sig"])
+
+
+def test_c3_full_config_sampled_lanes_and_probes():
+    cfg = workloads.CONFIGS["C3"]
+    nl = cfg.netlist()
+    W_ = cfg.lanes // 64
+    tw = [0, 1, W_ // 2, W_ - 1]
+    r = run_gpu(nl, cfg.lanes, cfg.cycles, "lut", seed=cfg.stim_seed, trace_words=tw)
+    sample = np.array([0, 1, 63, 64, 65, 127, W_ // 2 * 64 + 5, W_ // 2 * 64 + 40,
+                       cfg.lanes - 64, cfg.lanes - 2, cfg.lanes - 1])
+    sampled_lane_check(nl, r, sample, 0, cfg.cycles, cfg.stim_seed, tw)
+    probe_closed_forms(nl, gs.unpack_lanes(r["outputs"]).T, cfg.cycles - 1, cfg.stim_seed, cfg.lanes)
+    assert r["signature"]["cycles"] == cfg.cycles
+
+
+def test_c3_kernel_ab_cross_check_and_poly_parity():
+    cfg = workloads.CONFIGS["C3"]
+    nl = cfg.netlist()
+    prog = compile_nl(nl)
+    a = run_gpu(nl, 4096, 40, "ab", seed=cfg.stim_seed, prog=prog)
+    assert a["signature"]["ab_mismatch"] == 0 and a["signature"]["invariant_violations"] == 0
+    b = run_gpu(nl, 4096, 40, "poly", seed=cfg.stim_seed, prog=prog)
+    c = run_gpu(nl, 4096, 40, "lut", seed=cfg.stim_seed, prog=prog)
+    assert np.array_equal(b["sigs"], c["sigs"]) and np.array_equal(b["regs"], c["regs"])
+    assert b["signature"]["invariant_violations"] == 0
+
+
+def test_sharding_and_balance_invariance():
+    """lane_sig_sum of P shards (global lane offsets) == 1 shard; levels do not matter."""
+    cfg = workloads.CONFIGS["C3"]
+    nl = cfg.netlist()
+    prog = compile_nl(nl)
+    full = run_gpu(nl, 8192, 60, "lut", seed=9, prog=prog)
+    tot = 0
+    for sh in range(4):
+        part = run_gpu(nl, 2048, 60, "lut", seed=9, lane_offset=sh * 2048, prog=prog)
+        assert np.array_equal(part["sigs"], full["sigs"][sh * 2048:(sh + 1) * 2048])
+        tot = (tot + part["signature"]["lane_sig_sum"]) % (1 << 64)
+    assert tot == full["signature"]["lane_sig_sum"]
+    unbal = run_gpu(nl, 8192, 60, "lut", seed=9, balance=False)
+    assert np.array_equal(unbal["sigs"], full["sigs"])
+
+
+def test_step_granularity_graphs_and_resume():
+    nl = workloads.synthetic(20000, 800, 32, 48, 24, seed=12, name="s")
+    prog = compile_nl(nl)
+    ref = run_gpu(nl, 2048, 50, "lut", seed=3, prog=prog)
+    sim = gs.Sim(prog, 2048, use_graphs=False)
+    sim.bind_generated(3)
+    for _ in range(20):
+        sim.step(1)
+    regs = sim.read_registers()
+    sim.step(30)
+    assert np.array_equal(sim.read_registers(), ref["regs"])
+    assert np.array_equal(sim.read_lane_signatures(), ref["sigs"])
+    sim.close()
+    # resume: a fresh sim whose own history diverged (zeroed registers), restored from
+    # the checkpoint (registers at cycle 20) -> identical registers and outputs after
+    sim2 = gs.Sim(prog, 2048)
+    sim2.bind_generated(3)
+    sim2.write_registers(np.zeros_like(regs))
+    sim2.step(20)
+    sim2.write_registers(regs)
+    sim2.step(30)
+    assert np.array_equal(sim2.read_registers(), ref["regs"])
+    assert np.array_equal(sim2.read_outputs(), ref["outputs"])
+    sim2.reset()
+    sim2.step(50)
+    assert np.array_equal(sim2.read_lane_signatures(), ref["sigs"])
+    sim2.close()
+
+
+def test_negative_flipped_truth_table_bit_is_detected():
+    nl = workloads.synthetic(5000, 200, 32, 48, 16, seed=10, name="s")
+    bad = workloads.Netlist(nl.n_pi, nl.reg_init, nl.reg_d, nl.gate_k, nl.gate_in_off, nl.gate_in,
+                            nl.gate_tt.copy(), nl.po, name="bad", meta=nl.meta)
+    g = int(np.nonzero(nl.gate_k == 3)[0][-1])
+    bad.gate_tt[g] ^= np.uint64(1 << 5)
+    r = run_gpu(bad, 1024, 20, "lut", seed=5)
+    o = oracle.simulate(nl, np.arange(1024), 20, seed=5)
+    assert not np.array_equal(r["sigs"], o["sig"])
+
+
+def test_errors_on_device():
+    prog = compile_nl(workloads.adder(8))
+    sim = gs.Sim(prog, 128)
+    with pytest.raises(gs.GsError) as e:
+        sim.step(1)
+    assert e.value.code == gs.GS_ERR_STATE
+    sim.bind_host(np.zeros((2, 16, 2), dtype=np.uint64))
+    sim.step(2)
+    with pytest.raises(gs.GsError) as e:
+        sim.step(1)
+    assert e.value.code == gs.GS_ERR_STATE
+    with pytest.raises(gs.GsError) as e:
+        gs._call("gs_sim_read_outputs", sim.h, np.zeros(4, np.uint64).ctypes.data_as(gs.C.c_void_p), 4)
+    assert e.value.code == gs.GS_ERR_BUFFER_TOO_SMALL
+    sim.close()
+
+
+# ------------------------------------------------------------------ full-size configs
+@pytest.mark.slow
+def test_c4_full_config_sampled_lanes_and_probes():
+    cfg = workloads.CONFIGS["C4"]
+    nl = cfg.netlist()
+    W_ = cfg.lanes // 64
+    tw = [0, 1, W_ // 2, W_ - 1]
+    r = run_gpu(nl, cfg.lanes, cfg.cycles, "lut", seed=cfg.stim_seed, trace_words=tw)
+    sample = np.array([0, 63, 64, 127, W_ // 2 * 64 + 17, cfg.lanes - 64, cfg.lanes - 1])
+    sampled_lane_check(nl, r, sample, 0, cfg.cycles, cfg.stim_seed, tw)
+    probe_closed_forms(nl, gs.unpack_lanes(r["outputs"]).T, cfg.cycles - 1, cfg.stim_seed, cfg.lanes)
+
+
+@pytest.mark.slow
+def test_c5_shard_full_netlist_sampled_lanes():
+    cfg = workloads.CONFIGS["C5"]
+    nl = cfg.netlist()
+    lanes = cfg.lanes // cfg.shards
+    shard = 5
+    off = shard * lanes
+    W_ = lanes // 64
+    tw = [0, W_ - 1]
+    r = run_gpu(nl, lanes, cfg.cycles, "lut", seed=cfg.stim_seed, trace_words=tw, lane_offset=off)
+    sample = np.array([0, 1, 63, lanes - 64, lanes - 1])
+    sampled_lane_check(nl, r, sample, off, cfg.cycles, cfg.stim_seed, tw)
+    probe_closed_forms(nl, gs.unpack_lanes(r["outputs"]).T, cfg.cycles - 1, cfg.stim_seed, lanes, off)

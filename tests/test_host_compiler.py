@@ -1,0 +1,213 @@
+"""Host-side logic of libgsim.so (CPU only): ABI exports, netlist validation, levelizer,
+balancing and the Möbius coefficient compiler — checked against the oracle / definitions."""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads
+from workloads import netlists as W
+import paper_conf_ipps_gavierrprs23_b200 as gs
+from tests._build import ensure_built
+
+ensure_built()
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_library_exports_every_header_symbol():
+    hdr = open(os.path.join(ROOT, "include", "gsim.h")).read()
+    declared = set(re.findall(r"^(?:gs_status|const char\*)\s+(gs_\w+)\s*\(", hdr, re.M))
+    assert len(declared) >= 35
+    lib = gs.lib()
+    for name in declared:
+        assert hasattr(lib, name), name
+    assert declared == set(gs.EXPORTED)
+    assert gs.version() == "0.1.0"
+
+
+def _compile(nl, balance=True):
+    return gs.Netlist.from_arrays(nl).compile(balance=balance)
+
+
+def test_mobius_all_4input_functions_match_definition():
+    b = W.Builder()
+    x = [b.pi() for _ in range(4)]
+    for tt in range(1 << 16):
+        b.gate(tt, *x)
+    b.out(("gate", 0))
+    prog = _compile(b.build("all4"))
+    for tt in range(1 << 16):
+        assert prog.coeffs(tt, 4) == oracle.mobius_def(tt, 4), tt
+
+
+@pytest.mark.parametrize("k", [0, 1, 2, 3, 5, 6])
+def test_mobius_other_arities_match_definition(k):
+    rng = np.random.default_rng(k)
+    b = W.Builder()
+    x = [b.pi() for _ in range(max(k, 1))]
+    tts = [int(t) for t in rng.integers(0, 2 ** min(1 << k, 62), size=200)]
+    if k == 6:
+        tts += [(1 << 64) - 1, 0x8000000000000000, 0x6996966996696996]
+    for tt in tts:
+        b.gate(tt, *x[:k])
+    b.out(("gate", 0))
+    prog = _compile(b.build("ar"))
+    for g, tt in enumerate(tts):
+        assert prog.coeffs(g, k) == oracle.mobius_def(tt, k)
+
+
+def _alap(nl, asap, depth):
+    G = nl.n_gates
+    base = nl.n_pi + nl.n_reg
+    alap = np.full(G, depth, dtype=np.int64)
+    order = oracle.topo_order(nl)
+    for g in order[::-1]:
+        if nl.gate_k[g] == 0:
+            continue
+        for x in nl.inputs_of(int(g)):
+            if x >= base and nl.gate_k[x - base] > 0:
+                alap[x - base] = min(alap[x - base], alap[g] - 1)
+    return alap
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C3"])
+def test_levelizer_asap_and_balanced(name):
+    nl = workloads.build_netlist(name)
+    asap = oracle.asap_levels(nl).astype(np.int64)
+    depth = int(asap.max())
+    p0 = _compile(nl, balance=False)
+    assert p0.info["n_levels"] == depth                        # merged layers = depth
+    assert np.array_equal(p0.gate_levels().astype(np.int64), asap)
+    p1 = _compile(nl, balance=True)
+    lv = p1.gate_levels().astype(np.int64)
+    assert p1.info["n_levels"] == depth
+    alap = _alap(nl, asap, depth)
+    ev = nl.gate_k > 0
+    assert (lv[ev] >= asap[ev]).all() and (lv[ev] <= alap[ev]).all()
+    base = nl.n_pi + nl.n_reg
+    for g in np.nonzero(ev)[0][:: max(1, nl.n_gates // 20000)]:
+        for x in nl.inputs_of(int(g)):
+            if x >= base and nl.gate_k[x - base] > 0:
+                assert lv[g] > lv[x - base]
+    w0, w1 = p0.level_widths(), p1.level_widths()
+    assert w0.sum() == w1.sum() == int(ev.sum())
+    assert w1.max() <= w0.max()
+    assert np.array_equal(np.bincount(lv[ev], minlength=depth + 1)[1:], w1)
+
+
+def test_balancing_flattens_synthetic_widths():
+    nl = workloads.build_netlist("C3")
+    w0 = _compile(nl, False).level_widths()
+    w1 = _compile(nl, True).level_widths()
+    assert np.std(w1) < 0.5 * np.std(w0)
+
+
+def test_program_info_counts():
+    nl = workloads.synthetic(4000, 100, 16, 40, 12, seed=1, name="s")
+    p = _compile(nl)
+    inf = p.info
+    k = nl.gate_k.astype(np.int64)
+    assert inf["n_gates"] == nl.n_gates and inf["n_eval_gates"] == int((k > 0).sum())
+    assert inf["k_hist"][:5] == np.bincount(k, minlength=7)[:5].tolist()
+    assert inf["hidden_neurons"] == int((1 << k[k > 0]).sum())          # sum 2^k
+    assert inf["n_edges"] == int(k.sum())
+    nnz = sum(sum(1 for w in oracle.mobius_def(int(t), int(kk)) if w) for t, kk in zip(nl.gate_tt, k))
+    assert inf["nnz_coeffs"] == nnz
+    assert inf["n_rows"] == 2 + nl.n_pi + 2 * nl.n_reg + inf["n_eval_gates"]
+
+
+def test_incremental_equals_bulk_load():
+    nl = workloads.register_edge_cases()
+    bulk = _compile(nl)
+    n = gs.Netlist()
+    pis = [n.add_input() for _ in range(nl.n_pi)]
+    qs = [n.add_register(int(i)) for i in nl.reg_init]
+    base = nl.n_pi + nl.n_reg
+    ids = pis + qs
+    # gates are created in netlist order; constants via gs_add_const
+    for g in range(nl.n_gates):
+        k = int(nl.gate_k[g])
+        if k == 0:
+            ids.append(n.add_const(int(nl.gate_tt[g])))
+        else:
+            ids.append(n.add_gate([ids[x] for x in nl.inputs_of(g)], int(nl.gate_tt[g])))
+    for r, d in enumerate(nl.reg_d):
+        n.set_register_d(qs[r], ids[int(d)])
+    for o in nl.po:
+        n.mark_output(ids[int(o)])
+    assert n.counts()["n_gates"] == nl.n_gates and base == len(pis) + len(qs)
+    inc = n.compile()
+    assert inc.info["program_hash"] == bulk.info["program_hash"]
+
+
+def test_errors():
+    # combinational loop
+    b = W.Builder()
+    p = b.pi()
+    b.gates.append(([("gate", 1), p], W.AND2))
+    b.gates.append(([("gate", 0), p], W.OR2))
+    b.out(("gate", 0))
+    with pytest.raises(gs.GsError) as e:
+        _compile(b.build())
+    assert e.value.code == gs.GS_ERR_COMB_LOOP
+    # undriven register
+    n = gs.Netlist()
+    n.add_register(0)
+    with pytest.raises(gs.GsError) as e:
+        n.compile()
+    assert e.value.code == gs.GS_ERR_UNDRIVEN
+    # arity
+    n = gs.Netlist()
+    x = [n.add_input() for _ in range(7)]
+    with pytest.raises(gs.GsError) as e:
+        n.add_gate(x, 1)
+    assert e.value.code == gs.GS_ERR_ARITY
+    n.add_gate(x[:5], 1)
+    with pytest.raises(gs.GsError) as e:
+        n.compile(max_k=4)
+    assert e.value.code == gs.GS_ERR_ARITY
+    # truth table wider than 2^k
+    with pytest.raises(gs.GsError) as e:
+        n.add_gate(x[:2], 0x1F)
+    assert e.value.code == gs.GS_ERR_ARG
+    # bulk load into a non-empty netlist
+    with pytest.raises(gs.GsError) as e:
+        gs.Netlist.from_arrays(workloads.adder(2)).__class__.from_arrays  # noqa: B018
+        m = gs.Netlist()
+        m.add_input()
+        nl = workloads.adder(2)
+        keep = [np.ascontiguousarray(a) for a in (nl.reg_init, nl.reg_d, nl.gate_k, nl.gate_in_off,
+                                                  nl.gate_in, nl.gate_tt, nl.po)]
+        a = gs.gs_netlist_arrays(nl.n_pi, nl.n_reg, nl.n_gates, nl.n_po,
+                                 *[k.ctypes.data_as(gs.C.c_void_p) for k in keep])
+        gs._call("gs_netlist_load_arrays", m.h, gs.C.byref(a))
+    assert e.value.code == gs.GS_ERR_STATE
+    # bad net id in a bulk load
+    nl = workloads.adder(2)
+    nl.gate_in = nl.gate_in.copy()
+    nl.gate_in[0] = 10_000
+    with pytest.raises(gs.GsError) as e:
+        gs.Netlist.from_arrays(nl)
+    assert e.value.code == gs.GS_ERR_ARG
+    assert "out of range" in gs.lib().gs_last_error().decode()
+
+
+def test_workspace_size_is_host_computable():
+    p = _compile(workloads.build_netlist("C3"))
+    o = gs.gs_sim_opts(0, None, 16384, 0, 1, 0, None, 0, 1)
+    n = gs.C.c_size_t()
+    gs._call("gs_sim_workspace_bytes", p.h, gs.C.byref(o), gs.C.byref(n))
+    state = p.info["n_rows"] * 16384 // 8
+    assert state <= n.value < state + 64 * 1024 * 1024
+    o.lanes = 100
+    with pytest.raises(gs.GsError):
+        gs._call("gs_sim_workspace_bytes", p.h, gs.C.byref(o), gs.C.byref(n))
+
+
+def test_permuted_netlist_same_asap_widths():
+    nl = workloads.synthetic(3000, 120, 16, 40, 12, seed=9, name="s")
+    a = _compile(nl, balance=False).level_widths()
+    b = _compile(nl.permuted(3), balance=False).level_widths()
+    assert np.array_equal(a, b)
