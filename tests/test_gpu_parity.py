@@ -248,14 +248,22 @@ def test_step_granularity_graphs_and_resume():
 
 
 def test_negative_flipped_truth_table_bit_is_detected():
+    """Tests the tests: one flipped truth-table bit in an observed gate must be caught."""
     nl = workloads.synthetic(5000, 200, 32, 48, 16, seed=10, name="s")
+    base = nl.n_pi + nl.n_reg
+    g = int(nl.po[40]) - base                       # a gate that drives a primary output
+    assert g >= 0 and nl.gate_k[g] >= 2
     bad = workloads.Netlist(nl.n_pi, nl.reg_init, nl.reg_d, nl.gate_k, nl.gate_in_off, nl.gate_in,
                             nl.gate_tt.copy(), nl.po, name="bad", meta=nl.meta)
-    g = int(np.nonzero(nl.gate_k == 3)[0][-1])
-    bad.gate_tt[g] ^= np.uint64(1 << 5)
-    r = run_gpu(bad, 1024, 20, "lut", seed=5)
-    o = oracle.simulate(nl, np.arange(1024), 20, seed=5)
+    bad.gate_tt[g] ^= np.uint64(1)                  # f(0,..,0) flipped
+    lanes = np.arange(1024)
+    r = run_gpu(bad, 1024, 20, "lut", seed=5, trace_words=range(16))
+    o = oracle.simulate(nl, lanes, 20, seed=5)
+    assert not np.array_equal(gpu_trace_bits(r["trace"], None), o["trace"])
     assert not np.array_equal(r["sigs"], o["sig"])
+    # and the flipped design agrees with the oracle run on the same flipped design
+    ob = oracle.simulate(bad, lanes, 20, seed=5)
+    assert np.array_equal(r["sigs"], ob["sig"])
 
 
 def test_errors_on_device():
