@@ -44,6 +44,8 @@ def parse():
     ap.add_argument("--cycles-per-step", type=int, default=100)
     ap.add_argument("--lanes", type=int, default=0, help="override lanes per GPU")
     ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab"])
+    ap.add_argument("--lane-slabs", type=int, default=0, help="L2 lane slabs (0 = library default)")
+    ap.add_argument("--lut-unroll", type=int, default=0, help="vectors per thread (0 = auto)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-roofline", action="store_true")
@@ -205,7 +207,8 @@ def main():
     if world > 1:
         gdist.check_same_program(info["program_hash"])
     stream = torch.cuda.Stream(device=local)
-    sim = gs.Sim(prog, lanes, lane_offset=lane_offset, kernel=args.kernel, device=local, stream=stream)
+    sim = gs.Sim(prog, lanes, lane_offset=lane_offset, kernel=args.kernel, device=local, stream=stream,
+                 lane_slabs=args.lane_slabs, lut_unroll=args.lut_unroll)
     sim.bind_generated(cfg.stim_seed)
     C = args.cycles_per_step
     launches_per_cycle = sim.launches_per_cycle()
@@ -299,6 +302,7 @@ def main():
             "config": {"workload": f"{cfg.name}: {cfg.label}", "gates": G, "registers": info["n_reg"],
                        "levels": info["n_levels"], "lanes_per_gpu": lanes, "lanes_total": lanes * world,
                        "cycles_per_step": C, "kernel": args.kernel, "balance": True,
+                       "lane_slabs": args.lane_slabs, "lut_unroll": args.lut_unroll,
                        "l2": "inputs larger than L2 (state %.1f GB per GPU)" % (info["n_rows"] * lanes / 8 / 1e9),
                        "parallelism": f"dp{world} (stimulus sharding)", "compile_s": round(compile_s, 2),
                        "paper_style_gcps": value * (G + info["n_reg"]) / G},

@@ -189,6 +189,10 @@ typedef struct {
     const uint32_t* trace_words;  /* [n_trace_words] local word indices (copied)           */
     uint32_t trace_cycles;        /* capacity of the trace, in cycles                      */
     int use_graphs;               /* 1: replay each cycle as a CUDA graph (default)        */
+    uint32_t lane_slabs;          /* kernel A: run all levels on 1/lane_slabs of the lanes at a
+                                     time so recent levels stay L2-resident (0/1 = off); needs
+                                     (lanes/128) % lane_slabs == 0 and slabs >= 4096 lanes   */
+    uint32_t lut_unroll;          /* kernel A: max 16-byte vectors per thread (0 = auto)   */
 } gs_sim_opts;
 
 /* Device workspace bytes required for (prog, opts). */

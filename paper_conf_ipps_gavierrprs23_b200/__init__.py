@@ -68,7 +68,8 @@ class gs_program_info(C.Structure):
 class gs_sim_opts(C.Structure):
     _fields_ = [("device", C.c_int), ("stream", C.c_void_p), ("lanes", C.c_uint64),
                 ("lane_offset", C.c_uint64), ("kernel", C.c_int), ("n_trace_words", C.c_uint32),
-                ("trace_words", C.c_void_p), ("trace_cycles", C.c_uint32), ("use_graphs", C.c_int)]
+                ("trace_words", C.c_void_p), ("trace_cycles", C.c_uint32), ("use_graphs", C.c_int),
+                ("lane_slabs", C.c_uint32), ("lut_unroll", C.c_uint32)]
 
 
 class gs_signature(C.Structure):
@@ -264,7 +265,7 @@ class Sim:
 
     def __init__(self, program: Program, lanes: int, lane_offset: int = 0, kernel="lut",
                  device: int = 0, stream=None, trace_words=(), trace_cycles: int = 0,
-                 use_graphs: bool = True):
+                 use_graphs: bool = True, lane_slabs: int = 0, lut_unroll: int = 0):
         import torch
         self.program = program
         self.lanes, self.words = int(lanes), int(lanes) // 64
@@ -274,7 +275,7 @@ class Sim:
         o = gs_sim_opts(device, C.c_void_p(self.stream.cuda_stream), self.lanes, int(lane_offset),
                         KERNELS[kernel] if isinstance(kernel, str) else int(kernel), len(self._tw),
                         _p(self._tw) if len(self._tw) else None, int(trace_cycles),
-                        1 if use_graphs else 0)
+                        1 if use_graphs else 0, int(lane_slabs), int(lut_unroll))
         nbytes = C.c_size_t()
         _call("gs_sim_workspace_bytes", program.h, C.byref(o), C.byref(nbytes))
         self.workspace = torch.empty(int(nbytes.value) + 256, dtype=torch.uint8, device=self.device)

@@ -182,8 +182,90 @@ __global__ void __launch_bounds__(256) k_level_lut(LevelArgs a, uint32_t vpr, ui
     }
 }
 
+// Wide-row variant: every warp owns one gate and U x 32 consecutive 16-byte vectors of
+// it; all U*k input loads are issued before any is consumed (memory-level parallelism
+// U*k per thread, one descriptor fetch per U vectors).
+template <int K, int U>
+__device__ __forceinline__ void lut_gate_u(const LevelArgs& a, uint32_t gate, uint4 in, uint32_t v0,
+                                           uint64_t tt, uint32_t qdst) {
+    uint32_t r[6];
+    r[0] = in.x; r[1] = in.y; r[2] = in.z; r[3] = in.w;
+    if (K > 4) {
+        const uint2 hi = __ldg(a.dhi + gate);
+        r[4] = hi.x; r[5] = hi.y;
+    }
+    const uint4* src[K];
+#pragma unroll
+    for (int i = 0; i < K; ++i)
+        src[i] = reinterpret_cast<const uint4*>(a.state + (uint64_t)resolve(r[i], a.qcur) * a.stride) + v0;
+    uint4 x[U][K];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int i = 0; i < K; ++i) x[u][i] = __ldg(src[i] + u * 32);
+    uint4* dst = reinterpret_cast<uint4*>(a.state + (uint64_t)(a.row_gate0 + gate) * a.stride) + v0;
+    uint4* qd = qdst != 0xFFFFFFFFu ? reinterpret_cast<uint4*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride) + v0
+                                    : nullptr;
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+        const uint4 y = lut_eval4<K>(tt, x[u]);
+        dst[u * 32] = y;
+        if (qd) qd[u * 32] = y;
+    }
+}
+
+template <int U>
+__global__ void __launch_bounds__(256, 4) k_level_lut_wide(LevelArgs a, uint32_t cpg_shift, uint32_t vec0) {
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t gi = warp >> cpg_shift;
+    if (gi >= a.ng) return;
+    const uint32_t chunk = warp & ((1u << cpg_shift) - 1);
+    const uint32_t v0 = vec0 + chunk * 32 * U + lane;
+    const uint32_t gate = a.g0 + gi;
+    const uint4 in = __ldg(a.din + gate);
+    const uint4 au = __ldg(reinterpret_cast<const uint4*>(a.aux) + gate);
+    const uint64_t tt = ((uint64_t)au.y << 32) | au.x;
+    const uint32_t qdst = au.z, k = au.w;
+    switch (k) {
+        case 1: lut_gate_u<1, U>(a, gate, in, v0, tt, qdst); break;
+        case 2: lut_gate_u<2, U>(a, gate, in, v0, tt, qdst); break;
+        case 3: lut_gate_u<3, U>(a, gate, in, v0, tt, qdst); break;
+        case 4: lut_gate_u<4, U>(a, gate, in, v0, tt, qdst); break;
+        case 5: lut_gate_u<5, 1>(a, gate, in, v0, tt, qdst);
+                if (U > 1) lut_gate_u<5, 1>(a, gate, in, v0 + 32, tt, qdst);
+                if (U > 2) { lut_gate_u<5, 1>(a, gate, in, v0 + 64, tt, qdst);
+                             lut_gate_u<5, 1>(a, gate, in, v0 + 96, tt, qdst); }
+                break;
+        default: lut_gate_u<6, 1>(a, gate, in, v0, tt, qdst);
+                if (U > 1) lut_gate_u<6, 1>(a, gate, in, v0 + 32, tt, qdst);
+                if (U > 2) { lut_gate_u<6, 1>(a, gate, in, v0 + 64, tt, qdst);
+                             lut_gate_u<6, 1>(a, gate, in, v0 + 96, tt, qdst); }
+                break;
+    }
+}
+
 cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s) {
     if (a.ng == 0) return cudaSuccess;
+    // slab: 16-byte vectors [a.vec0, a.vec0 + a.vslab) of every row (whole row if vslab == 0)
+    if ((a.words % 2) == 0) {
+        const uint32_t vrow = a.vslab ? a.vslab : a.words / 2;
+        for (uint32_t U : {4u, 2u, 1u}) {
+            if (a.unroll && U > a.unroll) continue;
+            const uint32_t cpg = vrow / (32 * U);
+            if (vrow % (32 * U) || cpg == 0 || (cpg & (cpg - 1))) continue;
+            uint32_t sh = 0;
+            while ((1u << sh) < cpg) ++sh;
+            const uint64_t threads = ((uint64_t)a.ng << sh) * 32;
+            if (threads >= (1ull << 31)) break;
+            const uint32_t blocks = (uint32_t)((threads + 255) / 256);
+            if (U == 4) k_level_lut_wide<4><<<blocks, 256, 0, s>>>(a, sh, a.vec0);
+            else if (U == 2) k_level_lut_wide<2><<<blocks, 256, 0, s>>>(a, sh, a.vec0);
+            else k_level_lut_wide<1><<<blocks, 256, 0, s>>>(a, sh, a.vec0);
+            return cudaGetLastError();
+        }
+    }
+    if (a.vslab) return cudaErrorInvalidValue;      // slabs only on the wide path
     const bool vec16 = (a.words % 2) == 0;
     const uint32_t vpr = vec16 ? a.words / 2 : a.words;
     const bool pow2 = (vpr & (vpr - 1)) == 0;

@@ -35,6 +35,8 @@ struct LevelArgs {
     uint32_t row_gate0;
     uint32_t qcur, qnext;             // bank offsets (0 or n_reg) for Q refs / latch stores
     Ctl* ctl;
+    uint32_t vec0, vslab;             // lane slab in 16-byte vectors (vslab 0 = whole row)
+    uint32_t unroll;                  // max vectors per thread on the wide path (0 = auto)
 };
 
 struct EndArgs {

@@ -66,6 +66,7 @@ struct gs_sim {
     uint8_t* ws = nullptr;
     cudaStream_t stream = nullptr, cap = nullptr;
     uint32_t words = 0;
+    uint32_t slabs = 1;
     uint64_t stride = 0;
     uint64_t cycle = 0;               // host mirror of Ctl::cycle
     int bound = 0;                    // 0 none, 1 generated, 2 host/device buffer
@@ -131,8 +132,14 @@ static EndArgs end_args(const gs_sim* s, uint32_t parity) {
     return e;
 }
 
-static cudaError_t level_launch(const gs_sim* s, uint32_t l, uint32_t parity, cudaStream_t st) {
-    const LevelArgs a = level_args(s, l, parity);
+static cudaError_t level_launch(const gs_sim* s, uint32_t l, uint32_t parity, cudaStream_t st,
+                                uint32_t slab = 0) {
+    LevelArgs a = level_args(s, l, parity);
+    a.unroll = s->opts.lut_unroll;
+    if (s->slabs > 1) {
+        a.vslab = (s->words / 2) / s->slabs;
+        a.vec0 = slab * a.vslab;
+    }
     switch (s->opts.kernel) {
         case GS_KERNEL_POLY: return launch_level_poly(a, 0, st);
         case GS_KERNEL_AB: {
@@ -150,12 +157,15 @@ static cudaError_t cycle_launches(const gs_sim* s, uint32_t parity, cudaStream_t
     cudaError_t e = launch_stim(s->ctl(), s->state(), s->stride, s->words, p.row_pi0, p.n_pi,
                                 s->opts.lane_offset / 64, st);
     if (e != cudaSuccess) return e;
-    for (uint32_t l = 0; l < p.n_levels; ++l) {
-        if (evs) cudaEventRecord((*evs)[2 * l], st);
-        e = level_launch(s, l, parity, st);
-        if (e != cudaSuccess) return e;
-        if (evs) cudaEventRecord((*evs)[2 * l + 1], st);
-    }
+    // slab-major order: every level on lanes [slab], then the next slab (lanes are
+    // independent; a slab's recent levels fit L2)
+    for (uint32_t sl = 0; sl < s->slabs; ++sl)
+        for (uint32_t l = 0; l < p.n_levels; ++l) {
+            if (evs) cudaEventRecord((*evs)[2 * ((size_t)sl * p.n_levels + l)], st);
+            e = level_launch(s, l, parity, st, sl);
+            if (e != cudaSuccess) return e;
+            if (evs) cudaEventRecord((*evs)[2 * ((size_t)sl * p.n_levels + l) + 1], st);
+        }
     return launch_end_cycle(end_args(s, parity), st);
 }
 
@@ -231,6 +241,16 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts, void* d
     s->stream = static_cast<cudaStream_t>(opts->stream);
     s->words = words;
     s->stride = (uint64_t)words * 8;
+    s->slabs = opts->lane_slabs ? opts->lane_slabs : 1;
+    if (s->slabs > 1) {
+        const uint32_t vrow = words / 2;
+        if (s->opts.kernel != GS_KERNEL_LUT || words % 2 || vrow % s->slabs || (vrow / s->slabs) % 32) {
+
+            delete s;
+            return fail(GS_ERR_ARG, "gs_sim_create: lane_slabs needs kernel A and (lanes/128) % slabs == 0 "
+                                    "with a multiple of 4096 lanes per slab");
+        }
+    }
     auto cleanup = [&](gs_status st) {
         if (s->cap) cudaStreamDestroy(s->cap);
         delete s;
@@ -492,7 +512,7 @@ gs_status gs_sim_launches_per_cycle(const gs_sim* s, uint64_t* launches) {
     for (uint32_t l = 0; l < p.n_levels; ++l)
         if (p.level_off[l + 1] > p.level_off[l]) lv++;
     const uint64_t per_level = s->opts.kernel == GS_KERNEL_AB ? 2 : 1;
-    *launches = (p.n_pi ? 1 : 0) + lv * per_level + 1;
+    *launches = (p.n_pi ? 1 : 0) + lv * per_level * s->slabs + 1;
     return GS_OK;
 }
 
@@ -504,7 +524,7 @@ gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
         return fail(GS_ERR_STATE, "gs_sim_profile_step: stepping past the bound stimulus cycles");
     const Program& p = *s->prog;
     CU(cudaSetDevice(s->opts.device));
-    std::vector<cudaEvent_t> evs(2 * (size_t)p.n_levels);
+    std::vector<cudaEvent_t> evs(2 * (size_t)p.n_levels * s->slabs);
     cudaEvent_t e0, e1;
     for (auto& e : evs) CU(cudaEventCreate(&e));
     CU(cudaEventCreate(&e0));
@@ -531,13 +551,15 @@ gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
         float ms = 0;
         cudaEventElapsedTime(&ms, e0, e1);
         total_ms += ms;
-        for (uint32_t l = 0; l < p.n_levels; ++l) {
-            if (p.level_off[l + 1] == p.level_off[l]) continue;
-            cudaEventElapsedTime(&ms, evs[2 * l], evs[2 * l + 1]);
-            level_ms += ms;
-            level_bytes += lb[l];
-            lvl_launches++;
-        }
+        for (uint32_t sl = 0; sl < s->slabs; ++sl)
+            for (uint32_t l = 0; l < p.n_levels; ++l) {
+                if (p.level_off[l + 1] == p.level_off[l]) continue;
+                const size_t ix = (size_t)sl * p.n_levels + l;
+                cudaEventElapsedTime(&ms, evs[2 * ix], evs[2 * ix + 1]);
+                level_ms += ms;
+                level_bytes += lb[l] / s->slabs;
+                lvl_launches++;
+            }
         launches += per;
     }
     for (auto& e : evs) cudaEventDestroy(e);
