@@ -43,9 +43,12 @@ def parse():
     ap.add_argument("--config", default="C4")
     ap.add_argument("--cycles-per-step", type=int, default=100)
     ap.add_argument("--lanes", type=int, default=0, help="override lanes per GPU")
-    ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab"])
+    ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab", "df"])
+    ap.add_argument("--df-interleave", type=int, default=0, help="kernel D: slabs walked together")
+    ap.add_argument("--df-gpw", type=int, default=0, help="kernel D: gates per warp per item")
     ap.add_argument("--lane-slabs", type=int, default=0, help="L2 lane slabs (0 = library default)")
     ap.add_argument("--lut-unroll", type=int, default=0, help="vectors per thread (0 = auto)")
+    ap.add_argument("--no-pdl", action="store_true", help="disable programmatic dependent launch")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-roofline", action="store_true")
@@ -110,6 +113,23 @@ def peaks():
         return {"hbm_gbs": 6650.0}, "fallback"
 
 
+KERNEL_NAMES = {"lut": "k_level_lut_wide<4>", "df": "k_dataflow<1>", "poly": "k_level_poly",
+                "ab": "k_level_lut_wide<4>"}
+
+
+def ncu_traffic(kernel: str):
+    """dram read+write bytes per launch of `kernel` from the committed ncu --set full summary
+    (profiles/traffic.json, written by scripts/ncu_summary.py from the same bench command)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            d = json.load(f)
+        e = d["kernels"][kernel]
+        return {"traffic_bytes_per_launch": e["traffic_bytes_per_launch"],
+                "source": e.get("source", d.get("source"))}
+    except Exception:
+        return None
+
+
 # ------------------------------------------------------------------ CPU oracle
 def oracle_rate(nl, cfg, lane_offset, seconds: float, cycles_cap: int | None = None):
     """Time the oracle (as it stands) on a bounded sample: n_threads lanes x c cycles."""
@@ -118,12 +138,12 @@ def oracle_rate(nl, cfg, lane_offset, seconds: float, cycles_cap: int | None = N
     threads = oracle.max_threads()
     G = int((nl.gate_k > 0).sum())
     lanes_total = cfg.lanes
-    # calibration: one lane per thread, 2 cycles
+    # calibration: one lane per thread, 8 cycles
     sample = np.linspace(0, lanes_total - 1, threads).astype(np.int64) + lane_offset
     t = time.perf_counter()
-    oracle.simulate(nl, sample, 2, seed=cfg.stim_seed, threads=threads, want=("sig",))
+    oracle.simulate(nl, sample, 8, seed=cfg.stim_seed, threads=threads, want=("sig",))
     dt = max(time.perf_counter() - t, 1e-3)
-    per_cycle = dt / 2
+    per_cycle = dt / 8
     cycles = max(2, int(seconds / per_cycle))
     if cycles_cap:
         cycles = min(cycles, cycles_cap)
@@ -208,7 +228,8 @@ def main():
         gdist.check_same_program(info["program_hash"])
     stream = torch.cuda.Stream(device=local)
     sim = gs.Sim(prog, lanes, lane_offset=lane_offset, kernel=args.kernel, device=local, stream=stream,
-                 lane_slabs=args.lane_slabs, lut_unroll=args.lut_unroll)
+                 lane_slabs=args.lane_slabs, lut_unroll=args.lut_unroll,
+                 df_interleave=args.df_interleave, df_gates_per_warp=args.df_gpw, pdl=not args.no_pdl)
     sim.bind_generated(cfg.stim_seed)
     C = args.cycles_per_step
     launches_per_cycle = sim.launches_per_cycle()
@@ -248,9 +269,15 @@ def main():
         pr = sim.profile_step(min(C, 10))
         achieved = pr["level_bytes"] / (pr["level_ms"] / 1e3) / 1e9
         per_launch_bytes = pr["level_bytes"] / max(pr["level_launches"], 1)
-        roof = {"bound": "hbm", "kernel": "k_level_lut (kernel A, one launch per level)",
+        kname = KERNEL_NAMES[args.kernel]
+        if args.kernel == "df":
+            kname = f"k_dataflow<{lanes // (args.lane_slabs or lanes // 4096) // 4096}>"
+        tr = ncu_traffic(kname)
+        roof = {"bound": "hbm", "kernel": kname,
                 "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
-                "frac": achieved / pk["hbm_gbs"], "traffic": None,
+                "frac": achieved / pk["hbm_gbs"],
+                "traffic": tr["traffic_bytes_per_launch"] if tr else None,
+                "traffic_source": tr["source"] if tr else None,
                 "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({pk_src})",
                 "algorithmic_bytes_per_launch": per_launch_bytes,
                 "level_share_of_step": pr["level_ms"] / pr["total_ms"],
@@ -303,6 +330,8 @@ def main():
                        "levels": info["n_levels"], "lanes_per_gpu": lanes, "lanes_total": lanes * world,
                        "cycles_per_step": C, "kernel": args.kernel, "balance": True,
                        "lane_slabs": args.lane_slabs, "lut_unroll": args.lut_unroll,
+                       "df_interleave": args.df_interleave, "df_gpw": args.df_gpw,
+                       "pdl": not args.no_pdl,
                        "l2": "inputs larger than L2 (state %.1f GB per GPU)" % (info["n_rows"] * lanes / 8 / 1e9),
                        "parallelism": f"dp{world} (stimulus sharding)", "compile_s": round(compile_s, 2),
                        "paper_style_gcps": value * (G + info["n_reg"]) / G},

@@ -176,7 +176,12 @@ enum {
     GS_KERNEL_LUT = 1,    /* kernel A: bit-sliced LUT evaluation, 64 stimuli per word      */
     GS_KERNEL_POLY = 2,   /* kernel B: the paper's network, sum_S w_S Theta(sum x - |S| + 1)
                              per stimulus in int32, ballot-packed (Eq. 1-3)                */
-    GS_KERNEL_AB = 3      /* A writes, B recomputes every level and counts mismatches      */
+    GS_KERNEL_AB = 3,     /* A writes, B recomputes every level and counts mismatches      */
+    GS_KERNEL_DATAFLOW = 4 /* kernel A evaluation in ONE persistent launch per cycle: lanes cut
+                             into slabs, (slab, level, gate chunk) items from a work queue, an
+                             item waits only for the previous level of its slab, so a slab's
+                             recent levels are read from L2 (DESIGN.md §6 "kernel D").
+                             Needs lanes/lane_slabs in {4096, 8192, 16384}.                 */
 };
 
 typedef struct {
@@ -189,11 +194,18 @@ typedef struct {
     const uint32_t* trace_words;  /* [n_trace_words] local word indices (copied)           */
     uint32_t trace_cycles;        /* capacity of the trace, in cycles                      */
     int use_graphs;               /* 1: replay each cycle as a CUDA graph (default)        */
-    uint32_t lane_slabs;          /* kernel A: run all levels on 1/lane_slabs of the lanes at a
+    uint32_t lane_slabs;          /* LUT: run all levels on 1/lane_slabs of the lanes at a
                                      time so recent levels stay L2-resident (0/1 = off); needs
-                                     (lanes/128) % lane_slabs == 0 and slabs >= 4096 lanes   */
+                                     (lanes/128) % lane_slabs == 0 and slabs >= 4096 lanes.
+                                     DATAFLOW: number of slabs (0 = lanes/4096)              */
     uint32_t lut_unroll;          /* kernel A: max 16-byte vectors per thread (0 = auto)   */
+    uint32_t df_interleave;       /* DATAFLOW: slabs walked level by level together (0 = 8) */
+    uint32_t df_gates_per_warp;   /* DATAFLOW: gates per warp per work item, 1..32 (0 = 8) */
+    uint32_t flags;               /* GS_SIM_* bits below                                   */
 } gs_sim_opts;
+/* flags: launch the per-cycle kernels WITHOUT programmatic dependent launch (by default a
+ * level kernel may become resident while its predecessor drains; A/B measurement only). */
+#define GS_SIM_NO_PDL 1u
 
 /* Device workspace bytes required for (prog, opts). */
 gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts, size_t* bytes);

@@ -24,8 +24,9 @@ GS_OK = 0
 GS_ERR_ARG, GS_ERR_ARITY, GS_ERR_UNDRIVEN, GS_ERR_COMB_LOOP = -1, -2, -3, -4
 GS_ERR_BUFFER_TOO_SMALL, GS_ERR_CUDA, GS_ERR_STATE, GS_ERR_NOMEM = -5, -6, -7, -8
 GS_MAX_K = 6
-GS_KERNEL_AUTO, GS_KERNEL_LUT, GS_KERNEL_POLY, GS_KERNEL_AB = 0, 1, 2, 3
-KERNELS = {"auto": 0, "lut": 1, "A": 1, "poly": 2, "B": 2, "ab": 3, "AB": 3}
+GS_SIM_NO_PDL = 1
+GS_KERNEL_AUTO, GS_KERNEL_LUT, GS_KERNEL_POLY, GS_KERNEL_AB, GS_KERNEL_DATAFLOW = 0, 1, 2, 3, 4
+KERNELS = {"auto": 0, "lut": 1, "A": 1, "poly": 2, "B": 2, "ab": 3, "AB": 3, "df": 4, "dataflow": 4}
 
 
 class GsError(RuntimeError):
@@ -69,7 +70,9 @@ class gs_sim_opts(C.Structure):
     _fields_ = [("device", C.c_int), ("stream", C.c_void_p), ("lanes", C.c_uint64),
                 ("lane_offset", C.c_uint64), ("kernel", C.c_int), ("n_trace_words", C.c_uint32),
                 ("trace_words", C.c_void_p), ("trace_cycles", C.c_uint32), ("use_graphs", C.c_int),
-                ("lane_slabs", C.c_uint32), ("lut_unroll", C.c_uint32)]
+                ("lane_slabs", C.c_uint32), ("lut_unroll", C.c_uint32),
+                ("df_interleave", C.c_uint32), ("df_gates_per_warp", C.c_uint32),
+                ("flags", C.c_uint32)]
 
 
 class gs_signature(C.Structure):
@@ -265,7 +268,8 @@ class Sim:
 
     def __init__(self, program: Program, lanes: int, lane_offset: int = 0, kernel="lut",
                  device: int = 0, stream=None, trace_words=(), trace_cycles: int = 0,
-                 use_graphs: bool = True, lane_slabs: int = 0, lut_unroll: int = 0):
+                 use_graphs: bool = True, lane_slabs: int = 0, lut_unroll: int = 0,
+                 df_interleave: int = 0, df_gates_per_warp: int = 0, pdl: bool = True):
         import torch
         self.program = program
         self.lanes, self.words = int(lanes), int(lanes) // 64
@@ -275,7 +279,8 @@ class Sim:
         o = gs_sim_opts(device, C.c_void_p(self.stream.cuda_stream), self.lanes, int(lane_offset),
                         KERNELS[kernel] if isinstance(kernel, str) else int(kernel), len(self._tw),
                         _p(self._tw) if len(self._tw) else None, int(trace_cycles),
-                        1 if use_graphs else 0, int(lane_slabs), int(lut_unroll))
+                        1 if use_graphs else 0, int(lane_slabs), int(lut_unroll),
+                        int(df_interleave), int(df_gates_per_warp), 0 if pdl else GS_SIM_NO_PDL)
         nbytes = C.c_size_t()
         _call("gs_sim_workspace_bytes", program.h, C.byref(o), C.byref(nbytes))
         self.workspace = torch.empty(int(nbytes.value) + 256, dtype=torch.uint8, device=self.device)

@@ -39,6 +39,32 @@ __device__ __forceinline__ unsigned long long dmix64(unsigned long long z) {
     return z ^ (z >> 31);
 }
 
+// ------------------------------------------------------- programmatic dependent launch
+// Every kernel of the per-cycle chain is launched with programmatic stream serialization
+// (when enabled): it may become resident while its predecessor drains, and waits at
+// griddepcontrol.wait until the predecessor has completed and its writes are visible.
+// It immediately allows its own successor to launch.  Without the launch attribute both
+// instructions are no-ops, so the kernels are correct either way.
+__device__ __forceinline__ void pdl_entry() {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
+template <typename... KArgs, typename... Args>
+static cudaError_t launch_k(void (*kern)(KArgs...), uint32_t blocks, cudaStream_t s, uint32_t pdl,
+                            Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(blocks);
+    cfg.blockDim = dim3(256);
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = pdl ? at : nullptr;
+    cfg.numAttrs = pdl ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+
 // ------------------------------------------------------------------ kernel A: LUT
 // Bit-sliced Shannon expansion of an LSB-first truth table: stage 0 selects between
 // the minterm constants with x_0, stage i muxes pairs with x_i.  All operands are
@@ -152,6 +178,7 @@ __device__ __forceinline__ void lut_gate_vec8(const LevelArgs& a, uint32_t gate,
 // single gate (k is warp-uniform, loads are 512 B contiguous per input row).
 template <bool VEC16, bool POW2>
 __global__ void __launch_bounds__(256) k_level_lut(LevelArgs a, uint32_t vpr, uint32_t vshift) {
+    pdl_entry();
     const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
     const uint32_t gi = POW2 ? (t >> vshift) : (t / vpr);
     if (gi >= a.ng) return;
@@ -216,6 +243,7 @@ __device__ __forceinline__ void lut_gate_u(const LevelArgs& a, uint32_t gate, ui
 
 template <int U>
 __global__ void __launch_bounds__(256, 4) k_level_lut_wide(LevelArgs a, uint32_t cpg_shift, uint32_t vec0) {
+    pdl_entry();
     const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t gi = warp >> cpg_shift;
@@ -254,15 +282,17 @@ cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s) {
             if (a.unroll && U > a.unroll) continue;
             const uint32_t cpg = vrow / (32 * U);
             if (vrow % (32 * U) || cpg == 0 || (cpg & (cpg - 1))) continue;
+            // auto: trade vectors per thread for warps while a narrow level would not
+            // fill the GPU (memory-level parallelism per thread vs threads in flight)
+            if (!a.unroll && U > 1 && (uint64_t)a.ng * cpg < a.min_warps) continue;
             uint32_t sh = 0;
             while ((1u << sh) < cpg) ++sh;
             const uint64_t threads = ((uint64_t)a.ng << sh) * 32;
             if (threads >= (1ull << 31)) break;
             const uint32_t blocks = (uint32_t)((threads + 255) / 256);
-            if (U == 4) k_level_lut_wide<4><<<blocks, 256, 0, s>>>(a, sh, a.vec0);
-            else if (U == 2) k_level_lut_wide<2><<<blocks, 256, 0, s>>>(a, sh, a.vec0);
-            else k_level_lut_wide<1><<<blocks, 256, 0, s>>>(a, sh, a.vec0);
-            return cudaGetLastError();
+            if (U == 4) return launch_k(k_level_lut_wide<4>, blocks, s, a.pdl, a, sh, a.vec0);
+            if (U == 2) return launch_k(k_level_lut_wide<2>, blocks, s, a.pdl, a, sh, a.vec0);
+            return launch_k(k_level_lut_wide<1>, blocks, s, a.pdl, a, sh, a.vec0);
         }
     }
     if (a.vslab) return cudaErrorInvalidValue;      // slabs only on the wide path
@@ -275,13 +305,192 @@ cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s) {
     if (threads >= (1ull << 31)) return cudaErrorInvalidValue;
     const uint32_t blocks = (uint32_t)((threads + 255) / 256);
     if (vec16) {
-        if (pow2) k_level_lut<true, true><<<blocks, 256, 0, s>>>(a, vpr, vshift);
-        else k_level_lut<true, false><<<blocks, 256, 0, s>>>(a, vpr, vshift);
-    } else {
-        if (pow2) k_level_lut<false, true><<<blocks, 256, 0, s>>>(a, vpr, vshift);
-        else k_level_lut<false, false><<<blocks, 256, 0, s>>>(a, vpr, vshift);
+        if (pow2) return launch_k(k_level_lut<true, true>, blocks, s, a.pdl, a, vpr, vshift);
+        return launch_k(k_level_lut<true, false>, blocks, s, a.pdl, a, vpr, vshift);
     }
-    return cudaGetLastError();
+    if (pow2) return launch_k(k_level_lut<false, true>, blocks, s, a.pdl, a, vpr, vshift);
+    return launch_k(k_level_lut<false, false>, blocks, s, a.pdl, a, vpr, vshift);
+}
+
+// ------------------------------------------- kernel A, persistent slab dataflow ("D")
+// One launch evaluates every level of one cycle.  The lanes are cut into slabs of
+// 4096*VPL stimuli (512*VPL bytes per row); slabs are independent, so the levels of
+// different slabs need no ordering.  Work items (slab, level, chunk of 8*gpw gates)
+// are handed out in a fixed order through one atomic queue head; an item waits only
+// until every item of the previous level of ITS slab is done (a per-(slab, level)
+// counter, release/acquire).  Consequences:
+//   * no launch boundary per level: the tail of level l of slab s overlaps level l
+//     of slab s+1 (slabs are walked `interleave` at a time, level-major);
+//   * a slab's recent levels (~15k gates x 512 B per level on C4) stay in L2, so most
+//     gate-input reads (inputs from level l-1..l-8) are L2 hits rather than HBM reads;
+//   * no deadlock for any grid size: an item only waits for items taken earlier from
+//     the queue, which are held by running CTAs (induction on the queue index).
+// Loads use ld.global.cg (L2, never a stale L1 line); stores are plain.
+__device__ __forceinline__ unsigned ld_acquire(const unsigned* p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// A gate's slab row segment (slab_vec 16-byte vectors) is owned by a group of LPG
+// lanes, each holding VPT = slab_vec / LPG vectors, so every thread keeps VPT * k
+// independent loads in flight (the memory-level parallelism of kernel A's U = 4) and
+// a warp works on 32 / LPG gates at once.
+template <int K, int VPT, int LPG>
+__device__ __forceinline__ void df_gate(const DfArgs& a, uint32_t gate, uint4 in, uint64_t tt, uint32_t qdst,
+                                        uint32_t v0) {
+    uint32_t r[6];
+    r[0] = in.x; r[1] = in.y; r[2] = in.z; r[3] = in.w;
+    if (K > 4) {
+        const uint2 hi = __ldg(a.dhi + gate);
+        r[4] = hi.x; r[5] = hi.y;
+    }
+    const uint4* src[K];
+#pragma unroll
+    for (int i = 0; i < K; ++i)
+        src[i] = reinterpret_cast<const uint4*>(a.state + (uint64_t)resolve(r[i], a.qcur) * a.stride) + v0;
+    uint4 x[VPT][K];
+#pragma unroll
+    for (int u = 0; u < VPT; ++u)
+#pragma unroll
+        for (int i = 0; i < K; ++i) x[u][i] = __ldcg(src[i] + u * LPG);
+    uint4* dst = reinterpret_cast<uint4*>(a.state + (uint64_t)(a.row_gate0 + gate) * a.stride) + v0;
+    uint4* qd = qdst != 0xFFFFFFFFu ? reinterpret_cast<uint4*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride) + v0
+                                    : nullptr;
+#pragma unroll
+    for (int u = 0; u < VPT; ++u) {
+        const uint4 y = lut_eval4<K>(tt, x[u]);
+        dst[u * LPG] = y;
+        if (qd) qd[u * LPG] = y;
+    }
+}
+
+// k = 5, 6: one vector at a time (keeps the register footprint of k <= 4)
+template <int K, int VPT, int LPG>
+__device__ __forceinline__ void df_gate_wide(const DfArgs& a, uint32_t gate, uint4 in, uint64_t tt, uint32_t qdst,
+                                             uint32_t v0) {
+#pragma unroll 1
+    for (int u = 0; u < VPT; ++u) df_gate<K, 1, LPG>(a, gate, in, tt, qdst, v0 + u * LPG);
+}
+
+// Work item = (slab, level, chunk of 8 * gpw gates) for one CTA (8 warps x gpw gates).
+// Items are numbered groups of `interleave` slabs -> level -> slab -> chunk and handed
+// out by one atomic queue head; the claim of the next item is issued while the current
+// one is processed.  No deadlock for any grid size: an item only waits for items
+// claimed earlier, which are held by running CTAs (induction on the queue index).
+template <int VPT, int LPG>
+__global__ void __launch_bounds__(256, 4) k_dataflow(DfArgs a) {
+    pdl_entry();
+    __shared__ unsigned s_item[2];
+    constexpr uint32_t GPP = 32 / LPG;                            // gates per warp pass
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t grp = lane / LPG, li = lane % LPG;
+    const uint32_t per_group = a.interleave * a.items_per_slab;
+    if (threadIdx.x == 0) s_item[0] = atomicAdd(a.qhead, 1u);
+    __syncthreads();
+    for (uint32_t it = 0;; it ^= 1) {
+        const uint32_t q = s_item[it];
+        if (q >= a.total_items) return;                           // block-uniform
+        unsigned next = 0;
+        if (threadIdx.x == 0) next = atomicAdd(a.qhead, 1u);      // in flight during the item
+        // ---- decode q -> (slab, level, chunk)
+        const uint32_t sg = q / per_group;
+        uint32_t rr = q - sg * per_group;
+        const uint32_t s0 = sg * a.interleave;
+        const uint32_t I = min(a.interleave, a.n_slabs - s0);
+        uint32_t lo = 0, hi = a.nl;                               // I*item0[lo] <= rr < I*item0[hi]
+        while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (I * __ldg(a.lv_item0 + mid) <= rr) lo = mid; else hi = mid;
+        }
+        const uint32_t l = lo;
+        const uint32_t it0 = __ldg(a.lv_item0 + l);
+        const uint32_t nli = __ldg(a.lv_item0 + l + 1) - it0;
+        rr -= I * it0;
+        const uint32_t si = rr / nli, chunk = rr - si * nli;
+        const uint32_t slab = s0 + si;
+        // ---- this warp's gates and their descriptors (issued before the wait)
+        const uint32_t lg1 = __ldg(a.lv_gate0 + l + 1);
+        const uint32_t gb = __ldg(a.lv_gate0 + l) + (chunk * 8 + warp) * a.gpw;
+        const uint32_t ge = min(gb + a.gpw, lg1);
+        uint4 my_in = make_uint4(0, 0, 0, 0), my_au = make_uint4(0, 0, 0, 0);
+        if (gb + lane < ge) {
+            my_in = __ldg(a.din + gb + lane);
+            my_au = __ldg(reinterpret_cast<const uint4*>(a.aux) + gb + lane);
+        }
+        // ---- wait until every item of the previous level of this slab is done
+        if (l > 0) {
+            if (threadIdx.x == 0) {
+                const unsigned need = it0 - __ldg(a.lv_item0 + l - 1);
+                const unsigned* p = a.done + (uint64_t)slab * a.nl + (l - 1);
+                if (ld_acquire(p) < need) {
+                    const long long t0 = clock64();
+                    while (ld_acquire(p) < need) {
+                        __nanosleep(64);
+                        if (clock64() - t0 > (1ll << 35)) __trap();   // ~17 s: never hang the GPU
+                    }
+                }
+            }
+            __syncthreads();
+        }
+        const uint32_t v0 = slab * a.slab_vec + li;
+        for (uint32_t p0 = 0; gb + p0 < ge; p0 += GPP) {
+            const uint32_t j = p0 + grp;
+            uint4 in, au;
+            in.x = __shfl_sync(FULL, my_in.x, j & 31); in.y = __shfl_sync(FULL, my_in.y, j & 31);
+            in.z = __shfl_sync(FULL, my_in.z, j & 31); in.w = __shfl_sync(FULL, my_in.w, j & 31);
+            au.x = __shfl_sync(FULL, my_au.x, j & 31); au.y = __shfl_sync(FULL, my_au.y, j & 31);
+            au.z = __shfl_sync(FULL, my_au.z, j & 31); au.w = __shfl_sync(FULL, my_au.w, j & 31);
+            if (gb + j >= ge) continue;
+            const uint32_t g = gb + j;
+            const uint64_t tt = ((uint64_t)au.y << 32) | au.x;
+            switch (au.w) {
+                case 1: df_gate<1, VPT, LPG>(a, g, in, tt, au.z, v0); break;
+                case 2: df_gate<2, VPT, LPG>(a, g, in, tt, au.z, v0); break;
+                case 3: df_gate<3, VPT, LPG>(a, g, in, tt, au.z, v0); break;
+                case 4: df_gate<4, VPT, LPG>(a, g, in, tt, au.z, v0); break;
+                case 5: df_gate_wide<5, VPT, LPG>(a, g, in, tt, au.z, v0); break;
+                default: df_gate_wide<6, VPT, LPG>(a, g, in, tt, au.z, v0); break;
+            }
+        }
+        if (threadIdx.x == 0) s_item[it ^ 1] = next;
+        // ---- publish: all of this item's stores happen-before the counter increment
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            __threadfence();
+            atomicAdd(a.done + (uint64_t)slab * a.nl + l, 1u);
+        }
+    }
+}
+
+// slab_vec = 16-byte vectors per slab row (32, 64 or 128); lanes per gate = slab_vec / 4
+#define DF_SWITCH(SV, CALL)                                                  \
+    switch (SV) {                                                            \
+        case 32: CALL(4, 8); break;                                          \
+        case 64: CALL(4, 16); break;                                         \
+        case 128: CALL(4, 32); break;                                        \
+        default: return cudaErrorInvalidValue;                               \
+    }
+
+cudaError_t dataflow_grid(uint32_t slab_vec, int device, uint32_t* grid) {
+    int sms = 0, per = 0;
+    cudaError_t e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    if (e != cudaSuccess) return e;
+#define DF_OCC(V, L) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_dataflow<V, L>, 256, 0)
+    DF_SWITCH(slab_vec, DF_OCC)
+#undef DF_OCC
+    if (e != cudaSuccess) return e;
+    *grid = (uint32_t)(sms * (per > 0 ? per : 1));
+    return cudaSuccess;
+}
+
+cudaError_t launch_dataflow(const DfArgs& a, uint32_t grid, cudaStream_t s) {
+    if (a.total_items == 0) return cudaSuccess;
+    cudaError_t e = cudaSuccess;
+#define DF_LAUNCH(V, L) e = launch_k(k_dataflow<V, L>, grid, s, 0u, a)
+    DF_SWITCH(a.slab_vec, DF_LAUNCH)
+#undef DF_LAUNCH
+    return e;
 }
 
 // ------------------------------------------------------------ kernel B: polynomial
@@ -289,6 +498,7 @@ cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s) {
 // stimulus t of every word b; the words are transposed with shuffles so each lane
 // builds its own input point idx[b] (bit i = x_i), then evaluates the network.
 __global__ void __launch_bounds__(256) k_level_poly(LevelArgs a, uint32_t words32, uint32_t wpg, int check_only) {
+    pdl_entry();
     const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t gi = warp / wpg;
@@ -374,13 +584,13 @@ cudaError_t launch_level_poly(const LevelArgs& a, int check_only, cudaStream_t s
     const uint64_t warps = (uint64_t)a.ng * wpg;
     if (warps * 32 >= (1ull << 31)) return cudaErrorInvalidValue;
     const uint32_t blocks = (uint32_t)((warps * 32 + 255) / 256);
-    k_level_poly<<<blocks, 256, 0, s>>>(a, words32, wpg, check_only);
-    return cudaGetLastError();
+    return launch_k(k_level_poly, blocks, s, a.pdl, a, words32, wpg, check_only);
 }
 
 // --------------------------------------------------------------------- stimulus
 __global__ void __launch_bounds__(256) k_stim(Ctl* ctl, uint8_t* state, uint64_t stride, uint32_t words,
                                               uint32_t row_pi0, uint32_t n_pi, uint64_t word_off) {
+    pdl_entry();
     const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (uint64_t)n_pi * words) return;
     const uint32_t p = (uint32_t)(t / words), w = (uint32_t)(t - (uint64_t)p * words);
@@ -396,11 +606,11 @@ __global__ void __launch_bounds__(256) k_stim(Ctl* ctl, uint8_t* state, uint64_t
 }
 
 cudaError_t launch_stim(Ctl* ctl, uint8_t* state, uint64_t stride, uint32_t words, uint32_t row_pi0,
-                        uint32_t n_pi, uint64_t word_off, cudaStream_t s) {
+                        uint32_t n_pi, uint64_t word_off, uint32_t pdl, cudaStream_t s) {
     const uint64_t n = (uint64_t)n_pi * words;
     if (n == 0) return cudaSuccess;
-    k_stim<<<(uint32_t)((n + 255) / 256), 256, 0, s>>>(ctl, state, stride, words, row_pi0, n_pi, word_off);
-    return cudaGetLastError();
+    return launch_k(k_stim, (uint32_t)((n + 255) / 256), s, pdl, ctl, state, stride, words, row_pi0, n_pi,
+                    word_off);
 }
 
 // --------------------------------------------------------------- end of cycle
@@ -412,6 +622,7 @@ cudaError_t launch_stim(Ctl* ctl, uint8_t* state, uint64_t stride, uint32_t word
 constexpr unsigned long long MISR_POLY = 0x42F0E1EBA9EA3693ULL;   // CRC-64/ECMA-182
 
 __global__ void __launch_bounds__(256) k_end_cycle(EndArgs a, uint32_t latch_blocks) {
+    pdl_entry();
     const unsigned long long c = a.ctl->cycle;
     if (blockIdx.x < latch_blocks) {
         const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -477,8 +688,7 @@ cudaError_t launch_end_cycle(const EndArgs& a, cudaStream_t s) {
     const uint64_t lt = (uint64_t)a.n_latch * a.words;
     const uint32_t latch_blocks = (uint32_t)((lt + 255) / 256);
     const uint32_t misr_blocks = (a.words * 32 + 255) / 256;
-    k_end_cycle<<<latch_blocks + misr_blocks, 256, 0, s>>>(a, latch_blocks);
-    return cudaGetLastError();
+    return launch_k(k_end_cycle, latch_blocks + misr_blocks, s, a.pdl, a, latch_blocks);
 }
 
 // --------------------------------------------------------------------- utilities

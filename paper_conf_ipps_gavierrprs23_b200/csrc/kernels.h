@@ -37,6 +37,8 @@ struct LevelArgs {
     Ctl* ctl;
     uint32_t vec0, vslab;             // lane slab in 16-byte vectors (vslab 0 = whole row)
     uint32_t unroll;                  // max vectors per thread on the wide path (0 = auto)
+    uint32_t pdl;                     // launch with programmatic stream serialization
+    uint32_t min_warps;               // auto U: prefer smaller U below this many warps
 };
 
 struct EndArgs {
@@ -54,12 +56,37 @@ struct EndArgs {
     const int32_t* trace_slot;        // [words]
     unsigned long long* trace;        // [trace_cap][n_po][ntw]
     uint32_t ntw, trace_cap;
+    uint32_t pdl;
+};
+
+// Persistent slab-dataflow schedule of kernel A (kernels.cu, DESIGN.md §6 "kernel D"):
+// one launch per cycle runs every (lane slab, level, gate chunk) item; an item waits
+// only for the previous level of its own slab.
+struct DfArgs {
+    const uint4* din;
+    const GateAux* aux;
+    const uint2* dhi;
+    uint8_t* state;
+    uint64_t stride;
+    uint32_t row_gate0, qcur, qnext;
+    const uint32_t* lv_gate0;         // [nl + 1] exec-order first gate of compact level i
+    const uint32_t* lv_item0;         // [nl + 1] prefix sum of items per level (one slab)
+    uint32_t nl;                      // non-empty levels
+    uint32_t items_per_slab;          // lv_item0[nl]
+    uint32_t n_slabs, interleave;     // slabs; slabs walked level-by-level together
+    uint32_t slab_vec;                // 16-byte vectors per slab row (32 * VPL)
+    uint32_t gpw;                     // gates per warp per work item (item = 8 warps)
+    uint32_t total_items;
+    unsigned int* qhead;              // work-queue head (zeroed every cycle)
+    unsigned int* done;               // [n_slabs * nl] finished items (zeroed every cycle)
 };
 
 cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s);
+cudaError_t launch_dataflow(const DfArgs& a, uint32_t grid, cudaStream_t s);
+cudaError_t dataflow_grid(uint32_t slab_vec, int device, uint32_t* grid);
 cudaError_t launch_level_poly(const LevelArgs& a, int check_only, cudaStream_t s);
 cudaError_t launch_stim(Ctl* ctl, uint8_t* state, uint64_t stride, uint32_t words, uint32_t row_pi0,
-                        uint32_t n_pi, uint64_t word_off, cudaStream_t s);
+                        uint32_t n_pi, uint64_t word_off, uint32_t pdl, cudaStream_t s);
 cudaError_t launch_end_cycle(const EndArgs& a, cudaStream_t s);
 cudaError_t launch_fill_rows(uint8_t* state, uint64_t stride, uint32_t words, uint32_t row0, uint32_t nrows,
                              const uint8_t* init, int value, cudaStream_t s);

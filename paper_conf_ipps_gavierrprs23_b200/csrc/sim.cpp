@@ -5,6 +5,7 @@
 // The per-cycle launch sequence only depends on the Q-bank parity, so it is captured
 // once per parity as a CUDA graph and replayed; the cycle index lives on the device
 // (Ctl::cycle) and is advanced by the end-of-cycle kernel.
+#include <algorithm>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -22,10 +23,47 @@ size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 
 struct Layout {
     size_t ctl, state, din, aux, dhi, term_off, terms, po_rows, latch_src, latch_dst, reg_init,
-        trace_slot, misr, trace, lane_sigs, scratch, total;
+        trace_slot, misr, trace, lane_sigs, scratch, lv_gate0, lv_item0, dfctl, dfctl_bytes, total;
 };
 
-Layout make_layout(const Program& p, const gs_sim_opts& o) {
+// Work-item plan of the DATAFLOW schedule (kernels.cu k_dataflow): non-empty levels only
+// (an empty level would break the "previous level done => all earlier levels done" chain).
+struct DfPlan {
+    uint32_t vpl = 0, n_slabs = 0, interleave = 0, gpw = 0, nl = 0;
+    std::vector<uint32_t> lv_gate0, lv_item0;
+};
+
+gs_status df_plan(const Program& p, const gs_sim_opts& o, DfPlan& d) {
+    if (o.kernel != GS_KERNEL_DATAFLOW) return GS_OK;
+    const uint64_t slabs = o.lane_slabs ? o.lane_slabs : o.lanes / 4096;
+    if (slabs == 0 || o.lanes % slabs)
+        return fail(GS_ERR_ARG, "DATAFLOW: lanes must be a multiple of lane_slabs (and of 4096)");
+    const uint64_t sl = o.lanes / slabs;
+    if (sl != 4096 && sl != 8192 && sl != 16384)
+        return fail(GS_ERR_ARG, "DATAFLOW: lanes / lane_slabs must be 4096, 8192 or 16384");
+    d.vpl = (uint32_t)(sl / 4096);
+    d.n_slabs = (uint32_t)slabs;
+    d.interleave = o.df_interleave ? o.df_interleave : 8;
+    if (d.interleave > d.n_slabs) d.interleave = d.n_slabs;
+    d.gpw = o.df_gates_per_warp ? o.df_gates_per_warp : 8;
+    if (d.gpw > 32) return fail(GS_ERR_ARG, "DATAFLOW: df_gates_per_warp must be <= 32");
+    const uint32_t gpi = 8 * d.gpw;              // one item = 8 warps x gpw gates
+    d.lv_gate0.clear();
+    d.lv_item0.assign(1, 0);
+    for (uint32_t l = 0; l < p.n_levels; ++l) {
+        const uint32_t w = p.level_off[l + 1] - p.level_off[l];
+        if (!w) continue;
+        d.lv_gate0.push_back(p.level_off[l]);
+        d.lv_item0.push_back(d.lv_item0.back() + (w + gpi - 1) / gpi);
+    }
+    d.nl = (uint32_t)d.lv_gate0.size();
+    d.lv_gate0.push_back(p.n_eval);
+    if ((uint64_t)d.lv_item0.back() * d.n_slabs >= (1ull << 32))
+        return fail(GS_ERR_ARG, "DATAFLOW: too many work items per cycle; raise df_gates_per_warp");
+    return GS_OK;
+}
+
+Layout make_layout(const Program& p, const gs_sim_opts& o, const DfPlan& d) {
     Layout L{};
     const uint64_t words = o.lanes / 64;
     const uint64_t stride = words * 8;
@@ -52,6 +90,10 @@ Layout make_layout(const Program& p, const gs_sim_opts& o) {
     L.trace = take((size_t)o.trace_cycles * p.n_po * o.n_trace_words * 8);
     L.lane_sigs = take((size_t)o.lanes * 8);
     L.scratch = take((size_t)p.n_po * words * 8);
+    L.lv_gate0 = take(d.lv_gate0.size() * 4);
+    L.lv_item0 = take(d.lv_item0.size() * 4);
+    L.dfctl_bytes = d.nl ? 4 + (size_t)d.n_slabs * d.nl * 4 : 0;
+    L.dfctl = take(L.dfctl_bytes);
     L.total = off;
     return L;
 }
@@ -76,6 +118,10 @@ struct gs_sim {
     void* host_stage = nullptr;       // library-owned device copy of host stimulus
     size_t host_stage_bytes = 0;
     cudaGraphExec_t exec[2] = {nullptr, nullptr};
+    DfPlan df;
+    uint32_t df_grid = 0;
+    uint32_t pdl = 1;                 // programmatic dependent launch between cycle kernels
+    uint32_t min_warps = 0;           // kernel A auto-U threshold (2 waves of resident warps)
 
     Ctl* ctl() const { return reinterpret_cast<Ctl*>(ws + L.ctl); }
     uint8_t* state() const { return ws + L.state; }
@@ -106,6 +152,8 @@ static LevelArgs level_args(const gs_sim* s, uint32_t l, uint32_t parity) {
     a.qcur = parity ? p.n_reg : 0;
     a.qnext = parity ? 0 : p.n_reg;
     a.ctl = s->ctl();
+    a.pdl = s->pdl;
+    a.min_warps = s->min_warps;
     return a;
 }
 
@@ -129,6 +177,7 @@ static EndArgs end_args(const gs_sim* s, uint32_t parity) {
     e.trace = (s->opts.n_trace_words && s->opts.trace_cycles) ? s->at<unsigned long long>(s->L.trace) : nullptr;
     e.ntw = s->opts.n_trace_words;
     e.trace_cap = s->opts.trace_cycles;
+    e.pdl = s->pdl;
     return e;
 }
 
@@ -151,12 +200,48 @@ static cudaError_t level_launch(const gs_sim* s, uint32_t l, uint32_t parity, cu
     }
 }
 
+static cudaError_t dataflow_launch(const gs_sim* s, uint32_t parity, cudaStream_t st) {
+    const Program& p = *s->prog;
+    const DfPlan& d = s->df;
+    DfArgs a{};
+    a.din = s->at<const uint4>(s->L.din);
+    a.aux = s->at<const GateAux>(s->L.aux);
+    a.dhi = p.any_wide ? s->at<const uint2>(s->L.dhi) : nullptr;
+    a.state = s->state();
+    a.stride = s->stride;
+    a.row_gate0 = p.row_gate0;
+    a.qcur = parity ? p.n_reg : 0;
+    a.qnext = parity ? 0 : p.n_reg;
+    a.lv_gate0 = s->at<const uint32_t>(s->L.lv_gate0);
+    a.lv_item0 = s->at<const uint32_t>(s->L.lv_item0);
+    a.nl = d.nl;
+    a.items_per_slab = d.lv_item0.back();
+    a.n_slabs = d.n_slabs;
+    a.interleave = d.interleave;
+    a.slab_vec = 32 * d.vpl;
+    a.gpw = d.gpw;
+    a.total_items = a.items_per_slab * d.n_slabs;
+    a.qhead = s->at<unsigned int>(s->L.dfctl);
+    a.done = a.qhead + 1;
+    if (!d.nl) return cudaSuccess;
+    cudaError_t e = cudaMemsetAsync(a.qhead, 0, s->L.dfctl_bytes, st);
+    if (e != cudaSuccess) return e;
+    return launch_dataflow(a, s->df_grid, st);
+}
+
 static cudaError_t cycle_launches(const gs_sim* s, uint32_t parity, cudaStream_t st,
                                   std::vector<cudaEvent_t>* evs = nullptr) {
     const Program& p = *s->prog;
     cudaError_t e = launch_stim(s->ctl(), s->state(), s->stride, s->words, p.row_pi0, p.n_pi,
-                                s->opts.lane_offset / 64, st);
+                                s->opts.lane_offset / 64, s->pdl, st);
     if (e != cudaSuccess) return e;
+    if (s->opts.kernel == GS_KERNEL_DATAFLOW) {
+        if (evs) cudaEventRecord((*evs)[0], st);
+        e = dataflow_launch(s, parity, st);
+        if (evs) cudaEventRecord((*evs)[1], st);
+        if (e != cudaSuccess) return e;
+        return launch_end_cycle(end_args(s, parity), st);
+    }
     // slab-major order: every level on lanes [slab], then the next slab (lanes are
     // independent; a slab's recent levels fit L2)
     for (uint32_t sl = 0; sl < s->slabs; ++sl)
@@ -211,7 +296,9 @@ gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts
     if (!prog || !opts || !bytes) return fail(GS_ERR_ARG, "gs_sim_workspace_bytes: NULL argument");
     if (opts->lanes == 0 || opts->lanes % 64) return fail(GS_ERR_ARG, "lanes must be a positive multiple of 64");
     if (opts->lanes / 64 >= (1ull << 31)) return fail(GS_ERR_ARG, "too many lanes");
-    *bytes = make_layout(*prog->p, *opts).total;
+    DfPlan d;
+    if (gs_status st = df_plan(*prog->p, *opts, d)) return st;
+    *bytes = make_layout(*prog->p, *opts, d).total;
     clear_error();
     return GS_OK;
 }
@@ -220,14 +307,16 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts, void* d
     if (!prog || !opts || !out || !dev_ws) return fail(GS_ERR_ARG, "gs_sim_create: NULL argument");
     if (opts->lanes == 0 || opts->lanes % 64) return fail(GS_ERR_ARG, "gs_sim_create: lanes must be a positive multiple of 64");
     if (opts->lane_offset % 64) return fail(GS_ERR_ARG, "gs_sim_create: lane_offset must be a multiple of 64");
-    if (opts->kernel < GS_KERNEL_AUTO || opts->kernel > GS_KERNEL_AB) return fail(GS_ERR_ARG, "gs_sim_create: bad kernel");
+    if (opts->kernel < GS_KERNEL_AUTO || opts->kernel > GS_KERNEL_DATAFLOW) return fail(GS_ERR_ARG, "gs_sim_create: bad kernel");
     if (opts->n_trace_words && !opts->trace_words) return fail(GS_ERR_ARG, "gs_sim_create: trace_words is NULL");
     if ((reinterpret_cast<uintptr_t>(dev_ws) & 255) != 0) return fail(GS_ERR_ARG, "gs_sim_create: workspace must be 256-byte aligned");
     const Program& p = *prog->p;
     const uint32_t words = (uint32_t)(opts->lanes / 64);
     for (uint32_t i = 0; i < opts->n_trace_words; ++i)
         if (opts->trace_words[i] >= words) return fail(GS_ERR_ARG, "gs_sim_create: trace word out of range");
-    Layout L = make_layout(p, *opts);
+    DfPlan plan;
+    if (gs_status st = df_plan(p, *opts, plan)) return st;
+    Layout L = make_layout(p, *opts, plan);
     if (bytes < L.total) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_create: workspace smaller than gs_sim_workspace_bytes");
     CU(cudaSetDevice(opts->device));
     gs_sim* s = new gs_sim();
@@ -241,7 +330,14 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts, void* d
     s->stream = static_cast<cudaStream_t>(opts->stream);
     s->words = words;
     s->stride = (uint64_t)words * 8;
-    s->slabs = opts->lane_slabs ? opts->lane_slabs : 1;
+    s->df = plan;
+    s->pdl = (opts->flags & GS_SIM_NO_PDL) ? 0u : 1u;
+    {
+        int sms = 148;
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, opts->device);
+        s->min_warps = (uint32_t)sms * 32u * 2u;   // 4 CTAs x 8 warps per SM, two waves
+    }
+    s->slabs = (opts->lane_slabs && s->opts.kernel != GS_KERNEL_DATAFLOW) ? opts->lane_slabs : 1;
     if (s->slabs > 1) {
         const uint32_t vrow = words / 2;
         if (s->opts.kernel != GS_KERNEL_LUT || words % 2 || vrow % s->slabs || (vrow / s->slabs) % 32) {
@@ -256,13 +352,21 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts, void* d
         delete s;
         return st;
     };
-    cudaError_t e = cudaStreamCreateWithFlags(&s->cap, cudaStreamNonBlocking);
+    cudaError_t e = cudaSuccess;
+    if (s->opts.kernel == GS_KERNEL_DATAFLOW) {
+        e = dataflow_grid(32 * plan.vpl, opts->device, &s->df_grid);
+        if (e != cudaSuccess) {
+            delete s;
+            return fail(GS_ERR_CUDA, std::string("dataflow occupancy: ") + cudaGetErrorString(e));
+        }
+    }
+    e = cudaStreamCreateWithFlags(&s->cap, cudaStreamNonBlocking);
     if (e != cudaSuccess) return cleanup(fail(GS_ERR_CUDA, std::string("cudaStreamCreate: ") + cudaGetErrorString(e)));
     // upload the program (descriptors are device-resident for the sim's lifetime)
     struct Up { size_t off; const void* src; size_t n; };
     std::vector<int32_t> slot(words, -1);
     for (uint32_t i = 0; i < opts->n_trace_words; ++i) slot[opts->trace_words[i]] = (int32_t)i;
-    const bool poly = s->opts.kernel != GS_KERNEL_LUT;
+    const bool poly = s->opts.kernel == GS_KERNEL_POLY || s->opts.kernel == GS_KERNEL_AB;
     std::vector<Up> ups = {
         {L.din, p.in_lo.data(), p.in_lo.size() * 4},
         {L.aux, p.aux.data(), p.aux.size() * sizeof(GateAux)},
@@ -274,6 +378,8 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts, void* d
         {L.latch_dst, p.latch_dst.data(), p.latch_dst.size() * 4},
         {L.reg_init, p.reg_init.data(), p.reg_init.size()},
         {L.trace_slot, slot.data(), slot.size() * 4},
+        {L.lv_gate0, plan.lv_gate0.data(), plan.lv_gate0.size() * 4},
+        {L.lv_item0, plan.lv_item0.data(), plan.lv_item0.size() * 4},
     };
     for (const Up& u : ups) {
         if (!u.n) continue;
@@ -512,7 +618,8 @@ gs_status gs_sim_launches_per_cycle(const gs_sim* s, uint64_t* launches) {
     for (uint32_t l = 0; l < p.n_levels; ++l)
         if (p.level_off[l + 1] > p.level_off[l]) lv++;
     const uint64_t per_level = s->opts.kernel == GS_KERNEL_AB ? 2 : 1;
-    *launches = (p.n_pi ? 1 : 0) + lv * per_level * s->slabs + 1;
+    if (s->opts.kernel == GS_KERNEL_DATAFLOW) lv = s->df.nl ? 1 : 0, *launches = (p.n_pi ? 1 : 0) + lv + 1;
+    else *launches = (p.n_pi ? 1 : 0) + lv * per_level * s->slabs + 1;
     return GS_OK;
 }
 
@@ -524,7 +631,8 @@ gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
         return fail(GS_ERR_STATE, "gs_sim_profile_step: stepping past the bound stimulus cycles");
     const Program& p = *s->prog;
     CU(cudaSetDevice(s->opts.device));
-    std::vector<cudaEvent_t> evs(2 * (size_t)p.n_levels * s->slabs);
+    std::vector<cudaEvent_t> evs(std::max<size_t>(2, 2 * (size_t)p.n_levels * s->slabs));
+    const bool df = s->opts.kernel == GS_KERNEL_DATAFLOW;
     cudaEvent_t e0, e1;
     for (auto& e : evs) CU(cudaEventCreate(&e));
     CU(cudaEventCreate(&e0));
@@ -551,6 +659,12 @@ gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
         float ms = 0;
         cudaEventElapsedTime(&ms, e0, e1);
         total_ms += ms;
+        if (df) {                      // one persistent launch covers every level
+            cudaEventElapsedTime(&ms, evs[0], evs[1]);
+            level_ms += ms;
+            for (uint32_t l = 0; l < p.n_levels; ++l) level_bytes += lb[l];
+            lvl_launches += s->df.nl ? 1 : 0;
+        } else
         for (uint32_t sl = 0; sl < s->slabs; ++sl)
             for (uint32_t l = 0; l < p.n_levels; ++l) {
                 if (p.level_off[l + 1] == p.level_off[l]) continue;

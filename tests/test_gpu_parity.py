@@ -29,10 +29,10 @@ def gpu_trace_bits(tr, words_sel):
 
 
 def run_gpu(nl, lanes, cycles, kernel="lut", seed=None, host_stim=None, trace_words=(),
-            lane_offset=0, balance=True, use_graphs=True, prog=None):
+            lane_offset=0, balance=True, use_graphs=True, prog=None, **simkw):
     prog = prog or compile_nl(nl, balance)
     sim = gs.Sim(prog, lanes, lane_offset=lane_offset, kernel=kernel, trace_words=trace_words,
-                 trace_cycles=cycles if len(trace_words) else 0, use_graphs=use_graphs)
+                 trace_cycles=cycles if len(trace_words) else 0, use_graphs=use_graphs, **simkw)
     if host_stim is not None:
         sim.bind_host(host_stim)
     else:
@@ -283,6 +283,52 @@ def test_errors_on_device():
     sim.close()
 
 
+# ------------------------------------------------------------------ DATAFLOW schedule
+DF_CASES = [  # (lanes, lane_slabs, interleave, gates per warp)
+    (4096, 0, 0, 0), (8192, 0, 1, 1), (16384, 0, 3, 7), (16384, 2, 2, 4), (32768, 2, 1, 32),
+    (65536, 4, 2, 2)]
+
+
+@pytest.mark.parametrize("lanes,slabs,inter,gpw", DF_CASES)
+def test_dataflow_equals_lut_and_oracle_c3(lanes, slabs, inter, gpw):
+    """Kernel D (one persistent launch per cycle, slab dataflow) == kernel A == oracle."""
+    cfg = workloads.CONFIGS["C3"]
+    nl = cfg.netlist()
+    prog = compile_nl(nl)
+    W_ = lanes // 64
+    tw = [0, W_ // 3, W_ - 1]
+    cycles = 24
+    d = run_gpu(nl, lanes, cycles, "df", seed=7, prog=prog, trace_words=tw, lane_slabs=slabs,
+                df_interleave=inter, df_gates_per_warp=gpw)
+    a = run_gpu(nl, lanes, cycles, "lut", seed=7, prog=prog)
+    for key in ("outputs", "regs", "sigs"):
+        assert np.array_equal(d[key], a[key]), key
+    assert d["signature"]["lane_sig_sum"] == a["signature"]["lane_sig_sum"]
+    sample = np.array([0, 1, 63, (W_ // 3) * 64 + 9, lanes - 64, lanes - 1])
+    sampled_lane_check(nl, d, sample, 0, cycles, 7, tw)
+
+
+@pytest.mark.parametrize("balance", [False, True])
+def test_dataflow_unbalanced_wide_gates_and_registers_all_lanes(balance):
+    """k up to 6, register edge cases, unbalanced levels: every lane vs the oracle."""
+    nls = [workloads.random_tiny(s, n_pi=6, n_reg=5, n_gates=300, n_po=12, max_k=6) for s in (3, 4)]
+    nls.append(workloads.register_edge_cases())
+    for nl in nls:
+        r = run_gpu(nl, 4096, 9, "df", seed=11, balance=balance)
+        o = oracle.simulate(nl, np.arange(4096), 9, seed=11, want=("last", "regs", "sig"))
+        assert np.array_equal(gs.unpack_lanes(r["outputs"]).T, o["last"])
+        assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"])
+        assert np.array_equal(r["sigs"], o["sig"])
+
+
+def test_dataflow_rejects_bad_slab_sizes():
+    prog = compile_nl(workloads.adder(8))
+    for lanes, slabs in ((2048, 0), (8192, 3), (65536, 2)):
+        with pytest.raises(gs.GsError) as e:
+            gs.Sim(prog, lanes, kernel="df", lane_slabs=slabs)
+        assert e.value.code == gs.GS_ERR_ARG
+
+
 # ------------------------------------------------------------------ full-size configs
 @pytest.mark.slow
 def test_c4_full_config_sampled_lanes_and_probes():
@@ -294,6 +340,20 @@ def test_c4_full_config_sampled_lanes_and_probes():
     sample = np.array([0, 63, 64, 127, W_ // 2 * 64 + 17, cfg.lanes - 64, cfg.lanes - 1])
     sampled_lane_check(nl, r, sample, 0, cfg.cycles, cfg.stim_seed, tw)
     probe_closed_forms(nl, gs.unpack_lanes(r["outputs"]).T, cfg.cycles - 1, cfg.stim_seed, cfg.lanes)
+
+
+@pytest.mark.slow
+def test_c4_full_config_dataflow_bench_launch_config():
+    """C4 at full size in the launch configuration bench.py times (kernel D defaults)."""
+    cfg = workloads.CONFIGS["C4"]
+    nl = cfg.netlist()
+    W_ = cfg.lanes // 64
+    tw = [0, 1, 63, 64, W_ // 2 + 3, W_ - 1]          # slab boundaries (4096 lanes = 64 words)
+    cycles = 200
+    r = run_gpu(nl, cfg.lanes, cycles, "df", seed=cfg.stim_seed, trace_words=tw)
+    sample = np.array([0, 63, 64, 4095, 4096, (W_ // 2 + 3) * 64 + 33, cfg.lanes - 64, cfg.lanes - 1])
+    sampled_lane_check(nl, r, sample, 0, cycles, cfg.stim_seed, tw)
+    probe_closed_forms(nl, gs.unpack_lanes(r["outputs"]).T, cycles - 1, cfg.stim_seed, cfg.lanes)
 
 
 @pytest.mark.slow
