@@ -43,7 +43,9 @@ def parse():
     ap.add_argument("--config", default="C4")
     ap.add_argument("--cycles-per-step", type=int, default=100)
     ap.add_argument("--lanes", type=int, default=0, help="override lanes per GPU")
-    ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab", "df"])
+    ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab", "df", "tile"])
+    ap.add_argument("--tile-words", type=int, default=0, help="kernel T: 32-bit words per slot")
+    ap.add_argument("--tile-groups", type=int, default=0, help="kernel T: thread groups per CTA")
     ap.add_argument("--df-interleave", type=int, default=0, help="kernel D: slabs walked together")
     ap.add_argument("--df-gpw", type=int, default=0, help="kernel D: gates per warp per item")
     ap.add_argument("--lane-slabs", type=int, default=0, help="L2 lane slabs (0 = library default)")
@@ -114,7 +116,7 @@ def peaks():
 
 
 KERNEL_NAMES = {"lut": "k_level_lut_wide<4>", "df": "k_dataflow<1>", "poly": "k_level_poly",
-                "ab": "k_level_lut_wide<4>"}
+                "ab": "k_level_lut_wide<4>", "tile": "k_tile"}
 
 
 def ncu_traffic(kernel: str):
@@ -229,7 +231,8 @@ def main():
     stream = torch.cuda.Stream(device=local)
     sim = gs.Sim(prog, lanes, lane_offset=lane_offset, kernel=args.kernel, device=local, stream=stream,
                  lane_slabs=args.lane_slabs, lut_unroll=args.lut_unroll,
-                 df_interleave=args.df_interleave, df_gates_per_warp=args.df_gpw, pdl=not args.no_pdl)
+                 df_interleave=args.df_interleave, df_gates_per_warp=args.df_gpw, pdl=not args.no_pdl,
+                 tile_words=args.tile_words, tile_groups=args.tile_groups)
     sim.bind_generated(cfg.stim_seed)
     C = args.cycles_per_step
     launches_per_cycle = sim.launches_per_cycle()
@@ -331,11 +334,12 @@ def main():
                        "cycles_per_step": C, "kernel": args.kernel, "balance": True,
                        "lane_slabs": args.lane_slabs, "lut_unroll": args.lut_unroll,
                        "df_interleave": args.df_interleave, "df_gpw": args.df_gpw,
-                       "pdl": not args.no_pdl,
+                       "pdl": not args.no_pdl, "tile_words": args.tile_words,
+                       "tile_groups": args.tile_groups,
                        "l2": "inputs larger than L2 (state %.1f GB per GPU)" % (info["n_rows"] * lanes / 8 / 1e9),
                        "parallelism": f"dp{world} (stimulus sharding)", "compile_s": round(compile_s, 2),
                        "paper_style_gcps": value * (G + info["n_reg"]) / G},
-            "gpu_launches": int(launches_per_cycle * C * args.steps),
+            "gpu_launches": int(launches_per_cycle * (1 if args.kernel == "tile" else C) * args.steps),
             "signature": {k: str(v) for k, v in red.items()},
             "clocks": clk,
             "roofline": roof,

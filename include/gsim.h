@@ -170,18 +170,30 @@ gs_status gs_program_gate_levels(const gs_program* prog, uint32_t* level, uint32
  * as compiled by the Möbius butterfly (Algorithm 1 in iterative form).  n >= 2^k. */
 gs_status gs_program_coeffs(const gs_program* prog, uint32_t gate, int32_t* w, uint32_t n);
 
+/* Shared-memory slots one lane tile of kernel T needs (constants, PIs, two register banks,
+ * gate values reused by live range; tile.cpp).  A tile of 32*w lanes needs
+ * (slots + 64) * 4 * w bytes of shared memory (<= 227 KB). */
+gs_status gs_program_tile_slots(const gs_program* prog, uint32_t* slots);
+
 /* ======================================================================= simulate */
 enum {
-    GS_KERNEL_AUTO = 0,   /* = GS_KERNEL_LUT                                               */
+    GS_KERNEL_AUTO = 0,   /* GS_KERNEL_TILE when one tile's live state and every gate
+                             descriptor fit shared memory, else GS_KERNEL_LUT             */
     GS_KERNEL_LUT = 1,    /* kernel A: bit-sliced LUT evaluation, 64 stimuli per word      */
     GS_KERNEL_POLY = 2,   /* kernel B: the paper's network, sum_S w_S Theta(sum x - |S| + 1)
                              per stimulus in int32, ballot-packed (Eq. 1-3)                */
     GS_KERNEL_AB = 3,     /* A writes, B recomputes every level and counts mismatches      */
-    GS_KERNEL_DATAFLOW = 4 /* kernel A evaluation in ONE persistent launch per cycle: lanes cut
+    GS_KERNEL_DATAFLOW = 4, /* kernel A evaluation in ONE persistent launch per cycle: lanes cut
                              into slabs, (slab, level, gate chunk) items from a work queue, an
                              item waits only for the previous level of its slab, so a slab's
                              recent levels are read from L2 (DESIGN.md §6 "kernel D").
-                             Needs lanes/lane_slabs in {4096, 8192, 16384}.                 */
+                             Needs lanes/lane_slabs in {4096, 8192, 16384}.  Experimental:
+                             measured slower than LUT on C2-C4.              */
+    GS_KERNEL_TILE = 5     /* kernel T: each CTA owns a tile of 32*tile_words lanes and runs
+                             every level of every cycle of a gs_sim_step in shared memory
+                             (gate values in slots reused by live range); one launch per
+                             step, HBM touched only for registers/MISR at step boundaries.
+                             Needs the live slots of one tile to fit shared memory.          */
 };
 
 typedef struct {
@@ -202,6 +214,10 @@ typedef struct {
     uint32_t df_interleave;       /* DATAFLOW: slabs walked level by level together (0 = 8) */
     uint32_t df_gates_per_warp;   /* DATAFLOW: gates per warp per work item, 1..32 (0 = 8) */
     uint32_t flags;               /* GS_SIM_* bits below                                   */
+    uint32_t tile_words;          /* TILE: 32-bit words per slot, lanes per tile = 32 * this
+                                     (4, 8, 16 or 32; 0 = auto); lanes % (32 * it) == 0   */
+    uint32_t tile_groups;         /* TILE: independent thread groups (tiles) per 512-thread
+                                     CTA, each with its own barrier (1, 2 or 4; 0 = auto)  */
 } gs_sim_opts;
 /* flags: launch the per-cycle kernels WITHOUT programmatic dependent launch (by default a
  * level kernel may become resident while its predecessor drains; A/B measurement only). */

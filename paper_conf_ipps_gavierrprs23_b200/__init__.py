@@ -26,7 +26,9 @@ GS_ERR_BUFFER_TOO_SMALL, GS_ERR_CUDA, GS_ERR_STATE, GS_ERR_NOMEM = -5, -6, -7, -
 GS_MAX_K = 6
 GS_SIM_NO_PDL = 1
 GS_KERNEL_AUTO, GS_KERNEL_LUT, GS_KERNEL_POLY, GS_KERNEL_AB, GS_KERNEL_DATAFLOW = 0, 1, 2, 3, 4
-KERNELS = {"auto": 0, "lut": 1, "A": 1, "poly": 2, "B": 2, "ab": 3, "AB": 3, "df": 4, "dataflow": 4}
+GS_KERNEL_TILE = 5
+KERNELS = {"auto": 0, "lut": 1, "A": 1, "poly": 2, "B": 2, "ab": 3, "AB": 3, "df": 4, "dataflow": 4,
+           "tile": 5, "T": 5}
 
 
 class GsError(RuntimeError):
@@ -72,7 +74,7 @@ class gs_sim_opts(C.Structure):
                 ("trace_words", C.c_void_p), ("trace_cycles", C.c_uint32), ("use_graphs", C.c_int),
                 ("lane_slabs", C.c_uint32), ("lut_unroll", C.c_uint32),
                 ("df_interleave", C.c_uint32), ("df_gates_per_warp", C.c_uint32),
-                ("flags", C.c_uint32)]
+                ("flags", C.c_uint32), ("tile_words", C.c_uint32), ("tile_groups", C.c_uint32)]
 
 
 class gs_signature(C.Structure):
@@ -110,6 +112,7 @@ _SIGS = {
     "gs_program_level_widths": (C.c_int32, [_P, _P, C.c_uint32]),
     "gs_program_gate_levels": (C.c_int32, [_P, _P, C.c_uint32]),
     "gs_program_coeffs": (C.c_int32, [_P, C.c_uint32, _P, C.c_uint32]),
+    "gs_program_tile_slots": (C.c_int32, [_P, _P]),
     "gs_sim_workspace_bytes": (C.c_int32, [_P, _P, _P]),
     "gs_sim_create": (C.c_int32, [_P, _P, _P, C.c_size_t, _P]),
     "gs_sim_destroy": (C.c_int32, [_P]),
@@ -257,6 +260,11 @@ class Program:
         _call("gs_program_gate_levels", self.h, _p(lv), len(lv))
         return lv[:self.info["n_gates"]]
 
+    def tile_slots(self) -> int:
+        v = C.c_uint32()
+        _call("gs_program_tile_slots", self.h, C.byref(v))
+        return v.value
+
     def coeffs(self, gate: int, k: int) -> list[int]:
         w = np.zeros(1 << k, dtype=np.int32)
         _call("gs_program_coeffs", self.h, gate, _p(w), len(w))
@@ -269,7 +277,8 @@ class Sim:
     def __init__(self, program: Program, lanes: int, lane_offset: int = 0, kernel="lut",
                  device: int = 0, stream=None, trace_words=(), trace_cycles: int = 0,
                  use_graphs: bool = True, lane_slabs: int = 0, lut_unroll: int = 0,
-                 df_interleave: int = 0, df_gates_per_warp: int = 0, pdl: bool = True):
+                 df_interleave: int = 0, df_gates_per_warp: int = 0, pdl: bool = True,
+                 tile_words: int = 0, tile_groups: int = 0, flags: int = 0):
         import torch
         self.program = program
         self.lanes, self.words = int(lanes), int(lanes) // 64
@@ -280,7 +289,8 @@ class Sim:
                         KERNELS[kernel] if isinstance(kernel, str) else int(kernel), len(self._tw),
                         _p(self._tw) if len(self._tw) else None, int(trace_cycles),
                         1 if use_graphs else 0, int(lane_slabs), int(lut_unroll),
-                        int(df_interleave), int(df_gates_per_warp), 0 if pdl else GS_SIM_NO_PDL)
+                        int(df_interleave), int(df_gates_per_warp),
+                        (0 if pdl else GS_SIM_NO_PDL) | int(flags), int(tile_words), int(tile_groups))
         nbytes = C.c_size_t()
         _call("gs_sim_workspace_bytes", program.h, C.byref(o), C.byref(nbytes))
         self.workspace = torch.empty(int(nbytes.value) + 256, dtype=torch.uint8, device=self.device)

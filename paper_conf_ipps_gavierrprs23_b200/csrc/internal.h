@@ -75,6 +75,28 @@ struct Program {
 
 gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out);
 
+// ---------------------------------------------------------------- kernel T plan
+// Shared-memory slots of one lane tile (tile.cpp): [const0, const1 | PI | Q bank 0 |
+// Q bank 1 | gate values, reused by live range].
+struct TileDesc {
+    uint32_t in01, in23;      // input slots (16 bits each; Q refs name the bank-0 slot)
+    uint32_t tt;              // truth table bits 15..0 | output slot << 16
+    uint32_t kreg;            // k | (fused-latch register index + 1) << 4
+};
+static_assert(sizeof(TileDesc) == 16, "TileDesc layout");
+
+struct TilePlan {
+    uint32_t n_slots = 0, q0 = 0;
+    std::vector<TileDesc> desc;         // [n_eval] exec order
+    std::vector<uint32_t> desc_hi;      // [n_eval][4] if any k > 4: in4|in5<<16, tt[47:16], tt[63:48], 0
+    std::vector<uint32_t> po_slot;      // [n_po]
+    std::vector<uint32_t> latch_src;    // slots (leftover latches)
+    std::vector<uint32_t> latch_dst;    // register index
+    std::vector<uint32_t> wb_row, wb_slot;   // PO values written back to state rows
+};
+
+gs_status tile_plan(const Program& p, TilePlan& t);
+
 // Möbius transform of one LSB-first truth table (Algorithm 1 as an iterative butterfly)
 void mobius_butterfly(uint64_t tt, uint32_t k, int32_t* w);
 

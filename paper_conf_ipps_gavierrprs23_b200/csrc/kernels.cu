@@ -20,109 +20,9 @@
 #include <cuda_runtime.h>
 
 #include "kernels.h"
+#include "device.cuh"
 
 namespace gs {
-
-#define FULL 0xFFFFFFFFu
-
-__device__ __forceinline__ uint32_t resolve(uint32_t ref, uint32_t qcur) {
-    // Q rows are referenced bank-0 relative with QFLAG; add the current bank offset
-    return (ref & 0x7FFFFFFFu) + ((ref >> 31) ? qcur : 0u);
-}
-
-// ----------------------------------------------------------------------------- hash
-// splitmix64 finaliser + the counter-based stimulus hash of DESIGN.md reading R2.
-__device__ __forceinline__ unsigned long long dmix64(unsigned long long z) {
-    z += 0x9E3779B97F4A7C15ULL;
-    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
-    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
-    return z ^ (z >> 31);
-}
-
-// ------------------------------------------------------- programmatic dependent launch
-// Every kernel of the per-cycle chain is launched with programmatic stream serialization
-// (when enabled): it may become resident while its predecessor drains, and waits at
-// griddepcontrol.wait until the predecessor has completed and its writes are visible.
-// It immediately allows its own successor to launch.  Without the launch attribute both
-// instructions are no-ops, so the kernels are correct either way.
-__device__ __forceinline__ void pdl_entry() {
-    asm volatile("griddepcontrol.wait;" ::: "memory");
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-}
-
-template <typename... KArgs, typename... Args>
-static cudaError_t launch_k(void (*kern)(KArgs...), uint32_t blocks, cudaStream_t s, uint32_t pdl,
-                            Args... args) {
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(blocks);
-    cfg.blockDim = dim3(256);
-    cfg.stream = s;
-    cudaLaunchAttribute at[1];
-    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    at[0].val.programmaticStreamSerializationAllowed = 1;
-    cfg.attrs = pdl ? at : nullptr;
-    cfg.numAttrs = pdl ? 1 : 0;
-    return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
-}
-
-// ------------------------------------------------------------------ kernel A: LUT
-// Bit-sliced Shannon expansion of an LSB-first truth table: stage 0 selects between
-// the minterm constants with x_0, stage i muxes pairs with x_i.  All operands are
-// 32-bit so every mux is one LOP3.
-template <int K>
-__device__ __forceinline__ uint32_t lut_eval(uint64_t tt, const uint32_t* x);
-
-// K = 5, 6: Shannon-expand on the top variables over 16-entry sub-tables, one at a
-// time, so the register footprint stays that of K = 4 (keeps occupancy up).
-template <int K>
-__device__ __forceinline__ uint32_t lut_eval_wide(uint64_t tt, const uint32_t* x) {
-    uint32_t y[4];
-#pragma unroll 1
-    for (int j = 0; j < (1 << (K - 4)); ++j) y[j] = lut_eval<4>(tt >> (16 * j), x);
-    if (K == 5) return (x[4] & y[1]) | (~x[4] & y[0]);
-    const uint32_t lo = (x[4] & y[1]) | (~x[4] & y[0]);
-    const uint32_t hi = (x[4] & y[3]) | (~x[4] & y[2]);
-    return (x[5] & hi) | (~x[5] & lo);
-}
-
-template <int K>
-__device__ __forceinline__ uint32_t lut_eval(uint64_t tt, const uint32_t* x) {
-    if (K > 4) return lut_eval_wide<K>(tt, x);
-    constexpr int KK = K > 4 ? 4 : K;
-    uint32_t v[1 << (KK - 1)];
-#pragma unroll
-    for (int j = 0; j < (1 << (KK - 1)); ++j) {
-        const uint32_t c0 = 0u - (uint32_t)((tt >> (2 * j)) & 1u);
-        const uint32_t c1 = 0u - (uint32_t)((tt >> (2 * j + 1)) & 1u);
-        v[j] = (x[0] & c1) | (~x[0] & c0);
-    }
-#pragma unroll
-    for (int i = 1; i < KK; ++i) {
-#pragma unroll
-        for (int j = 0; j < (1 << (KK - 1 - i)); ++j) v[j] = (x[i] & v[2 * j + 1]) | (~x[i] & v[2 * j]);
-    }
-    return v[0];
-}
-
-// evaluate 4 x 32-bit lanes-words (one 16-byte vector) of a K-input gate
-template <int K>
-__device__ __forceinline__ uint4 lut_eval4(uint64_t tt, const uint4* xv) {
-    uint4 y;
-    uint32_t x[K];
-#pragma unroll
-    for (int i = 0; i < K; ++i) x[i] = xv[i].x;
-    y.x = lut_eval<K>(tt, x);
-#pragma unroll
-    for (int i = 0; i < K; ++i) x[i] = xv[i].y;
-    y.y = lut_eval<K>(tt, x);
-#pragma unroll
-    for (int i = 0; i < K; ++i) x[i] = xv[i].z;
-    y.z = lut_eval<K>(tt, x);
-#pragma unroll
-    for (int i = 0; i < K; ++i) x[i] = xv[i].w;
-    y.w = lut_eval<K>(tt, x);
-    return y;
-}
 
 template <int K>
 __device__ __forceinline__ void lut_gate_vec16(const LevelArgs& a, uint32_t gate, uint4 in, uint32_t v,

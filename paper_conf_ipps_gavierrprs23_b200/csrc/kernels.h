@@ -81,6 +81,41 @@ struct DfArgs {
     unsigned int* done;               // [n_slabs * nl] finished items (zeroed every cycle)
 };
 
+// Kernel T (kernels_tile.cu): one lane tile per CTA at a time, all levels x all cycles of
+// a step in shared memory (slots of tile.cpp); descriptors resident in shared memory
+// when they fit.
+struct TileArgs {
+    const TileDesc* desc;             // [n_eval]
+    const uint4* desc_hi;             // [n_eval] (k > 4 only)
+    const uint32_t* level_off;        // [n_levels + 1]
+    uint32_t n_eval, n_levels;
+    uint32_t desc_smem;               // 1: copy desc + level_off into shared memory once
+    const uint32_t* po_slot;
+    uint32_t n_po;
+    const uint32_t* latch_src;
+    const uint32_t* latch_dst;
+    uint32_t n_latch;
+    const uint32_t* wb_row;
+    const uint32_t* wb_slot;
+    uint32_t n_wb;
+    uint32_t n_pi, n_reg, q0, n_slots;
+    uint8_t* state;
+    uint32_t words;                   // 64-bit words per state row (lanes / 64)
+    uint32_t row_q0;
+    Ctl* ctl;
+    unsigned long long* misr;         // [64][words]
+    const int32_t* trace_slot;
+    unsigned long long* trace;
+    uint32_t ntw, trace_cap;
+    uint64_t word_off;                // global 64-bit word of local lane 0
+    uint32_t ncycles, n_tiles;
+};
+size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
+                       int desc_smem);
+cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
+                       int desc_smem, uint32_t has_q, uint32_t* per_sm);
+cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s);
+
 cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s);
 cudaError_t launch_dataflow(const DfArgs& a, uint32_t grid, cudaStream_t s);
 cudaError_t dataflow_grid(uint32_t slab_vec, int device, uint32_t* grid);

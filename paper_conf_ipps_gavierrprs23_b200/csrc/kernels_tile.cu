@@ -1,0 +1,258 @@
+// kernels_tile.cu — kernel T: tile-resident simulation in shared memory (sm_100a).
+//
+// Stimuli are independent, so a tile of 32*TW lanes can run every level of
+// every cycle of a step without ever synchronising with another tile.  One CTA owns a
+// tile at a time: its live state (slots of tile.cpp: constants, PIs, both register
+// banks, gate values by live range) sits in shared memory as TW 32-bit words per slot,
+// and each level (one merged NN layer) is one pass of the CTA over
+// (gate, word) units separated by __syncthreads.  HBM sees only the register rows and
+// MISR planes at the start and end of a step: no per-level launch, no per-level round
+// trip through HBM.  Narrow, deep circuits (the 32x32 multiplier has 184 levels of median
+// width 28) are latency-bound per tile, so many tiles run per SM at once.
+//
+// Semantics are exactly kernel A's: the same PI hash (R2), the same double-buffered
+// latch (R3), outputs sampled before the latch (R4), the same bit-sliced MISR (R5), so
+// lane signatures, outputs, registers and the trace are bit-identical.
+#include <cuda_runtime.h>
+
+#include "device.cuh"
+#include "kernels.h"
+
+namespace gs {
+
+constexpr uint32_t TILE_CTA = 512;                   // threads per CTA (one CTA per SM)
+constexpr unsigned long long TILE_MISR_POLY = 0x42F0E1EBA9EA3693ULL;   // CRC-64/ECMA-182
+
+// Shared memory: [desc: 16 B x n_eval (if desc_smem)] [level_off: 4 B x (n_levels + 1),
+// padded to 16 B] then per thread group: [slots: n_slots x TW words] [MISR: 64 x TW words].
+size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
+                       int desc_smem) {
+    size_t b = desc_smem ? (size_t)n_eval * 16 + (((size_t)n_levels + 1) * 4 + 15) / 16 * 16 : 0;
+    return b + (size_t)ng * ((size_t)n_slots + 64) * 4 * tw;
+}
+
+// One gate on one 16-byte group (4 words = 128 lanes) of its slots.  HASQ: the circuit has
+// registers, so an input slot may name a bank-0 register slot that must be moved to the
+// current bank.
+template <int K, bool HASQ>
+__device__ __forceinline__ void tile_gate(uint4* sl, uint32_t V, uint32_t v, const uint4& d, const uint4* desc_hi,
+                                          uint32_t g, uint32_t q0, uint32_t R, uint32_t qcur, uint32_t qnext) {
+    uint32_t s[6] = {d.x & 0xFFFFu, d.x >> 16, d.y & 0xFFFFu, d.y >> 16, 0u, 0u};
+    uint64_t tt = d.z & 0xFFFFu;
+    if (K > 4) {
+        const uint4 hi = __ldg(desc_hi + g);
+        s[4] = hi.x & 0xFFFFu;
+        s[5] = hi.x >> 16;
+        tt |= ((uint64_t)hi.y << 16) | ((uint64_t)hi.z << 48);
+    }
+    uint4 x[K];
+#pragma unroll
+    for (int i = 0; i < K; ++i) {
+        uint32_t si = s[i];
+        if (HASQ) si += (si - q0) < R ? qcur : 0u;
+        x[i] = sl[(size_t)si * V + v];
+    }
+    const uint4 y = lut_eval4<K>(tt, x);
+    sl[(size_t)(d.z >> 16) * V + v] = y;
+    if (HASQ) {
+        const uint32_t reg = d.w >> 4;
+        if (reg) sl[(size_t)(q0 + reg - 1 + qnext) * V + v] = y;      // fused latch
+    }
+}
+
+__device__ __forceinline__ void group_sync(uint32_t id, uint32_t nthreads) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
+// TW = 32-bit words per slot (tile = 32 * TW lanes).  A thread evaluates one gate on one
+// 16-byte group of 4 words (128 lanes): k 16-byte shared-memory loads, 4 x (2^k - 1) LOP3,
+// one 16-byte store.  The CTA (TILE_CTA threads) is split into NG independent groups; each
+// group simulates its own tile and synchronises only with itself (named barrier 1 + gid),
+// so one group's level barrier overlaps the other groups' work.  All groups share the
+// descriptor table in shared memory.
+template <int TW, bool HASQ, int NG>
+__global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
+    constexpr uint32_t V = TW / 4;                       // uint4 per slot
+    constexpr uint32_t GT = TILE_CTA / NG;               // threads per group
+    extern __shared__ uint4 smem[];
+    const uint4* dsm = a.desc_smem ? smem : reinterpret_cast<const uint4*>(a.desc);
+    const uint32_t* lvl = a.level_off;
+    uint4* base = smem;
+    if (a.desc_smem) {
+        uint32_t* lv = reinterpret_cast<uint32_t*>(smem + a.n_eval);
+        const uint4* gd = reinterpret_cast<const uint4*>(a.desc);
+        for (uint32_t i = threadIdx.x; i < a.n_eval; i += blockDim.x) smem[i] = __ldg(gd + i);
+        for (uint32_t i = threadIdx.x; i <= a.n_levels; i += blockDim.x) lv[i] = __ldg(a.level_off + i);
+        lvl = lv;
+        base = smem + a.n_eval + ((a.n_levels + 1) * 4 + 15) / 16;
+    }
+    __syncthreads();
+    const uint32_t gid = threadIdx.x / GT, tid = threadIdx.x % GT, bd = GT;
+    const uint32_t bar = 1 + gid;
+    uint4* sl = base + (size_t)gid * (a.n_slots + 64) * V;   // this group's slots
+    uint32_t* sw = reinterpret_cast<uint32_t*>(sl);          // slots as 32-bit words
+    uint32_t* mp = sw + (size_t)a.n_slots * TW;               // MISR planes [64][TW]
+    const unsigned long long c0 = a.ctl->cycle;
+    const uint32_t R = a.n_reg, q0 = a.q0;
+    const uint32_t w32_row = a.words * 2;                     // 32-bit words per state row
+    const uint32_t* st32 = reinterpret_cast<const uint32_t*>(a.state);
+    uint32_t* st32w = reinterpret_cast<uint32_t*>(a.state);
+    uint32_t* misr32 = reinterpret_cast<uint32_t*>(a.misr);
+    unsigned long long pop = 0;
+
+    for (uint32_t tile = blockIdx.x * NG + gid; tile < a.n_tiles; tile += gridDim.x * NG) {
+        const uint32_t t0 = tile * TW;                    // first 32-bit word of the tile (shard-local)
+        // ---- load: constants, both register banks, MISR planes
+        for (uint32_t u = tid; u < TW; u += bd) {
+            sw[u] = 0u;
+            sw[TW + u] = 0xFFFFFFFFu;
+        }
+        for (uint32_t u = tid; u < 2 * R * TW; u += bd) {
+            const uint32_t r = u / TW, w = u % TW;
+            sw[(size_t)(q0 + r) * TW + w] = st32[(uint64_t)(a.row_q0 + r) * w32_row + t0 + w];
+        }
+        for (uint32_t u = tid; u < 64 * TW; u += bd) {
+            const uint32_t j = u / TW, w = u % TW;
+            mp[u] = misr32[(uint64_t)j * w32_row + t0 + w];
+        }
+        group_sync(bar, GT);
+        for (uint32_t c = 0; c < a.ncycles; ++c) {
+            const unsigned long long cyc = c0 + c;
+            const uint32_t qcur = (cyc & 1) ? R : 0u, qnext = R - qcur;
+            // ---- primary inputs of this cycle (R2): one 64-bit hash per pair of words
+            for (uint32_t u = tid; u < a.n_pi * (TW / 2); u += bd) {
+                const uint32_t p = u / (TW / 2), w2 = u % (TW / 2);
+                const uint32_t g64 = (t0 >> 1) + w2;      // shard-local 64-bit word
+                unsigned long long v;
+                if (a.ctl->stim_mode == 0) {
+                    v = dmix64(dmix64(dmix64(a.ctl->seed ^ p) ^ cyc) ^ (a.word_off + g64));
+                } else {
+                    const unsigned long long* src = reinterpret_cast<const unsigned long long*>(a.ctl->stim_ptr);
+                    v = src[((cyc - a.ctl->stim_base) * a.n_pi + p) * a.words + g64];
+                }
+                reinterpret_cast<unsigned long long*>(sw + (size_t)(2 + p) * TW)[w2] = v;
+            }
+            group_sync(bar, GT);
+            // ---- levels: every (gate, 16-byte group) unit of the level, then a barrier
+            for (uint32_t l = 0; l < a.n_levels; ++l) {
+                const uint32_t g0 = lvl[l], n = (lvl[l + 1] - g0) * V;
+                for (uint32_t u = tid; u < n; u += bd) {
+                    const uint32_t gi = u / V, v = u % V;
+                    const uint32_t g = g0 + gi;
+                    const uint4 d = dsm[g];
+                    switch (d.w & 15u) {                       // k: warp-uniform except at k-group edges
+                        case 1: tile_gate<1, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
+                        case 2: tile_gate<2, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
+                        case 3: tile_gate<3, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
+                        case 4: tile_gate<4, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
+                        case 5: tile_gate<5, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
+                        default: tile_gate<6, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
+                    }
+                }
+                group_sync(bar, GT);
+            }
+            // ---- leftover latches into the next bank; MISR / popcount / trace of the POs
+            for (uint32_t u = tid; u < a.n_latch * V; u += bd) {
+                const uint32_t e = u / V, v = u % V;
+                uint32_t s = __ldg(a.latch_src + e);
+                s += (s - q0) < R ? qcur : 0u;
+                sl[(size_t)(q0 + __ldg(a.latch_dst + e) + qnext) * V + v] = sl[(size_t)s * V + v];
+            }
+            constexpr uint32_t NP = (64 * TW + GT - 1) / GT;    // MISR plane words per thread
+            uint32_t newp[NP];
+            const bool tr = a.trace && cyc < a.trace_cap;
+#pragma unroll
+            for (uint32_t i = 0; i < NP; ++i) {
+                const uint32_t u = tid + i * bd;
+                if (u >= 64 * TW) break;
+                const uint32_t j = u / TW, w = u % TW;
+                const uint32_t g32 = t0 + w;
+                const int32_t tslot = tr ? __ldg(a.trace_slot + (g32 >> 1)) : -1;
+                uint32_t vv = 0;
+                for (uint32_t o = j; o < a.n_po; o += 64) {
+                    uint32_t s = __ldg(a.po_slot + o);
+                    s += (s - q0) < R ? qcur : 0u;
+                    const uint32_t x = sw[(size_t)s * TW + w];
+                    vv ^= x;
+                    pop += __popc(x);
+                    if (tslot >= 0)
+                        reinterpret_cast<uint32_t*>(a.trace)[(((uint64_t)cyc * a.n_po + o) * a.ntw + tslot) * 2 +
+                                                             (g32 & 1)] = x;
+                }
+                const uint32_t prev = j ? mp[(j - 1) * TW + w] : 0u;
+                const uint32_t fb = ((TILE_MISR_POLY >> j) & 1ULL) ? mp[63 * TW + w] : 0u;
+                newp[i] = prev ^ fb ^ vv;
+            }
+            group_sync(bar, GT);
+#pragma unroll
+            for (uint32_t i = 0; i < NP; ++i)
+                if (tid + i * bd < 64 * TW) mp[tid + i * bd] = newp[i];
+            group_sync(bar, GT);
+        }
+        // ---- write back: both register banks, PO rows (read_outputs), MISR planes
+        for (uint32_t u = tid; u < 2 * R * TW; u += bd) {
+            const uint32_t r = u / TW, w = u % TW;
+            st32w[(uint64_t)(a.row_q0 + r) * w32_row + t0 + w] = sw[(size_t)(q0 + r) * TW + w];
+        }
+        for (uint32_t u = tid; u < a.n_wb * TW; u += bd) {
+            const uint32_t e = u / TW, w = u % TW;
+            st32w[(uint64_t)__ldg(a.wb_row + e) * w32_row + t0 + w] = sw[(size_t)__ldg(a.wb_slot + e) * TW + w];
+        }
+        for (uint32_t u = tid; u < 64 * TW; u += bd) {
+            const uint32_t j = u / TW, w = u % TW;
+            misr32[(uint64_t)j * w32_row + t0 + w] = mp[u];
+        }
+        group_sync(bar, GT);                              // before the next tile reuses smem
+    }
+    // ---- counters; the last CTA advances the device clock
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) pop += __shfl_xor_sync(FULL, pop, o);
+    if ((threadIdx.x & 31) == 0 && pop) atomicAdd(&a.ctl->popcount, pop);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        const unsigned int prev = atomicAdd(&a.ctl->done, 1u);
+        if (prev == gridDim.x - 1) {
+            a.ctl->done = 0u;
+            a.ctl->cycle = c0 + a.ncycles;
+            __threadfence();
+        }
+    }
+}
+
+// instantiations: TW in {4, 8, 16, 32} x registers present x groups {1, 2, 4}
+#define TILE_CASES_TW(T, CALL)                                                                        \
+    case T * 16 + 0: CALL(T, false, 1); break; case T * 16 + 1: CALL(T, false, 2); break;           \
+    case T * 16 + 2: CALL(T, false, 4); break;                                                       \
+    case T * 16 + 8: CALL(T, true, 1); break;  case T * 16 + 9: CALL(T, true, 2); break;            \
+    case T * 16 + 10: CALL(T, true, 4); break;
+#define TILE_SWITCH(TWV, Q, NGV, CALL)                                                                \
+    switch ((TWV) * 16 + ((Q) ? 8 : 0) + ((NGV) == 1 ? 0 : (NGV) == 2 ? 1 : (NGV) == 4 ? 2 : 7)) {  \
+        TILE_CASES_TW(4, CALL) TILE_CASES_TW(8, CALL) TILE_CASES_TW(16, CALL) TILE_CASES_TW(32, CALL)  \
+        default: return cudaErrorInvalidValue;                                                        \
+    }
+
+cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
+                       int desc_smem, uint32_t has_q, uint32_t* per_sm) {
+    const size_t smem = tile_smem_bytes(tw, ng, n_slots, n_eval, n_levels, desc_smem);
+    cudaError_t e = cudaSuccess;
+    int per = 0;
+#define TILE_PREP(T, Q, G)                                                                                        \
+    e = cudaFuncSetAttribute(k_tile<T, Q, G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);           \
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_tile<T, Q, G>, TILE_CTA, smem)
+    TILE_SWITCH(tw, has_q, ng, TILE_PREP)
+#undef TILE_PREP
+    *per_sm = (uint32_t)per;
+    return e;
+}
+
+cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s) {
+    if (a.n_tiles == 0 || a.ncycles == 0) return cudaSuccess;
+    const size_t smem = tile_smem_bytes(tw, ng, a.n_slots, a.n_eval, a.n_levels, a.desc_smem);
+#define TILE_LAUNCH(T, Q, G) k_tile<T, Q, G><<<grid, TILE_CTA, smem, s>>>(a)
+    TILE_SWITCH(tw, a.n_reg > 0, ng, TILE_LAUNCH)
+#undef TILE_LAUNCH
+    return cudaGetLastError();
+}
+
+}  // namespace gs

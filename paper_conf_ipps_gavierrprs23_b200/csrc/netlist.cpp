@@ -265,4 +265,13 @@ gs_status gs_program_coeffs(const gs_program* prog, uint32_t gate, int32_t* w, u
     return GS_OK;
 }
 
+gs_status gs_program_tile_slots(const gs_program* prog, uint32_t* slots) {
+    if (!prog || !slots) return fail(GS_ERR_ARG, "gs_program_tile_slots: NULL argument");
+    TilePlan t;
+    if (gs_status st = tile_plan(*prog->p, t)) return st;
+    *slots = t.n_slots;
+    clear_error();
+    return GS_OK;
+}
+
 }  // extern "C"

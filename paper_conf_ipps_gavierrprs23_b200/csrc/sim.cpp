@@ -23,7 +23,8 @@ size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 
 struct Layout {
     size_t ctl, state, din, aux, dhi, term_off, terms, po_rows, latch_src, latch_dst, reg_init,
-        trace_slot, misr, trace, lane_sigs, scratch, lv_gate0, lv_item0, dfctl, dfctl_bytes, total;
+        trace_slot, misr, trace, lane_sigs, scratch, lv_gate0, lv_item0, dfctl, dfctl_bytes,
+        t_desc, t_desc_hi, t_po, t_lsrc, t_ldst, t_wbrow, t_wbslot, t_lvl, total;
 };
 
 // Work-item plan of the DATAFLOW schedule (kernels.cu k_dataflow): non-empty levels only
@@ -63,7 +64,69 @@ gs_status df_plan(const Program& p, const gs_sim_opts& o, DfPlan& d) {
     return GS_OK;
 }
 
-Layout make_layout(const Program& p, const gs_sim_opts& o, const DfPlan& d) {
+struct Plans {
+    DfPlan df;
+    TilePlan tile;
+    uint32_t tw = 0;                  // kernel T: 32-bit words per slot
+    uint32_t ng = 0;                  // kernel T: thread groups (tiles) per CTA
+    int desc_smem = 0;                // kernel T: descriptors resident in shared memory
+};
+
+constexpr size_t TILE_SMEM_MAX = 232448;   // 227 KB opt-in shared memory per CTA (sm_100a)
+
+gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
+    if (gs_status st = df_plan(p, o, pl.df)) return st;
+    if (o.kernel != GS_KERNEL_TILE) return GS_OK;
+    if (gs_status st = tile_plan(p, pl.tile)) return st;
+    auto smem = [&](uint32_t tw, uint32_t ng, int ds) {
+        return tile_smem_bytes(tw, ng, pl.tile.n_slots, p.n_eval, p.n_levels, ds);
+    };
+    int sms = 148;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, o.device);
+    if (o.tile_words && (o.tile_words != 4 && o.tile_words != 8 && o.tile_words != 16 && o.tile_words != 32))
+        return fail(GS_ERR_ARG, "TILE: tile_words must be 4, 8, 16 or 32");
+    if (o.tile_groups && (o.tile_groups != 1 && o.tile_groups != 2 && o.tile_groups != 4))
+        return fail(GS_ERR_ARG, "TILE: tile_groups must be 1, 2 or 4");
+    if (o.tile_words && o.lanes % (32ull * o.tile_words))
+        return fail(GS_ERR_ARG, "TILE: lanes must be a multiple of 32 * tile_words");
+    // choose (tile words, groups per CTA): descriptors resident if possible, then the most
+    // lanes in flight on the GPU (groups x tile lanes x SMs, capped by the batch), then
+    // fewer groups and wider tiles (measured best on C2: one group of 32 words)
+    uint64_t best = 0;
+    for (int ds : {1, 0}) {
+        for (uint32_t ng : {4u, 2u, 1u}) {
+            if (o.tile_groups && ng != o.tile_groups) continue;
+            for (uint32_t tw : {4u, 8u, 16u, 32u}) {
+                if (o.tile_words && tw != o.tile_words) continue;
+                if (o.lanes % (32ull * tw) || smem(tw, ng, ds) > TILE_SMEM_MAX) continue;
+                const uint64_t inflight = std::min<uint64_t>((uint64_t)ng * tw * 32 * sms, o.lanes);
+                const uint64_t score = (inflight << 8) | ((8 - ng) << 4) | tw;
+                if (score > best) { best = score; pl.tw = tw; pl.ng = ng; }
+            }
+        }
+        if (best) { pl.desc_smem = ds; break; }
+    }
+    if (!best) return fail(GS_ERR_ARG, "TILE: live state of a 128-lane tile exceeds shared memory (or lanes % 128)");
+    return GS_OK;
+}
+
+// GS_KERNEL_AUTO: kernel T when one tile's live state AND the whole descriptor table fit
+// shared memory (small, deep circuits: measured 1.8x kernel A on C2, 5.8x on C1), else
+// kernel A (large circuits are HBM-bound; kernel T cannot hold them).
+gs_sim_opts resolve_auto(const Program& p, const gs_sim_opts& o) {
+    gs_sim_opts r = o;
+    if (o.kernel != GS_KERNEL_AUTO) return r;
+    r.kernel = GS_KERNEL_TILE;
+    Plans pl;
+    const std::string saved = gs_last_error();
+    if (p.n_eval == 0 || make_plans(p, r, pl) != GS_OK || !pl.desc_smem) r.kernel = GS_KERNEL_LUT;
+    set_error(saved);
+    return r;
+}
+
+Layout make_layout(const Program& p, const gs_sim_opts& o, const Plans& pl) {
+    const DfPlan& d = pl.df;
+    const TilePlan& t = pl.tile;
     Layout L{};
     const uint64_t words = o.lanes / 64;
     const uint64_t stride = words * 8;
@@ -94,6 +157,14 @@ Layout make_layout(const Program& p, const gs_sim_opts& o, const DfPlan& d) {
     L.lv_item0 = take(d.lv_item0.size() * 4);
     L.dfctl_bytes = d.nl ? 4 + (size_t)d.n_slabs * d.nl * 4 : 0;
     L.dfctl = take(L.dfctl_bytes);
+    L.t_desc = take(t.desc.size() * sizeof(TileDesc));
+    L.t_desc_hi = take(t.desc_hi.size() * 4);
+    L.t_po = take(t.po_slot.size() * 4);
+    L.t_lsrc = take(t.latch_src.size() * 4);
+    L.t_ldst = take(t.latch_dst.size() * 4);
+    L.t_wbrow = take(t.wb_row.size() * 4);
+    L.t_wbslot = take(t.wb_slot.size() * 4);
+    L.t_lvl = take(pl.tw ? p.level_off.size() * 4 : 0);
     L.total = off;
     return L;
 }
@@ -120,6 +191,10 @@ struct gs_sim {
     cudaGraphExec_t exec[2] = {nullptr, nullptr};
     DfPlan df;
     uint32_t df_grid = 0;
+    TilePlan tile;
+    uint32_t tw = 0, tile_grid = 0;
+    int desc_smem = 0;
+    uint32_t tile_groups = 1;
     uint32_t pdl = 1;                 // programmatic dependent launch between cycle kernels
     uint32_t min_warps = 0;           // kernel A auto-U threshold (2 waves of resident warps)
 
@@ -229,6 +304,43 @@ static cudaError_t dataflow_launch(const gs_sim* s, uint32_t parity, cudaStream_
     return launch_dataflow(a, s->df_grid, st);
 }
 
+static cudaError_t tile_launch(const gs_sim* s, uint32_t ncycles, cudaStream_t st) {
+    const Program& p = *s->prog;
+    const TilePlan& t = s->tile;
+    TileArgs a{};
+    a.desc = s->at<const TileDesc>(s->L.t_desc);
+    a.desc_hi = s->at<const uint4>(s->L.t_desc_hi);
+    a.level_off = s->at<const uint32_t>(s->L.t_lvl);
+    a.n_eval = p.n_eval;
+    a.n_levels = p.n_levels;
+    a.desc_smem = (uint32_t)s->desc_smem;
+    a.po_slot = s->at<const uint32_t>(s->L.t_po);
+    a.n_po = p.n_po;
+    a.latch_src = s->at<const uint32_t>(s->L.t_lsrc);
+    a.latch_dst = s->at<const uint32_t>(s->L.t_ldst);
+    a.n_latch = (uint32_t)t.latch_src.size();
+    a.wb_row = s->at<const uint32_t>(s->L.t_wbrow);
+    a.wb_slot = s->at<const uint32_t>(s->L.t_wbslot);
+    a.n_wb = (uint32_t)t.wb_row.size();
+    a.n_pi = p.n_pi;
+    a.n_reg = p.n_reg;
+    a.q0 = t.q0;
+    a.n_slots = t.n_slots;
+    a.state = s->state();
+    a.words = s->words;
+    a.row_q0 = p.row_q0;
+    a.ctl = s->ctl();
+    a.misr = s->at<unsigned long long>(s->L.misr);
+    a.trace_slot = s->at<const int32_t>(s->L.trace_slot);
+    a.trace = (s->opts.n_trace_words && s->opts.trace_cycles) ? s->at<unsigned long long>(s->L.trace) : nullptr;
+    a.ntw = s->opts.n_trace_words;
+    a.trace_cap = s->opts.trace_cycles;
+    a.word_off = s->opts.lane_offset / 64;
+    a.ncycles = ncycles;
+    a.n_tiles = (uint32_t)(s->opts.lanes / (32ull * s->tw));
+    return launch_tile(a, s->tw, s->tile_groups, s->tile_grid, st);
+}
+
 static cudaError_t cycle_launches(const gs_sim* s, uint32_t parity, cudaStream_t st,
                                   std::vector<cudaEvent_t>* evs = nullptr) {
     const Program& p = *s->prog;
@@ -296,33 +408,36 @@ gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts
     if (!prog || !opts || !bytes) return fail(GS_ERR_ARG, "gs_sim_workspace_bytes: NULL argument");
     if (opts->lanes == 0 || opts->lanes % 64) return fail(GS_ERR_ARG, "lanes must be a positive multiple of 64");
     if (opts->lanes / 64 >= (1ull << 31)) return fail(GS_ERR_ARG, "too many lanes");
-    DfPlan d;
-    if (gs_status st = df_plan(*prog->p, *opts, d)) return st;
-    *bytes = make_layout(*prog->p, *opts, d).total;
+    const gs_sim_opts o = resolve_auto(*prog->p, *opts);
+    Plans pl;
+    if (gs_status st = make_plans(*prog->p, o, pl)) return st;
+    *bytes = make_layout(*prog->p, o, pl).total;
     clear_error();
     return GS_OK;
 }
 
-gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts, void* dev_ws, size_t bytes, gs_sim** out) {
-    if (!prog || !opts || !out || !dev_ws) return fail(GS_ERR_ARG, "gs_sim_create: NULL argument");
+gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void* dev_ws, size_t bytes, gs_sim** out) {
+    if (!prog || !opts_in || !out || !dev_ws) return fail(GS_ERR_ARG, "gs_sim_create: NULL argument");
+    const gs_sim_opts resolved = resolve_auto(*prog->p, *opts_in);
+    const gs_sim_opts* opts = &resolved;
     if (opts->lanes == 0 || opts->lanes % 64) return fail(GS_ERR_ARG, "gs_sim_create: lanes must be a positive multiple of 64");
     if (opts->lane_offset % 64) return fail(GS_ERR_ARG, "gs_sim_create: lane_offset must be a multiple of 64");
-    if (opts->kernel < GS_KERNEL_AUTO || opts->kernel > GS_KERNEL_DATAFLOW) return fail(GS_ERR_ARG, "gs_sim_create: bad kernel");
+    if (opts->kernel < GS_KERNEL_AUTO || opts->kernel > GS_KERNEL_TILE) return fail(GS_ERR_ARG, "gs_sim_create: bad kernel");
     if (opts->n_trace_words && !opts->trace_words) return fail(GS_ERR_ARG, "gs_sim_create: trace_words is NULL");
     if ((reinterpret_cast<uintptr_t>(dev_ws) & 255) != 0) return fail(GS_ERR_ARG, "gs_sim_create: workspace must be 256-byte aligned");
     const Program& p = *prog->p;
     const uint32_t words = (uint32_t)(opts->lanes / 64);
     for (uint32_t i = 0; i < opts->n_trace_words; ++i)
         if (opts->trace_words[i] >= words) return fail(GS_ERR_ARG, "gs_sim_create: trace word out of range");
-    DfPlan plan;
-    if (gs_status st = df_plan(p, *opts, plan)) return st;
-    Layout L = make_layout(p, *opts, plan);
+    Plans pls;
+    if (gs_status st = make_plans(p, *opts, pls)) return st;
+    const DfPlan& plan = pls.df;
+    Layout L = make_layout(p, *opts, pls);
     if (bytes < L.total) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_create: workspace smaller than gs_sim_workspace_bytes");
     CU(cudaSetDevice(opts->device));
     gs_sim* s = new gs_sim();
     s->prog = &p;
     s->opts = *opts;
-    if (s->opts.kernel == GS_KERNEL_AUTO) s->opts.kernel = GS_KERNEL_LUT;
     s->trace_words.assign(opts->trace_words, opts->trace_words + opts->n_trace_words);
     s->opts.trace_words = s->trace_words.data();
     s->L = L;
@@ -331,6 +446,9 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts, void* d
     s->words = words;
     s->stride = (uint64_t)words * 8;
     s->df = plan;
+    s->tile = pls.tile;
+    s->tw = pls.tw;
+    s->desc_smem = pls.desc_smem;
     s->pdl = (opts->flags & GS_SIM_NO_PDL) ? 0u : 1u;
     {
         int sms = 148;
@@ -360,6 +478,21 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts, void* d
             return fail(GS_ERR_CUDA, std::string("dataflow occupancy: ") + cudaGetErrorString(e));
         }
     }
+    if (s->opts.kernel == GS_KERNEL_TILE) {
+        uint32_t per = 0;
+        int sms = 148;
+        s->tile_groups = pls.ng;
+        e = tile_setup(s->tw, s->tile_groups, s->tile.n_slots, p.n_eval, p.n_levels, s->desc_smem, p.n_reg > 0,
+                       &per);
+        if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, opts->device);
+        if (e != cudaSuccess || per == 0) {
+            delete s;
+            return fail(e != cudaSuccess ? GS_ERR_CUDA : GS_ERR_ARG,
+                        std::string("TILE: kernel setup: ") + (e != cudaSuccess ? cudaGetErrorString(e) : "0 CTAs fit an SM"));
+        }
+        const uint32_t tiles = (uint32_t)(opts->lanes / (32ull * s->tw));
+        s->tile_grid = std::min<uint32_t>((tiles + s->tile_groups - 1) / s->tile_groups, per * (uint32_t)sms);
+    }
     e = cudaStreamCreateWithFlags(&s->cap, cudaStreamNonBlocking);
     if (e != cudaSuccess) return cleanup(fail(GS_ERR_CUDA, std::string("cudaStreamCreate: ") + cudaGetErrorString(e)));
     // upload the program (descriptors are device-resident for the sim's lifetime)
@@ -380,6 +513,14 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts, void* d
         {L.trace_slot, slot.data(), slot.size() * 4},
         {L.lv_gate0, plan.lv_gate0.data(), plan.lv_gate0.size() * 4},
         {L.lv_item0, plan.lv_item0.data(), plan.lv_item0.size() * 4},
+        {L.t_desc, s->tile.desc.data(), s->tile.desc.size() * sizeof(TileDesc)},
+        {L.t_desc_hi, s->tile.desc_hi.data(), s->tile.desc_hi.size() * 4},
+        {L.t_po, s->tile.po_slot.data(), s->tile.po_slot.size() * 4},
+        {L.t_lsrc, s->tile.latch_src.data(), s->tile.latch_src.size() * 4},
+        {L.t_ldst, s->tile.latch_dst.data(), s->tile.latch_dst.size() * 4},
+        {L.t_wbrow, s->tile.wb_row.data(), s->tile.wb_row.size() * 4},
+        {L.t_wbslot, s->tile.wb_slot.data(), s->tile.wb_slot.size() * 4},
+        {L.t_lvl, p.level_off.data(), s->tw ? p.level_off.size() * 4 : 0},
     };
     for (const Up& u : ups) {
         if (!u.n) continue;
@@ -485,6 +626,12 @@ gs_status gs_sim_step(gs_sim* s, uint32_t n) {
     if (s->bound == 2 && s->cycle + n > s->bound_base + s->bound_cycles)
         return fail(GS_ERR_STATE, "gs_sim_step: stepping past the bound stimulus cycles");
     CU(cudaSetDevice(s->opts.device));
+    if (s->opts.kernel == GS_KERNEL_TILE) {       // every cycle of the step in one launch
+        CU(tile_launch(s, n, s->stream));
+        s->cycle += n;
+        clear_error();
+        return GS_OK;
+    }
     for (uint32_t i = 0; i < n; ++i) {
         const uint32_t parity = (uint32_t)(s->cycle & 1);
         if (s->opts.use_graphs) {
@@ -618,7 +765,8 @@ gs_status gs_sim_launches_per_cycle(const gs_sim* s, uint64_t* launches) {
     for (uint32_t l = 0; l < p.n_levels; ++l)
         if (p.level_off[l + 1] > p.level_off[l]) lv++;
     const uint64_t per_level = s->opts.kernel == GS_KERNEL_AB ? 2 : 1;
-    if (s->opts.kernel == GS_KERNEL_DATAFLOW) lv = s->df.nl ? 1 : 0, *launches = (p.n_pi ? 1 : 0) + lv + 1;
+    if (s->opts.kernel == GS_KERNEL_TILE) *launches = 1;      // per gs_sim_step call, not per cycle
+    else if (s->opts.kernel == GS_KERNEL_DATAFLOW) lv = s->df.nl ? 1 : 0, *launches = (p.n_pi ? 1 : 0) + lv + 1;
     else *launches = (p.n_pi ? 1 : 0) + lv * per_level * s->slabs + 1;
     return GS_OK;
 }
@@ -631,6 +779,32 @@ gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
         return fail(GS_ERR_STATE, "gs_sim_profile_step: stepping past the bound stimulus cycles");
     const Program& p = *s->prog;
     CU(cudaSetDevice(s->opts.device));
+    if (s->opts.kernel == GS_KERNEL_TILE) {
+        // one launch runs all n cycles; "level" bytes are the same algorithmic gather model
+        cudaEvent_t a0, a1;
+        CU(cudaEventCreate(&a0));
+        CU(cudaEventCreate(&a1));
+        cudaEventRecord(a0, s->stream);
+        cudaError_t e = tile_launch(s, n, s->stream);
+        cudaEventRecord(a1, s->stream);
+        if (e == cudaSuccess) e = cudaEventSynchronize(a1);
+        float ms = 0;
+        if (e == cudaSuccess) cudaEventElapsedTime(&ms, a0, a1);
+        cudaEventDestroy(a0);
+        cudaEventDestroy(a1);
+        if (e != cudaSuccess) return fail(GS_ERR_CUDA, cudaGetErrorString(e));
+        s->cycle += n;
+        double bytes = 0;
+        for (uint32_t g = 0; g < p.n_eval; ++g)
+            bytes += (double)(p.aux[g].k + 1 + (p.aux[g].qdst != NONE32 ? 1 : 0)) * (double)s->stride;
+        out->level_ms = ms;
+        out->total_ms = ms;
+        out->level_launches = n ? 1 : 0;
+        out->total_launches = n ? 1 : 0;
+        out->level_bytes = bytes * n;
+        clear_error();
+        return GS_OK;
+    }
     std::vector<cudaEvent_t> evs(std::max<size_t>(2, 2 * (size_t)p.n_levels * s->slabs));
     const bool df = s->opts.kernel == GS_KERNEL_DATAFLOW;
     cudaEvent_t e0, e1;

@@ -329,6 +329,120 @@ def test_dataflow_rejects_bad_slab_sizes():
         assert e.value.code == gs.GS_ERR_ARG
 
 
+# ------------------------------------------------------------------ kernel T (tile-resident)
+@pytest.mark.parametrize("tw", [0, 4, 8, 16, 32])
+def test_tile_adder_all_lanes_and_exhaustive(tw):
+    cfg = workloads.CONFIGS["C1"]
+    nl = cfg.netlist()
+    r = run_gpu(nl, cfg.lanes, 1, "tile", seed=cfg.stim_seed, tile_words=tw)
+    o = oracle.simulate(nl, np.arange(cfg.lanes), 1, seed=cfg.stim_seed)
+    assert np.array_equal(gs.unpack_lanes(r["outputs"]).T, o["last"])
+    assert np.array_equal(r["sigs"], o["sig"])
+    # exhaustive 2^16 inputs through host-bound stimuli
+    a = np.arange(1 << 16) & 0xFF
+    b = np.arange(1 << 16) >> 8
+    bits = np.concatenate([(a[None, :] >> np.arange(8)[:, None]) & 1,
+                           (b[None, :] >> np.arange(8)[:, None]) & 1]).astype(np.uint8)
+    words = np.packbits(bits, axis=1, bitorder="little").view(np.uint64)[None]
+    e = run_gpu(nl, 1 << 16, 1, "tile", host_stim=words, tile_words=tw)
+    out = gs.unpack_lanes(e["outputs"]).astype(np.int64)
+    assert np.array_equal((out << np.arange(9)[:, None]).sum(0), a + b)
+
+
+@pytest.mark.parametrize("balance", [False, True])
+def test_tile_tiny_wide_gates_registers_all_lanes_step_split(balance):
+    """k up to 6, register edge cases; cycles split over several gs_sim_step calls."""
+    nls = [workloads.random_tiny(s, n_pi=6, n_reg=5, n_gates=300, n_po=12, max_k=6) for s in (5, 6)]
+    nls += [workloads.register_edge_cases(), workloads.probes_circuit()]
+    for nl in nls:
+        prog = compile_nl(nl, balance)
+        sim = gs.Sim(prog, 2048, kernel="tile", trace_words=[0, 7, 31], trace_cycles=11)
+        sim.bind_generated(13)
+        for n in (1, 3, 7):
+            sim.step(n)
+        o = oracle.simulate(nl, np.arange(2048), 11, seed=13)
+        assert np.array_equal(gs.unpack_lanes(sim.read_outputs()).T, o["last"])
+        assert np.array_equal(gs.unpack_lanes(sim.read_registers()).T, o["regs"])
+        assert np.array_equal(sim.read_lane_signatures(), o["sig"])
+        tb = gpu_trace_bits(sim.read_trace(), None)
+        rows = np.concatenate([np.arange(0, 64), np.arange(7 * 64, 8 * 64), np.arange(31 * 64, 32 * 64)])
+        assert np.array_equal(tb, o["trace"][rows])
+        sig = sim.signature()
+        assert sig["cycles"] == 11
+        assert sig["out_popcount"] == int(o["trace"].sum())
+        sim.close()
+
+
+def test_tile_c2_multiplier_all_lanes_equals_lut():
+    cfg = workloads.CONFIGS["C2"]
+    nl = cfg.netlist()
+    prog = compile_nl(nl)
+    t = run_gpu(nl, cfg.lanes, 2, "tile", seed=cfg.stim_seed, prog=prog)
+    a = run_gpu(nl, cfg.lanes, 2, "lut", seed=cfg.stim_seed, prog=prog)
+    assert np.array_equal(t["outputs"], a["outputs"]) and np.array_equal(t["sigs"], a["sigs"])
+    bits = gs.unpack_lanes(t["outputs"]).astype(np.uint64)        # [64][lanes], last cycle = 1
+    prod = (bits << np.arange(64, dtype=np.uint64)[:, None]).sum(0, dtype=np.uint64)
+    from tests._ref import pi_lanes_np
+    pis = pi_lanes_np(cfg.stim_seed, 64, 1, cfg.lanes, 0).astype(np.uint64)
+    x = (pis[:32] << np.arange(32, dtype=np.uint64)[:, None]).sum(0, dtype=np.uint64)
+    y = (pis[32:] << np.arange(32, dtype=np.uint64)[:, None]).sum(0, dtype=np.uint64)
+    assert np.array_equal(prod, x * y)
+
+
+@pytest.mark.parametrize("tw,ng", [(0, 0), (4, 1), (4, 2), (8, 1)])
+def test_tile_sequential_synthetic_all_lanes_probes_resume(tw, ng):
+    """8k-gate sequential synthetic netlist (C3 recipe, smaller): every lane vs the oracle."""
+    nl = workloads.synthetic(8000, 300, 32, 48, 24, seed=21, name="t8k")
+    prog = compile_nl(nl)
+    lanes, cycles = 4096, 40
+    t = run_gpu(nl, lanes, cycles, "tile", seed=5, prog=prog, trace_words=[0, 33, 63], tile_words=tw,
+                tile_groups=ng)
+    a = run_gpu(nl, lanes, cycles, "lut", seed=5, prog=prog)
+    for key in ("outputs", "regs", "sigs"):
+        assert np.array_equal(t[key], a[key]), key
+    assert t["signature"]["out_popcount"] == a["signature"]["out_popcount"]
+    o = oracle.simulate(nl, np.arange(lanes), cycles, seed=5, want=("last", "regs", "sig"))
+    assert np.array_equal(t["sigs"], o["sig"])
+    assert np.array_equal(gs.unpack_lanes(t["regs"]).T, o["regs"])
+    probe_closed_forms(nl, gs.unpack_lanes(t["outputs"]).T, cycles - 1, 5, lanes)
+    # resume through register write-back
+    sim = gs.Sim(prog, lanes, kernel="tile", tile_words=tw, tile_groups=ng)
+    sim.bind_generated(5)
+    sim.step(13)
+    regs = sim.read_registers()
+    sim.write_registers(np.zeros_like(regs))
+    sim.write_registers(regs)
+    sim.step(cycles - 13)
+    assert np.array_equal(sim.read_registers(), a["regs"])
+    assert np.array_equal(sim.read_lane_signatures(), a["sigs"])
+    sim.close()
+
+
+def test_auto_kernel_selection():
+    """AUTO = kernel T (one launch per step) when the circuit fits shared memory, else A."""
+    for name, lanes, tile in (("C1", 1024, True), ("C2", 1 << 14, True), ("C3", 4096, False)):
+        prog = compile_nl(workloads.CONFIGS[name].netlist())
+        sim = gs.Sim(prog, lanes, kernel="auto")
+        assert (sim.launches_per_cycle() == 1) == tile, name
+        sim.bind_generated(1)
+        sim.step(2)
+        ref = run_gpu(workloads.CONFIGS[name].netlist(), lanes, 2, "lut", seed=1, prog=prog)
+        assert np.array_equal(sim.read_lane_signatures(), ref["sigs"])
+        sim.close()
+
+
+def test_tile_rejects_oversized_or_misaligned():
+    prog = compile_nl(workloads.adder(8))
+    with pytest.raises(gs.GsError) as e:
+        gs.Sim(prog, 1024 + 64, kernel="tile", tile_words=8)
+    assert e.value.code == gs.GS_ERR_ARG
+    for name in ("C3", "C4"):                     # live state larger than shared memory
+        big = compile_nl(workloads.CONFIGS[name].netlist())
+        with pytest.raises(gs.GsError) as e:
+            gs.Sim(big, 4096, kernel="tile")
+        assert e.value.code == gs.GS_ERR_ARG
+
+
 # ------------------------------------------------------------------ full-size configs
 @pytest.mark.slow
 def test_c4_full_config_sampled_lanes_and_probes():
