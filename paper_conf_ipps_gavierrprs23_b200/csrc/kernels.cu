@@ -17,6 +17,8 @@
 // x_s - |S| + 1), output sum_S w_S h_S (only the nonzero w_S, sparse as in P:187),
 // then ballot-packed back to 32 stimuli per word.  Outputs outside {0,1} are counted
 // (P:224 says they cannot happen).  Used standalone or as a cross-check of A.
+#include <algorithm>
+
 #include <cuda_runtime.h>
 
 #include "kernels.h"
@@ -525,52 +527,54 @@ __global__ void __launch_bounds__(256) k_end_cycle(EndArgs a, uint32_t latch_blo
     pdl_entry();
     const unsigned long long c = a.ctl->cycle;
     if (blockIdx.x < latch_blocks) {
-        const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-        if (t < (uint64_t)a.n_latch * a.words) {
-            const uint32_t e = (uint32_t)(t / a.words), w = (uint32_t)(t - (uint64_t)e * a.words);
-            const uint32_t src = resolve(__ldg(a.latch_src + e), a.qcur);
-            const uint32_t dst = a.row_q0 + __ldg(a.latch_dst + e) + a.qnext;
-            reinterpret_cast<unsigned long long*>(a.state + (uint64_t)dst * a.stride)[w] =
-                reinterpret_cast<const unsigned long long*>(a.state + (uint64_t)src * a.stride)[w];
+        // leftover latches (register D not fused into its gate's store): 16-byte copies,
+        // grid-stride over (latch, vector)
+        const uint32_t vpr = a.stride / 16;                         // stride is a multiple of 8
+        if (vpr * 16 == a.stride) {
+            const uint64_t n = (uint64_t)a.n_latch * vpr;
+            for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < n;
+                 t += (uint64_t)latch_blocks * blockDim.x) {
+                const uint32_t e = (uint32_t)(t / vpr), v = (uint32_t)(t - (uint64_t)e * vpr);
+                const uint32_t src = resolve(__ldg(a.latch_src + e), a.qcur);
+                const uint32_t dst = a.row_q0 + __ldg(a.latch_dst + e) + a.qnext;
+                reinterpret_cast<uint4*>(a.state + (uint64_t)dst * a.stride)[v] =
+                    __ldcs(reinterpret_cast<const uint4*>(a.state + (uint64_t)src * a.stride) + v);
+            }
+        } else {
+            const uint64_t n = (uint64_t)a.n_latch * a.words;
+            for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < n;
+                 t += (uint64_t)latch_blocks * blockDim.x) {
+                const uint32_t e = (uint32_t)(t / a.words), w = (uint32_t)(t - (uint64_t)e * a.words);
+                const uint32_t src = resolve(__ldg(a.latch_src + e), a.qcur);
+                const uint32_t dst = a.row_q0 + __ldg(a.latch_dst + e) + a.qnext;
+                reinterpret_cast<unsigned long long*>(a.state + (uint64_t)dst * a.stride)[w] =
+                    reinterpret_cast<const unsigned long long*>(a.state + (uint64_t)src * a.stride)[w];
+            }
         }
     } else {
-        const uint32_t warp = ((blockIdx.x - latch_blocks) * blockDim.x + threadIdx.x) >> 5;
-        const uint32_t lane = threadIdx.x & 31;
-        if (warp < a.words) {
-            const uint32_t w = warp;
-            unsigned long long v0 = 0, v1 = 0;
-            uint32_t pop = 0;
-            for (uint32_t o = lane; o < a.n_po; o += 32) {
+        // thread = (bit-plane j, word w), consecutive threads = consecutive words, so every
+        // PO row read is coalesced.  MISR planes are double-buffered by cycle parity: read
+        // misr_cur (state after cycle c-1), write misr_next.
+        const uint64_t t = (uint64_t)(blockIdx.x - latch_blocks) * blockDim.x + threadIdx.x;
+        uint32_t pop = 0;
+        if (t < (uint64_t)64 * a.words) {
+            const uint32_t j = (uint32_t)(t / a.words), w = (uint32_t)(t - (uint64_t)j * a.words);
+            const int32_t slot = (a.trace && c < a.trace_cap) ? __ldg(a.trace_slot + w) : -1;
+            unsigned long long v = 0;
+            for (uint32_t o = j; o < a.n_po; o += 64) {
                 const uint32_t row = resolve(__ldg(a.po_rows + o), a.qcur);
-                const unsigned long long x = reinterpret_cast<const unsigned long long*>(a.state + (uint64_t)row * a.stride)[w];
+                const unsigned long long x = __ldg(reinterpret_cast<const unsigned long long*>(a.state + (uint64_t)row * a.stride) + w);
+                v ^= x;
                 pop += __popcll(x);
-                if ((o & 63) < 32) v0 ^= x; else v1 ^= x;   // o mod 64 = lane or lane + 32
+                if (slot >= 0) a.trace[((uint64_t)c * a.n_po + o) * a.ntw + slot] = x;
             }
-            unsigned long long* m0 = a.misr + (uint64_t)lane * a.words + w;
-            unsigned long long* m1 = a.misr + (uint64_t)(lane + 32) * a.words + w;
-            const unsigned long long p0 = *m0, p1 = *m1;
-            const unsigned long long up0 = __shfl_up_sync(FULL, p0, 1);
-            const unsigned long long up1 = __shfl_up_sync(FULL, p1, 1);
-            const unsigned long long p31 = __shfl_sync(FULL, p0, 31);
-            const unsigned long long p63 = __shfl_sync(FULL, p1, 31);
-            const unsigned long long prev0 = lane == 0 ? 0ULL : up0;      // plane j-1 for j = lane
-            const unsigned long long prev1 = lane == 0 ? p31 : up1;       // plane j-1 for j = lane + 32
-            const unsigned long long fb0 = ((MISR_POLY >> lane) & 1ULL) ? p63 : 0ULL;
-            const unsigned long long fb1 = ((MISR_POLY >> (lane + 32)) & 1ULL) ? p63 : 0ULL;
-            *m0 = prev0 ^ fb0 ^ v0;
-            *m1 = prev1 ^ fb1 ^ v1;
-            const int32_t slot = a.trace ? __ldg(a.trace_slot + w) : -1;
-            if (slot >= 0 && c < a.trace_cap) {
-                for (uint32_t o = lane; o < a.n_po; o += 32) {
-                    const uint32_t row = resolve(__ldg(a.po_rows + o), a.qcur);
-                    a.trace[((uint64_t)c * a.n_po + o) * a.ntw + slot] =
-                        reinterpret_cast<const unsigned long long*>(a.state + (uint64_t)row * a.stride)[w];
-                }
-            }
-#pragma unroll
-            for (int o = 16; o > 0; o >>= 1) pop += __shfl_xor_sync(FULL, pop, o);
-            if (lane == 0 && pop) atomicAdd(&a.ctl->popcount, (unsigned long long)pop);
+            const unsigned long long prev = j ? a.misr_cur[(uint64_t)(j - 1) * a.words + w] : 0ULL;
+            const unsigned long long fb = ((MISR_POLY >> j) & 1ULL) ? a.misr_cur[(uint64_t)63 * a.words + w] : 0ULL;
+            a.misr_next[(uint64_t)j * a.words + w] = prev ^ fb ^ v;
         }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) pop += __shfl_xor_sync(FULL, pop, o);
+        if ((threadIdx.x & 31) == 0 && pop) atomicAdd(&a.ctl->popcount, (unsigned long long)pop);
     }
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -585,9 +589,10 @@ __global__ void __launch_bounds__(256) k_end_cycle(EndArgs a, uint32_t latch_blo
 }
 
 cudaError_t launch_end_cycle(const EndArgs& a, cudaStream_t s) {
-    const uint64_t lt = (uint64_t)a.n_latch * a.words;
-    const uint32_t latch_blocks = (uint32_t)((lt + 255) / 256);
-    const uint32_t misr_blocks = (a.words * 32 + 255) / 256;
+    // latch copies: grid-stride, at most ~8 blocks per SM worth of threads
+    const uint64_t lt = (uint64_t)a.n_latch * (a.words > 1 ? a.words / 2 : 1);
+    const uint32_t latch_blocks = (uint32_t)std::min<uint64_t>((lt + 255) / 256, 148 * 8);
+    const uint32_t misr_blocks = (uint32_t)(((uint64_t)a.words * 64 + 255) / 256);
     return launch_k(k_end_cycle, latch_blocks + misr_blocks, s, a.pdl, a, latch_blocks);
 }
 

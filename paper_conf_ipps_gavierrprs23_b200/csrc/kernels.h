@@ -52,7 +52,8 @@ struct EndArgs {
     uint32_t row_q0, qcur, qnext;
     const uint32_t* po_rows;
     uint32_t n_po;
-    unsigned long long* misr;         // [64][words]
+    const unsigned long long* misr_cur;   // [64][words] MISR after the previous cycle
+    unsigned long long* misr_next;        // [64][words] MISR after this cycle
     const int32_t* trace_slot;        // [words]
     unsigned long long* trace;        // [trace_cap][n_po][ntw]
     uint32_t ntw, trace_cap;
@@ -103,7 +104,7 @@ struct TileArgs {
     uint32_t words;                   // 64-bit words per state row (lanes / 64)
     uint32_t row_q0;
     Ctl* ctl;
-    unsigned long long* misr;         // [64][words]
+    unsigned long long* misr;         // 2 x [64][words] (buffer = cycle parity)
     const int32_t* trace_slot;
     unsigned long long* trace;
     uint32_t ntw, trace_cap;

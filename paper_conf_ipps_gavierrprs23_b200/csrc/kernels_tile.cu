@@ -97,7 +97,10 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     const uint32_t w32_row = a.words * 2;                     // 32-bit words per state row
     const uint32_t* st32 = reinterpret_cast<const uint32_t*>(a.state);
     uint32_t* st32w = reinterpret_cast<uint32_t*>(a.state);
-    uint32_t* misr32 = reinterpret_cast<uint32_t*>(a.misr);
+    // MISR planes are double-buffered by cycle parity (as k_end_cycle): read the buffer of
+    // the first cycle, write the buffer of the cycle after the last
+    const uint32_t* misr_in = reinterpret_cast<const uint32_t*>(a.misr + (size_t)(c0 & 1) * 64 * a.words);
+    uint32_t* misr_out = reinterpret_cast<uint32_t*>(a.misr + (size_t)((c0 + a.ncycles) & 1) * 64 * a.words);
     unsigned long long pop = 0;
 
     for (uint32_t tile = blockIdx.x * NG + gid; tile < a.n_tiles; tile += gridDim.x * NG) {
@@ -113,7 +116,7 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
         }
         for (uint32_t u = tid; u < 64 * TW; u += bd) {
             const uint32_t j = u / TW, w = u % TW;
-            mp[u] = misr32[(uint64_t)j * w32_row + t0 + w];
+            mp[u] = misr_in[(uint64_t)j * w32_row + t0 + w];
         }
         group_sync(bar, GT);
         for (uint32_t c = 0; c < a.ncycles; ++c) {
@@ -200,7 +203,7 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
         }
         for (uint32_t u = tid; u < 64 * TW; u += bd) {
             const uint32_t j = u / TW, w = u % TW;
-            misr32[(uint64_t)j * w32_row + t0 + w] = mp[u];
+            misr_out[(uint64_t)j * w32_row + t0 + w] = mp[u];
         }
         group_sync(bar, GT);                              // before the next tile reuses smem
     }

@@ -149,7 +149,7 @@ Layout make_layout(const Program& p, const gs_sim_opts& o, const Plans& pl) {
     L.latch_dst = take(p.latch_dst.size() * 4);
     L.reg_init = take(p.reg_init.size());
     L.trace_slot = take((size_t)words * 4);
-    L.misr = take((size_t)64 * words * 8);
+    L.misr = take((size_t)2 * 64 * words * 8);        // double-buffered by cycle parity
     L.trace = take((size_t)o.trace_cycles * p.n_po * o.n_trace_words * 8);
     L.lane_sigs = take((size_t)o.lanes * 8);
     L.scratch = take((size_t)p.n_po * words * 8);
@@ -247,7 +247,8 @@ static EndArgs end_args(const gs_sim* s, uint32_t parity) {
     e.qnext = parity ? 0 : p.n_reg;
     e.po_rows = s->at<const uint32_t>(s->L.po_rows);
     e.n_po = p.n_po;
-    e.misr = s->at<unsigned long long>(s->L.misr);
+    e.misr_cur = s->at<unsigned long long>(s->L.misr) + (size_t)parity * 64 * s->words;
+    e.misr_next = s->at<unsigned long long>(s->L.misr) + (size_t)(parity ^ 1) * 64 * s->words;
     e.trace_slot = s->at<const int32_t>(s->L.trace_slot);
     e.trace = (s->opts.n_trace_words && s->opts.trace_cycles) ? s->at<unsigned long long>(s->L.trace) : nullptr;
     e.ntw = s->opts.n_trace_words;
@@ -553,7 +554,7 @@ gs_status gs_sim_reset(gs_sim* s) {
     const Program& p = *s->prog;
     CU(cudaSetDevice(s->opts.device));
     CU(cudaMemsetAsync(s->ws + s->L.ctl, 0, sizeof(Ctl), s->stream));
-    CU(cudaMemsetAsync(s->ws + s->L.misr, 0, (size_t)64 * s->words * 8, s->stream));
+    CU(cudaMemsetAsync(s->ws + s->L.misr, 0, (size_t)2 * 64 * s->words * 8, s->stream));
     if (s->L.lane_sigs != s->L.scratch) CU(cudaMemsetAsync(s->ws + s->L.lane_sigs, 0, (size_t)s->opts.lanes * 8, s->stream));
     size_t tbytes = (size_t)s->opts.trace_cycles * p.n_po * s->opts.n_trace_words * 8;
     if (tbytes) CU(cudaMemsetAsync(s->ws + s->L.trace, 0, tbytes, s->stream));
@@ -724,7 +725,8 @@ gs_status gs_sim_read_trace(gs_sim* s, uint64_t* host, size_t nwords, uint32_t* 
 
 static gs_status compute_lane_sigs(gs_sim* s) {
     CU(cudaMemsetAsync(s->ws + s->L.ctl + offsetof(Ctl, sig_sum), 0, 8, s->stream));
-    CU(launch_lane_sigs(s->ctl(), s->at<const unsigned long long>(s->L.misr), s->words, s->opts.lane_offset,
+    CU(launch_lane_sigs(s->ctl(), s->at<const unsigned long long>(s->L.misr) + (size_t)(s->cycle & 1) * 64 * s->words,
+                        s->words, s->opts.lane_offset,
                         s->at<unsigned long long>(s->L.lane_sigs), s->stream));
     return GS_OK;
 }
