@@ -222,6 +222,11 @@ typedef struct {
 /* flags: launch the per-cycle kernels WITHOUT programmatic dependent launch (by default a
  * level kernel may become resident while its predecessor drains; A/B measurement only). */
 #define GS_SIM_NO_PDL 1u
+/* flags: kernel A stores a gate row that the next level reads with L2 evict_last and all
+ * other rows with evict_first (the compiler marks the rows). */
+#define GS_SIM_L2_HINTS 2u
+/* flags: with GS_SIM_L2_HINTS, also load gate inputs with L2 evict_first. */
+#define GS_SIM_L2_HINT_LOADS 4u
 
 /* Device workspace bytes required for (prog, opts). */
 gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts, size_t* bytes);

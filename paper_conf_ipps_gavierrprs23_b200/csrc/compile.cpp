@@ -212,6 +212,14 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
         pr.aux[pos].qdst = NONE32;
         pr.aux[pos].k = k;
     }
+    // "hot" rows: read by a gate of the very next level (kernel A keeps them in L2 with
+    // an evict_last store)
+    pr.hot.assign(n_eval, 0);
+    for (uint32_t g = 0; g < G; ++g) {
+        if (nl.gate_k[g] == 0) continue;
+        for (uint32_t e = cons_off[g]; e < cons_off[g + 1]; ++e)
+            if (level[cons[e]] == level[g] + 1) { pr.hot[exec_pos[g]] = 1; break; }
+    }
     // registers: fuse the latch into the D-driving gate's store when possible (the
     // recurrent connection of P:241 becomes a dual store into the other Q bank)
     pr.reg_init = nl.reg_init;

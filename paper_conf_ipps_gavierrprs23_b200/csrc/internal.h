@@ -58,6 +58,7 @@ struct Program {
     std::vector<uint32_t> in_lo;              // [n_eval * 4] row refs (QFLAG for Q rows)
     std::vector<uint32_t> in_hi;              // [n_eval * 2] (inputs 4, 5) if any_wide
     std::vector<GateAux> aux;                 // [n_eval]
+    std::vector<uint8_t> hot;                 // [n_eval] a gate of the next level reads it
     std::vector<uint32_t> term_off;           // [n_eval + 1] kernel B nonzero terms
     std::vector<uint32_t> terms;              // S | (|S|-1)<<8 | (w & 0xffff)<<16
     std::vector<uint32_t> po_rows;            // [n_po]  row refs

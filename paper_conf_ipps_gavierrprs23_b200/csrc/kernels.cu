@@ -89,7 +89,7 @@ __global__ void __launch_bounds__(256) k_level_lut(LevelArgs a, uint32_t vpr, ui
     const uint4 in = __ldg(a.din + gate);
     const uint4 au = __ldg(reinterpret_cast<const uint4*>(a.aux) + gate);
     const uint64_t tt = ((uint64_t)au.y << 32) | au.x;
-    const uint32_t qdst = au.z, k = au.w;
+    const uint32_t qdst = au.z, k = au.w & 0xFFu;
     if (VEC16) {
         switch (k) {
             case 1: lut_gate_vec16<1>(a, gate, in, v, tt, qdst); break;
@@ -113,10 +113,12 @@ __global__ void __launch_bounds__(256) k_level_lut(LevelArgs a, uint32_t vpr, ui
 
 // Wide-row variant: every warp owns one gate and U x 32 consecutive 16-byte vectors of
 // it; all U*k input loads are issued before any is consumed (memory-level parallelism
-// U*k per thread, one descriptor fetch per U vectors).
-template <int K, int U>
+// U*k per thread, one descriptor fetch per U vectors).  HINT: L2 eviction priority per
+// store (aux.k bit 8 = "a gate of the next level reads this row": evict_last; other rows
+// and the register next-bank store: evict_first).
+template <int K, int U, bool HINT>
 __device__ __forceinline__ void lut_gate_u(const LevelArgs& a, uint32_t gate, uint4 in, uint32_t v0,
-                                           uint64_t tt, uint32_t qdst) {
+                                           uint64_t tt, uint32_t qdst, bool hot) {
     uint32_t r[6];
     r[0] = in.x; r[1] = in.y; r[2] = in.z; r[3] = in.w;
     if (K > 4) {
@@ -128,22 +130,31 @@ __device__ __forceinline__ void lut_gate_u(const LevelArgs& a, uint32_t gate, ui
     for (int i = 0; i < K; ++i)
         src[i] = reinterpret_cast<const uint4*>(a.state + (uint64_t)resolve(r[i], a.qcur) * a.stride) + v0;
     uint4 x[U][K];
+    uint64_t pf = 0;
+    if (HINT) pf = l2_policy_first();
 #pragma unroll
     for (int u = 0; u < U; ++u)
 #pragma unroll
-        for (int i = 0; i < K; ++i) x[u][i] = __ldg(src[i] + u * 32);
+        for (int i = 0; i < K; ++i) x[u][i] = (HINT && a.hint_ld) ? ld_hint(src[i] + u * 32, pf) : __ldg(src[i] + u * 32);
     uint4* dst = reinterpret_cast<uint4*>(a.state + (uint64_t)(a.row_gate0 + gate) * a.stride) + v0;
     uint4* qd = qdst != 0xFFFFFFFFu ? reinterpret_cast<uint4*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride) + v0
                                     : nullptr;
+    uint64_t po = 0;
+    if (HINT) po = hot ? l2_policy_last() : pf;
 #pragma unroll
     for (int u = 0; u < U; ++u) {
         const uint4 y = lut_eval4<K>(tt, x[u]);
-        dst[u * 32] = y;
-        if (qd) qd[u * 32] = y;
+        if (HINT) {
+            st_hint(dst + u * 32, y, po);
+            if (qd) st_hint(qd + u * 32, y, pf);
+        } else {
+            dst[u * 32] = y;
+            if (qd) qd[u * 32] = y;
+        }
     }
 }
 
-template <int U>
+template <int U, bool HINT>
 __global__ void __launch_bounds__(256, 4) k_level_lut_wide(LevelArgs a, uint32_t cpg_shift, uint32_t vec0) {
     pdl_entry();
     const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -156,21 +167,22 @@ __global__ void __launch_bounds__(256, 4) k_level_lut_wide(LevelArgs a, uint32_t
     const uint4 in = __ldg(a.din + gate);
     const uint4 au = __ldg(reinterpret_cast<const uint4*>(a.aux) + gate);
     const uint64_t tt = ((uint64_t)au.y << 32) | au.x;
-    const uint32_t qdst = au.z, k = au.w;
+    const uint32_t qdst = au.z, k = au.w & 0xFFu;
+    const bool hot = (au.w >> 8) & 1u;
     switch (k) {
-        case 1: lut_gate_u<1, U>(a, gate, in, v0, tt, qdst); break;
-        case 2: lut_gate_u<2, U>(a, gate, in, v0, tt, qdst); break;
-        case 3: lut_gate_u<3, U>(a, gate, in, v0, tt, qdst); break;
-        case 4: lut_gate_u<4, U>(a, gate, in, v0, tt, qdst); break;
-        case 5: lut_gate_u<5, 1>(a, gate, in, v0, tt, qdst);
-                if (U > 1) lut_gate_u<5, 1>(a, gate, in, v0 + 32, tt, qdst);
-                if (U > 2) { lut_gate_u<5, 1>(a, gate, in, v0 + 64, tt, qdst);
-                             lut_gate_u<5, 1>(a, gate, in, v0 + 96, tt, qdst); }
+        case 1: lut_gate_u<1, U, HINT>(a, gate, in, v0, tt, qdst, hot); break;
+        case 2: lut_gate_u<2, U, HINT>(a, gate, in, v0, tt, qdst, hot); break;
+        case 3: lut_gate_u<3, U, HINT>(a, gate, in, v0, tt, qdst, hot); break;
+        case 4: lut_gate_u<4, U, HINT>(a, gate, in, v0, tt, qdst, hot); break;
+        case 5: lut_gate_u<5, 1, HINT>(a, gate, in, v0, tt, qdst, hot);
+                if (U > 1) lut_gate_u<5, 1, HINT>(a, gate, in, v0 + 32, tt, qdst, hot);
+                if (U > 2) { lut_gate_u<5, 1, HINT>(a, gate, in, v0 + 64, tt, qdst, hot);
+                             lut_gate_u<5, 1, HINT>(a, gate, in, v0 + 96, tt, qdst, hot); }
                 break;
-        default: lut_gate_u<6, 1>(a, gate, in, v0, tt, qdst);
-                if (U > 1) lut_gate_u<6, 1>(a, gate, in, v0 + 32, tt, qdst);
-                if (U > 2) { lut_gate_u<6, 1>(a, gate, in, v0 + 64, tt, qdst);
-                             lut_gate_u<6, 1>(a, gate, in, v0 + 96, tt, qdst); }
+        default: lut_gate_u<6, 1, HINT>(a, gate, in, v0, tt, qdst, hot);
+                if (U > 1) lut_gate_u<6, 1, HINT>(a, gate, in, v0 + 32, tt, qdst, hot);
+                if (U > 2) { lut_gate_u<6, 1, HINT>(a, gate, in, v0 + 64, tt, qdst, hot);
+                             lut_gate_u<6, 1, HINT>(a, gate, in, v0 + 96, tt, qdst, hot); }
                 break;
     }
 }
@@ -192,9 +204,14 @@ cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s) {
             const uint64_t threads = ((uint64_t)a.ng << sh) * 32;
             if (threads >= (1ull << 31)) break;
             const uint32_t blocks = (uint32_t)((threads + 255) / 256);
-            if (U == 4) return launch_k(k_level_lut_wide<4>, blocks, s, a.pdl, a, sh, a.vec0);
-            if (U == 2) return launch_k(k_level_lut_wide<2>, blocks, s, a.pdl, a, sh, a.vec0);
-            return launch_k(k_level_lut_wide<1>, blocks, s, a.pdl, a, sh, a.vec0);
+            if (a.hint) {
+                if (U == 4) return launch_k(k_level_lut_wide<4, true>, blocks, s, a.pdl, a, sh, a.vec0);
+                if (U == 2) return launch_k(k_level_lut_wide<2, true>, blocks, s, a.pdl, a, sh, a.vec0);
+                return launch_k(k_level_lut_wide<1, true>, blocks, s, a.pdl, a, sh, a.vec0);
+            }
+            if (U == 4) return launch_k(k_level_lut_wide<4, false>, blocks, s, a.pdl, a, sh, a.vec0);
+            if (U == 2) return launch_k(k_level_lut_wide<2, false>, blocks, s, a.pdl, a, sh, a.vec0);
+            return launch_k(k_level_lut_wide<1, false>, blocks, s, a.pdl, a, sh, a.vec0);
         }
     }
     if (a.vslab) return cudaErrorInvalidValue;      // slabs only on the wide path
@@ -346,7 +363,7 @@ __global__ void __launch_bounds__(256, 4) k_dataflow(DfArgs a) {
             if (gb + j >= ge) continue;
             const uint32_t g = gb + j;
             const uint64_t tt = ((uint64_t)au.y << 32) | au.x;
-            switch (au.w) {
+            switch (au.w & 0xFFu) {
                 case 1: df_gate<1, VPT, LPG>(a, g, in, tt, au.z, v0); break;
                 case 2: df_gate<2, VPT, LPG>(a, g, in, tt, au.z, v0); break;
                 case 3: df_gate<3, VPT, LPG>(a, g, in, tt, au.z, v0); break;
@@ -411,7 +428,7 @@ __global__ void __launch_bounds__(256) k_level_poly(LevelArgs a, uint32_t words3
     const bool valid = j < words32;
     const uint4 in = __ldg(a.din + gate);
     const uint4 au = __ldg(reinterpret_cast<const uint4*>(a.aux) + gate);
-    const uint32_t qdst = au.z, k = au.w;
+    const uint32_t qdst = au.z, k = au.w & 0xFFu;
     uint32_t r[6] = {in.x, in.y, in.z, in.w, 0u, 0u};
     if (k > 4) {
         const uint2 hi = __ldg(a.dhi + gate);

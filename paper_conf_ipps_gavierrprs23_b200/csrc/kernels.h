@@ -39,6 +39,8 @@ struct LevelArgs {
     uint32_t unroll;                  // max vectors per thread on the wide path (0 = auto)
     uint32_t pdl;                     // launch with programmatic stream serialization
     uint32_t min_warps;               // auto U: prefer smaller U below this many warps
+    uint32_t hint;                    // L2 eviction-priority stores (aux.k bit 8 = read next level)
+    uint32_t hint_ld;                 // ... and evict_first input loads
 };
 
 struct EndArgs {

@@ -229,6 +229,8 @@ static LevelArgs level_args(const gs_sim* s, uint32_t l, uint32_t parity) {
     a.ctl = s->ctl();
     a.pdl = s->pdl;
     a.min_warps = s->min_warps;
+    a.hint = (s->opts.flags & GS_SIM_L2_HINTS) ? 1u : 0u;
+    a.hint_ld = (s->opts.flags & GS_SIM_L2_HINT_LOADS) ? 1u : 0u;
     return a;
 }
 
@@ -501,9 +503,12 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
     std::vector<int32_t> slot(words, -1);
     for (uint32_t i = 0; i < opts->n_trace_words; ++i) slot[opts->trace_words[i]] = (int32_t)i;
     const bool poly = s->opts.kernel == GS_KERNEL_POLY || s->opts.kernel == GS_KERNEL_AB;
+    // device aux: k | hot << 8 (kernels mask k with 0xFF)
+    std::vector<GateAux> aux_dev = p.aux;
+    for (size_t g = 0; g < aux_dev.size(); ++g) aux_dev[g].k |= (uint32_t)p.hot[g] << 8;
     std::vector<Up> ups = {
         {L.din, p.in_lo.data(), p.in_lo.size() * 4},
-        {L.aux, p.aux.data(), p.aux.size() * sizeof(GateAux)},
+        {L.aux, aux_dev.data(), aux_dev.size() * sizeof(GateAux)},
         {L.dhi, p.in_hi.data(), p.any_wide ? p.in_hi.size() * 4 : 0},
         {L.term_off, p.term_off.data(), poly ? p.term_off.size() * 4 : 0},
         {L.terms, p.terms.data(), poly ? p.terms.size() * 4 : 0},

@@ -283,6 +283,18 @@ def test_errors_on_device():
     sim.close()
 
 
+@pytest.mark.parametrize("flags", [gs.GS_SIM_NO_PDL, 2, 6])
+def test_launch_and_cache_options_do_not_change_results(flags):
+    """PDL off, L2 eviction hints on stores, hints on stores and loads: bit-identical."""
+    cfg = workloads.CONFIGS["C3"]
+    nl = cfg.netlist()
+    prog = compile_nl(nl)
+    a = run_gpu(nl, 8192, 20, "lut", seed=4, prog=prog)
+    b = run_gpu(nl, 8192, 20, "lut", seed=4, prog=prog, flags=flags)
+    for key in ("outputs", "regs", "sigs"):
+        assert np.array_equal(a[key], b[key]), key
+
+
 # ------------------------------------------------------------------ DATAFLOW schedule
 DF_CASES = [  # (lanes, lane_slabs, interleave, gates per warp)
     (4096, 0, 0, 0), (8192, 0, 1, 1), (16384, 0, 3, 7), (16384, 2, 2, 4), (32768, 2, 1, 32),
