@@ -42,6 +42,7 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C4")
     ap.add_argument("--cycles-per-step", type=int, default=100)
+    ap.add_argument("--lut-k", type=int, default=0, help="cone-collapse into <= L-input LUTs first")
     ap.add_argument("--lanes", type=int, default=0, help="override lanes per GPU")
     ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab", "df", "tile"])
     ap.add_argument("--tile-words", type=int, default=0, help="kernel T: 32-bit words per slot")
@@ -223,7 +224,7 @@ def main():
     lanes = args.lanes or (cfg.lanes // cfg.shards if cfg.shards > 1 else cfg.lanes)
     lane_offset = rank * lanes
     t0 = time.perf_counter()
-    prog = gs.Netlist.from_arrays(nl).compile(balance=True)
+    prog = gs.Netlist.from_arrays(nl).compile(balance=True, lut_k=args.lut_k)
     compile_s = time.perf_counter() - t0
     info = prog.info
     G = info["n_eval_gates"]
@@ -337,7 +338,7 @@ def main():
                        "lane_slabs": args.lane_slabs, "lut_unroll": args.lut_unroll,
                        "df_interleave": args.df_interleave, "df_gpw": args.df_gpw,
                        "pdl": not args.no_pdl, "tile_words": args.tile_words,
-                       "tile_groups": args.tile_groups, "l2_hints": args.l2_hints,
+                       "tile_groups": args.tile_groups, "l2_hints": args.l2_hints, "lut_k": args.lut_k,
                        "l2": "inputs larger than L2 (state %.1f GB per GPU)" % (info["n_rows"] * lanes / 8 / 1e9),
                        "parallelism": f"dp{world} (stimulus sharding)", "compile_s": round(compile_s, 2),
                        "paper_style_gcps": value * (G + info["n_reg"]) / G},

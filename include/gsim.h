@@ -135,9 +135,17 @@ typedef struct {
     int balance;      /* 0: ASAP levels.  1: slack-based balancing within [ASAP, ALAP]
                          (same depth; flattens the unbalanced level widths) */
     uint32_t max_k;   /* reject gates wider than this (0 = GS_MAX_K)                  */
+    uint32_t lut_k;   /* 0: evaluate the netlist's LUTs as given.  L in [2, max_k]: first
+                         collapse cones into LUTs of at most L inputs (the paper's LUT
+                         mapping step and its main hyperparameter L):
+                         a gate absorbs its deepest gate input while the merged input set
+                         has <= L nets (logic is duplicated where a cone is shared); gates
+                         nobody reads any more report k = 0.  Same simulation results,
+                         fewer levels and LUTs.                                        */
 } gs_compile_opts;
 
-/* Validate (GS_ERR_UNDRIVEN, GS_ERR_COMB_LOOP, GS_ERR_ARITY), levelize (level(g) =
+/* Validate (GS_ERR_UNDRIVEN, GS_ERR_COMB_LOOP, GS_ERR_ARITY), optionally collapse cones
+ * into <= lut_k-input LUTs, levelize (level(g) =
  * 1 + max level of its gate inputs; PIs, Qs, constants are level 0; optional
  * balancing), compile every TT to multilinear coefficients, lay out state rows and
  * pack per-level device descriptors.  opts may be NULL (balance=1). */
@@ -169,6 +177,11 @@ gs_status gs_program_gate_levels(const gs_program* prog, uint32_t* level, uint32
 /* Multilinear coefficients w_S (LSB-first subset index) of gate g (netlist order),
  * as compiled by the Möbius butterfly (Algorithm 1 in iterative form).  n >= 2^k. */
 gs_status gs_program_coeffs(const gs_program* prog, uint32_t gate, int32_t* w, uint32_t n);
+
+/* The LUT the program evaluates for netlist gate `gate` (after optional cone collapsing):
+ * its fan-in *k, input nets in[0..k-1] (in must hold GS_MAX_K entries) and LSB-first truth
+ * table *tt.  Without lut_k this is the gate as added; absorbed gates report k = 0. */
+gs_status gs_program_gate_lut(const gs_program* prog, uint32_t gate, uint32_t* k, gs_net* in, uint64_t* tt);
 
 /* Shared-memory slots one lane tile of kernel T needs (constants, PIs, two register banks,
  * gate values reused by live range; tile.cpp).  A tile of 32*w lanes needs

@@ -51,7 +51,7 @@ class gs_netlist_counts(C.Structure):
 
 
 class gs_compile_opts(C.Structure):
-    _fields_ = [("balance", C.c_int), ("max_k", C.c_uint32)]
+    _fields_ = [("balance", C.c_int), ("max_k", C.c_uint32), ("lut_k", C.c_uint32)]
 
 
 class gs_program_info(C.Structure):
@@ -113,6 +113,7 @@ _SIGS = {
     "gs_program_gate_levels": (C.c_int32, [_P, _P, C.c_uint32]),
     "gs_program_coeffs": (C.c_int32, [_P, C.c_uint32, _P, C.c_uint32]),
     "gs_program_tile_slots": (C.c_int32, [_P, _P]),
+    "gs_program_gate_lut": (C.c_int32, [_P, C.c_uint32, _P, _P, _P]),
     "gs_sim_workspace_bytes": (C.c_int32, [_P, _P, _P]),
     "gs_sim_create": (C.c_int32, [_P, _P, _P, C.c_size_t, _P]),
     "gs_sim_destroy": (C.c_int32, [_P]),
@@ -231,14 +232,14 @@ class Netlist:
         _call("gs_netlist_get_counts", self.h, C.byref(c))
         return {f: int(getattr(c, f)) for f, _ in c._fields_}
 
-    def compile(self, balance: bool = True, max_k: int = 0) -> "Program":
-        return Program(self, balance, max_k)
+    def compile(self, balance: bool = True, max_k: int = 0, lut_k: int = 0) -> "Program":
+        return Program(self, balance, max_k, lut_k)
 
 
 class Program:
-    def __init__(self, netlist: Netlist, balance: bool = True, max_k: int = 0):
+    def __init__(self, netlist: Netlist, balance: bool = True, max_k: int = 0, lut_k: int = 0):
         h = C.c_void_p()
-        o = gs_compile_opts(1 if balance else 0, max_k)
+        o = gs_compile_opts(1 if balance else 0, max_k, lut_k)
         _call("gs_compile", netlist.h, C.byref(o), C.byref(h))
         self.h = h
         inf = gs_program_info()
@@ -259,6 +260,14 @@ class Program:
         lv = np.zeros(max(self.info["n_gates"], 1), dtype=np.uint32)
         _call("gs_program_gate_levels", self.h, _p(lv), len(lv))
         return lv[:self.info["n_gates"]]
+
+    def gate_lut(self, gate: int) -> tuple[list[int], int]:
+        """(input nets, truth table) of the LUT evaluated for netlist gate `gate`."""
+        k = C.c_uint32()
+        ins = np.zeros(GS_MAX_K, dtype=np.uint32)
+        tt = C.c_uint64()
+        _call("gs_program_gate_lut", self.h, int(gate), C.byref(k), _p(ins), C.byref(tt))
+        return ins[:k.value].tolist(), tt.value
 
     def tile_slots(self) -> int:
         v = C.c_uint32()

@@ -238,6 +238,11 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
     pr.po_rows.resize(O);
     for (uint32_t o = 0; o < O; ++o) pr.po_rows[o] = row_of(nl.po_net[o]);
 
+    pr.lut_k = nl.gate_k;
+    pr.lut_in_off = nl.gate_in_off;
+    pr.lut_in = nl.gate_in;
+    pr.lut_tt = nl.gate_tt;
+
     // ---------------------------------------------------------------- coefficients
     pr.gate_level.assign(G, 0);
     pr.coeff_off.assign(G + 1, 0);

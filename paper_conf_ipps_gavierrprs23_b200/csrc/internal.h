@@ -70,11 +70,17 @@ struct Program {
     std::vector<uint32_t> gate_level;         // per netlist gate (0 for constants)
     std::vector<uint32_t> coeff_off;          // per netlist gate into coeffs
     std::vector<int32_t> coeffs;
+    std::vector<uint8_t> lut_k;               // evaluated LUT of every netlist gate (after
+    std::vector<uint32_t> lut_in_off, lut_in; //   optional cone collapsing): k, inputs (net
+    std::vector<uint64_t> lut_tt;             //   ids) and truth table
     std::vector<uint32_t> exec_gate;          // exec index -> netlist gate (for G count / debug)
     gs_program_info info{};
 };
 
 gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out);
+
+// Cone collapsing into LUTs of <= L inputs (collapse.cpp; the paper's LUT mapping)
+gs_status collapse_luts(const Netlist& nl, uint32_t L, Netlist& out);
 
 // ---------------------------------------------------------------- kernel T plan
 // Shared-memory slots of one lane tile (tile.cpp): [const0, const1 | PI | Q bank 0 |

@@ -205,13 +205,21 @@ gs_status gs_netlist_get_counts(const gs_netlist* h, gs_netlist_counts* out) {
 // ------------------------------------------------------------------ compile front
 gs_status gs_compile(const gs_netlist* h, const gs_compile_opts* opts, gs_program** out) {
     if (!h || !out) return fail(GS_ERR_ARG, "gs_compile: NULL argument");
-    gs_compile_opts o{1, 0};
+    gs_compile_opts o{1, 0, 0};
     if (opts) o = *opts;
     if (o.max_k == 0 || o.max_k > GS_MAX_K) o.max_k = GS_MAX_K;
+    if (o.lut_k == 1 || o.lut_k > o.max_k)
+        return fail(GS_ERR_ARG, "gs_compile: lut_k must be 0 or in [2, max_k]");
     Program* p = nullptr;
     gs_status st;
     try {
-        st = compile(h->nl, o, p);
+        if (o.lut_k) {
+            Netlist collapsed;
+            st = collapse_luts(h->nl, o.lut_k, collapsed);
+            if (st == GS_OK) st = compile(collapsed, o, p);
+        } else {
+            st = compile(h->nl, o, p);
+        }
     } catch (const std::bad_alloc&) {
         return fail(GS_ERR_NOMEM, "gs_compile: out of host memory");
     }
@@ -261,6 +269,17 @@ gs_status gs_program_coeffs(const gs_program* prog, uint32_t gate, int32_t* w, u
     uint32_t cnt = p.coeff_off[gate + 1] - p.coeff_off[gate];
     if (n < cnt) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_program_coeffs: n < 2^k");
     std::memcpy(w, p.coeffs.data() + p.coeff_off[gate], sizeof(int32_t) * cnt);
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_program_gate_lut(const gs_program* prog, uint32_t gate, uint32_t* k, gs_net* in, uint64_t* tt) {
+    if (!prog || !k || !in || !tt) return fail(GS_ERR_ARG, "gs_program_gate_lut: NULL argument");
+    const Program& p = *prog->p;
+    if (gate >= p.n_gates) return fail(GS_ERR_ARG, "gs_program_gate_lut: gate out of range");
+    *k = p.lut_k[gate];
+    for (uint32_t j = 0; j < *k; ++j) in[j] = p.lut_in[p.lut_in_off[gate] + j];
+    *tt = p.lut_tt[gate];
     clear_error();
     return GS_OK;
 }

@@ -295,6 +295,40 @@ def test_launch_and_cache_options_do_not_change_results(flags):
         assert np.array_equal(a[key], b[key]), key
 
 
+# ------------------------------------------------------------------ cone collapsing (lut_k)
+@pytest.mark.parametrize("L", [3, 6])
+@pytest.mark.parametrize("kernel", ["lut", "poly", "ab", "tile"])
+def test_collapsed_program_equals_oracle_of_original_netlist(kernel, L):
+    """Programs compiled with lut_k = L (wider LUTs, fewer levels) vs the oracle run on the
+    ORIGINAL netlist: every lane, every cycle."""
+    nls = [workloads.adder(8), workloads.random_tiny(4, n_pi=6, n_reg=5, n_gates=300, n_po=12),
+           workloads.synthetic(3000, 120, 16, 40, 12, seed=9, name="s")]
+    for nl in nls:
+        prog = gs.Netlist.from_arrays(nl).compile(lut_k=L)
+        r = run_gpu(nl, 4096, 7, kernel, seed=23, prog=prog, trace_words=[0, 40, 63])
+        o = oracle.simulate(nl, np.arange(4096), 7, seed=23)
+        assert np.array_equal(gs.unpack_lanes(r["outputs"]).T, o["last"])
+        assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"])
+        assert np.array_equal(r["sigs"], o["sig"])
+        rows = np.concatenate([np.arange(0, 64), np.arange(40 * 64, 41 * 64), np.arange(63 * 64, 64 * 64)])
+        assert np.array_equal(gpu_trace_bits(r["trace"], None), o["trace"][rows])
+        assert r["signature"]["ab_mismatch"] == 0 and r["signature"]["invariant_violations"] == 0
+
+
+def test_collapsed_multiplier_all_lanes_equal_a_times_b():
+    cfg = workloads.CONFIGS["C2"]
+    nl = cfg.netlist()
+    prog = gs.Netlist.from_arrays(nl).compile(lut_k=6)
+    assert prog.info["n_levels"] <= 92
+    r = run_gpu(nl, cfg.lanes, 1, "auto", seed=cfg.stim_seed, prog=prog)
+    bits = gs.unpack_lanes(r["outputs"]).astype(np.uint64)
+    prod = (bits << np.arange(64, dtype=np.uint64)[:, None]).sum(0, dtype=np.uint64)
+    pis = _ref.pi_lanes_np(cfg.stim_seed, 64, 0, cfg.lanes).astype(np.uint64)
+    x = (pis[:32] << np.arange(32, dtype=np.uint64)[:, None]).sum(0, dtype=np.uint64)
+    y = (pis[32:] << np.arange(32, dtype=np.uint64)[:, None]).sum(0, dtype=np.uint64)
+    assert np.array_equal(prod, x * y)
+
+
 # ------------------------------------------------------------------ DATAFLOW schedule
 DF_CASES = [  # (lanes, lane_slabs, interleave, gates per warp)
     (4096, 0, 0, 0), (8192, 0, 1, 1), (16384, 0, 3, 7), (16384, 2, 2, 4), (32768, 2, 1, 32),
