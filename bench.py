@@ -54,6 +54,10 @@ def parse():
     ap.add_argument("--no-pdl", action="store_true", help="disable programmatic dependent launch")
     ap.add_argument("--l2-hints", type=int, default=0, help="kernel A L2 hints: 0 off, 1 stores, 2 +loads")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend (gloo + --same-device: multi-rank test on one GPU)")
+    ap.add_argument("--same-device", action="store_true",
+                    help="test only: every rank uses cuda:0 (timings are NOT a scaling measurement)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-roofline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle CPU time")
@@ -121,13 +125,13 @@ KERNEL_NAMES = {"lut": "k_level_lut_wide<4>", "df": "k_dataflow<1>", "poly": "k_
                 "ab": "k_level_lut_wide<4>", "tile": "k_tile"}
 
 
-def ncu_traffic(kernel: str):
-    """dram read+write bytes per launch of `kernel` from the committed ncu --set full summary
-    (profiles/traffic.json, written by scripts/ncu_summary.py from the same bench command)."""
+def ncu_traffic(config: str, kernel: str):
+    """dram read+write bytes per launch of `kernel` on `config` from the committed ncu --set
+    full summary (profiles/traffic.json, from scripts/ncu_summary.py on the same bench command)."""
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
             d = json.load(f)
-        e = d["kernels"][kernel]
+        e = d["kernels"][f"{config}:{kernel}"]
         return {"traffic_bytes_per_launch": e["traffic_bytes_per_launch"],
                 "source": e.get("source", d.get("source"))}
     except Exception:
@@ -215,9 +219,14 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         print(f"warning: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
+    if args.same_device:
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group("gloo")
 
     cfg = workloads.CONFIGS[args.config]
     nl = cfg.netlist()
@@ -278,7 +287,7 @@ def main():
         kname = KERNEL_NAMES[args.kernel]
         if args.kernel == "df":
             kname = f"k_dataflow<{lanes // (args.lane_slabs or lanes // 4096) // 4096}>"
-        tr = ncu_traffic(kname)
+        tr = ncu_traffic(args.config, kname)
         roof = {"bound": "hbm", "kernel": kname,
                 "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
                 "frac": achieved / pk["hbm_gbs"],
@@ -340,7 +349,9 @@ def main():
                        "pdl": not args.no_pdl, "tile_words": args.tile_words,
                        "tile_groups": args.tile_groups, "l2_hints": args.l2_hints, "lut_k": args.lut_k,
                        "l2": "inputs larger than L2 (state %.1f GB per GPU)" % (info["n_rows"] * lanes / 8 / 1e9),
-                       "parallelism": f"dp{world} (stimulus sharding)", "compile_s": round(compile_s, 2),
+                       "parallelism": f"dp{world} (stimulus sharding)" + (" TEST: all ranks on cuda:0"
+                                                                              if args.same_device else ""),
+                       "compile_s": round(compile_s, 2),
                        "paper_style_gcps": value * (G + info["n_reg"]) / G},
             "gpu_launches": int(launches_per_cycle * (1 if args.kernel == "tile" else C) * args.steps),
             "signature": {k: str(v) for k, v in red.items()},
