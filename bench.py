@@ -121,8 +121,8 @@ def peaks():
         return {"hbm_gbs": 6650.0}, "fallback"
 
 
-KERNEL_NAMES = {"lut": "k_level_lut_wide<4>", "df": "k_dataflow<1>", "poly": "k_level_poly",
-                "ab": "k_level_lut_wide<4>", "tile": "k_tile"}
+KERNEL_NAMES = {"lut": "k_level_lut_wide<4, 0>", "df": "k_dataflow<1>", "poly": "k_level_poly",
+                "ab": "k_level_lut_wide<4, 0>", "tile": "k_tile"}
 
 
 def ncu_traffic(config: str, kernel: str):

@@ -1,0 +1,27 @@
+#!/bin/bash
+# compute-sanitizer over small runs of every kernel: memcheck, racecheck
+# (shared memory of kernel T and its named barriers), synccheck.  usage: bash scripts/sanitize.sh <tag>
+OUT=gpurun_out/${1:-san}
+mkdir -p $OUT
+cat > /tmp/san_run.py <<'PY'
+import sys, numpy as np
+sys.path.insert(0, ".")
+import workloads, paper_conf_ipps_gavierrprs23_b200 as gs
+kernel = sys.argv[1]
+nl = workloads.synthetic(3000, 120, 16, 40, 12, seed=9, name="s")
+prog = gs.Netlist.from_arrays(nl).compile()
+lanes = 8192 if kernel == "df" else 2048
+sim = gs.Sim(prog, lanes, kernel=kernel, trace_words=[0, 5], trace_cycles=4,
+             use_graphs=(kernel != "lut"))
+sim.bind_generated(3)
+sim.step(3)
+sim.read_outputs(); sim.read_registers(); sim.read_lane_signatures(); sim.signature()
+sim.close()
+print("ok", kernel)
+PY
+for k in lut poly ab tile df; do
+  for tool in memcheck racecheck synccheck; do
+    timeout 600 compute-sanitizer --tool $tool --error-exitcode 9 python /tmp/san_run.py $k > $OUT/${k}_${tool}.log 2>&1
+    echo "$k $tool rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY' $OUT/${k}_${tool}.log | tr '\n' ' ')" >> $OUT/summary.txt
+  done
+done
