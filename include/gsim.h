@@ -45,7 +45,9 @@ extern "C" {
 #endif
 
 #define GSIM_VERSION "0.1.0"
-#define GS_MAX_K 6   /* largest LUT fan-in L supported by both kernels ("4, 6 or 8") */
+#define GS_MAX_K 6        /* largest LUT fan-in L of kernels A, T and D (64-bit truth tables) */
+#define GS_MAX_K_POLY 8   /* largest LUT fan-in L of kernel B (the polynomial network) and of
+                             the netlist / compiler ("4, 6 or 8"); tables of 2^8 bits   */
 
 typedef int32_t gs_status;
 enum {
@@ -91,6 +93,11 @@ gs_status gs_add_const(gs_netlist* nl, int value, gs_net* out);
  * the same table under k-bit index reversal).  Bits >= 2^k must be zero. */
 gs_status gs_add_gate(gs_netlist* nl, uint32_t k, const gs_net* in, uint64_t tt, gs_net* out);
 
+/* Same for 0 <= k <= GS_MAX_K_POLY: tt_words holds the table LSB-first in max(1, 2^k / 64)
+ * uint64 words (bit m of the table = bit m % 64 of word m / 64).  Gates with k > GS_MAX_K can
+ * only be simulated by kernel B (GS_KERNEL_POLY; AUTO selects it). */
+gs_status gs_add_gate_wide(gs_netlist* nl, uint32_t k, const gs_net* in, const uint64_t* tt_words, gs_net* out);
+
 /* D flip-flop on the global clock.  *q_out is its Q net (pseudo-input);
  * init (0/1) is Q at cycle 0 (reading R3).  Registers are numbered 0,1,... in
  * creation order (the "reg" index of register read/write layouts). */
@@ -119,8 +126,10 @@ typedef struct {
     const uint8_t* gate_k;        /* [n_gates]                               */
     const uint32_t* gate_in_off;  /* [n_gates+1] CSR offsets, gate_in_off[0]=0 */
     const uint32_t* gate_in;      /* [gate_in_off[n_gates]] net ids          */
-    const uint64_t* gate_tt;      /* [n_gates]   LSB-first truth tables      */
+    const uint64_t* gate_tt;      /* [n_gates]   LSB-first truth tables (bits 0..63) */
     const uint32_t* po;           /* [n_po]      net ids                     */
+    const uint64_t* gate_tt_hi;   /* [n_gates][3] table bits 64..255 of gates with k = 7, 8;
+                                     may be NULL when no gate has k > 6            */
 } gs_netlist_arrays;
 gs_status gs_netlist_load_arrays(gs_netlist* nl, const gs_netlist_arrays* a);
 
@@ -134,7 +143,7 @@ gs_status gs_netlist_get_counts(const gs_netlist* nl, gs_netlist_counts* out);
 typedef struct {
     int balance;      /* 0: ASAP levels.  1: slack-based balancing within [ASAP, ALAP]
                          (same depth; flattens the unbalanced level widths) */
-    uint32_t max_k;   /* reject gates wider than this (0 = GS_MAX_K)                  */
+    uint32_t max_k;   /* reject gates wider than this (0 = GS_MAX_K_POLY)             */
     uint32_t lut_k;   /* 0: evaluate the netlist's LUTs as given.  L in [2, max_k]: first
                          collapse cones into LUTs of at most L inputs (the paper's LUT
                          mapping step and its main hyperparameter L):
@@ -158,7 +167,7 @@ typedef struct {
     uint32_t n_eval_gates;     /* gates evaluated per cycle (k >= 1) = G of the metric   */
     uint32_t n_levels;         /* depth D = number of merged NN layers           */
     uint32_t max_width, min_width;
-    uint32_t k_hist[GS_MAX_K + 1];
+    uint32_t k_hist[GS_MAX_K_POLY + 1];
     uint64_t n_edges;          /* sum of k over evaluated gates                          */
     uint64_t nnz_coeffs;       /* nonzero w_S over all gates ("connections" of the merged
                                   hidden->output layer)                    */
@@ -179,8 +188,9 @@ gs_status gs_program_gate_levels(const gs_program* prog, uint32_t* level, uint32
 gs_status gs_program_coeffs(const gs_program* prog, uint32_t gate, int32_t* w, uint32_t n);
 
 /* The LUT the program evaluates for netlist gate `gate` (after optional cone collapsing):
- * its fan-in *k, input nets in[0..k-1] (in must hold GS_MAX_K entries) and LSB-first truth
- * table *tt.  Without lut_k this is the gate as added; absorbed gates report k = 0. */
+ * its fan-in *k, input nets in[0..k-1] (in must hold GS_MAX_K_POLY entries) and the
+ * LSB-first truth table in tt[0..3] (4 words; words past max(1, 2^k / 64) are zero).
+ * Without lut_k this is the gate as added; absorbed gates report k = 0. */
 gs_status gs_program_gate_lut(const gs_program* prog, uint32_t gate, uint32_t* k, gs_net* in, uint64_t* tt);
 
 /* Shared-memory slots one lane tile of kernel T needs (constants, PIs, two register banks,

@@ -43,7 +43,7 @@ class _Netlist(C.Structure):
                 ("n_po", C.c_uint32),
                 ("reg_init", C.c_void_p), ("reg_d", C.c_void_p), ("gate_k", C.c_void_p),
                 ("gate_in_off", C.c_void_p), ("gate_in", C.c_void_p), ("gate_tt", C.c_void_p),
-                ("po", C.c_void_p)]
+                ("po", C.c_void_p), ("gate_tt_hi", C.c_void_p)]
 
 
 def lib():
@@ -58,6 +58,7 @@ def lib():
                 ("orc_misr_step", u64, [u64, u64]),
                 ("orc_lane_sig_term", u64, [u64, u64]),
                 ("orc_mobius_def", None, [u64, C.c_int, C.c_void_p]),
+                ("orc_mobius_def_wide", None, [C.c_void_p, C.c_int, C.c_void_p]),
                 ("orc_poly_eval", i64, [C.c_void_p, C.c_int, u32]),
                 ("orc_topo_order", C.c_int, [C.c_void_p, C.c_void_p]),
                 ("orc_asap_levels", C.c_int, [C.c_void_p, C.c_void_p]),
@@ -88,6 +89,8 @@ class _NL:
                      np.ascontiguousarray(nl.gate_in, dtype=np.uint32),
                      np.ascontiguousarray(nl.gate_tt, dtype=np.uint64),
                      np.ascontiguousarray(nl.po, dtype=np.uint32)]
+        hi = getattr(nl, "gate_tt_hi", None)
+        self.arrs.append(None if hi is None else np.ascontiguousarray(hi, dtype=np.uint64))
         self.s = _Netlist(nl.n_pi, nl.n_reg, nl.n_gates, nl.n_po, *[_ptr(a) for a in self.arrs])
 
     @property
@@ -120,6 +123,15 @@ def lane_sig_sum(sigs, lanes) -> int:
 def mobius_def(tt: int, k: int) -> list[int]:
     w = np.zeros(1 << k, dtype=np.int64)
     lib().orc_mobius_def(tt, k, _ptr(w))
+    return w.tolist()
+
+
+def mobius_def_wide(words, k: int) -> list[int]:
+    """Definition of the coefficients for a table of up to 256 entries (4 uint64 words)."""
+    t = np.zeros(4, dtype=np.uint64)
+    t[:len(words)] = np.asarray(words, dtype=np.uint64)
+    w = np.zeros(1 << k, dtype=np.int64)
+    lib().orc_mobius_def_wide(_ptr(t), k, _ptr(w))
     return w.tolist()
 
 

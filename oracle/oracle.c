@@ -87,6 +87,20 @@ void orc_mobius_def(uint64_t tt, int k, int64_t* w) {
     }
 }
 
+/* The same definition for tables of up to 2^8 entries given as 4 uint64 words (k <= 8). */
+void orc_mobius_def_wide(const uint64_t* tt4, int k, int64_t* w) {
+    uint32_t n = 1u << k;
+    for (uint32_t S = 0; S < n; ++S) {
+        int64_t acc = 0;
+        for (uint32_t T = 0; T < n; ++T) {
+            if ((T & ~S) != 0) continue;                 /* T must be a subset of S */
+            int64_t f = (int64_t)((tt4[T >> 6] >> (T & 63)) & 1u);
+            acc += ((popc(S) - popc(T)) & 1) ? -f : f;
+        }
+        w[S] = acc;
+    }
+}
+
 /* The two-layer network of Fig. 2 for one input point x (bit i = x_i):
  * hidden neuron h_S = Theta(sum_{s in S} x_s - |S| + 1) (Eq. 3, weights 1,
  * bias |S|-1), Theta(z) = [z > 0] (Eq. 2); output = sum_S w_S h_S (Eq. 1),
@@ -117,7 +131,15 @@ typedef struct {
     const uint32_t* gate_in;
     const uint64_t* gate_tt;
     const uint32_t* po;
+    const uint64_t* gate_tt_hi;   /* [n_gates][3]: table bits 64..255 (k = 7, 8), or NULL */
 } orc_netlist;
+
+/* Bit idx of gate g's truth table (LSB-first, reading R1); tables of k = 7, 8 gates continue
+ * into gate_tt_hi. */
+static uint32_t tt_bit(const orc_netlist* nl, uint32_t g, uint32_t idx) {
+    if (idx < 64) return (uint32_t)((nl->gate_tt[g] >> idx) & 1u);
+    return (uint32_t)((nl->gate_tt_hi[(uint64_t)g * 3 + (idx >> 6) - 1] >> (idx & 63)) & 1u);
+}
 
 /* Kahn topological order of the gate DAG: a gate is ready when all of
  * its gate inputs are done; ties by gate id (FIFO seeded in id order).
@@ -209,6 +231,8 @@ int64_t orc_simulate(const orc_netlist* nl, int mode, uint64_t seed,
     uint32_t* order = (uint32_t*)malloc((G ? G : 1) * sizeof(uint32_t));
     if (orc_topo_order(nl, order) != 0) { free(order); return -1; }
     for (uint32_t r = 0; r < R; ++r) if (nl->reg_d[r] >= N) { free(order); return -1; }
+    for (uint32_t g = 0; g < G; ++g)
+        if (nl->gate_k[g] > 8 || (nl->gate_k[g] > 6 && !nl->gate_tt_hi)) { free(order); return -1; }
     for (uint32_t o = 0; o < O; ++o) if (nl->po[o] >= N) { free(order); return -1; }
 
     /* coefficients of every gate, by definition (mode 1 only) */
@@ -219,7 +243,12 @@ int64_t orc_simulate(const orc_netlist* nl, int mode, uint64_t seed,
         woff[0] = 0;
         for (uint32_t g = 0; g < G; ++g) woff[g + 1] = woff[g] + (1u << nl->gate_k[g]);
         wall = (int64_t*)malloc((woff[G] ? woff[G] : 1) * sizeof(int64_t));
-        for (uint32_t g = 0; g < G; ++g) orc_mobius_def(nl->gate_tt[g], nl->gate_k[g], wall + woff[g]);
+        for (uint32_t g = 0; g < G; ++g) {
+            uint64_t tt4[4] = {nl->gate_tt[g], 0, 0, 0};
+            if (nl->gate_k[g] > 6)
+                for (int j = 0; j < 3; ++j) tt4[1 + j] = nl->gate_tt_hi[(uint64_t)g * 3 + j];
+            orc_mobius_def_wide(tt4, nl->gate_k[g], wall + woff[g]);
+        }
     }
 
     int64_t violations = 0;
@@ -255,7 +284,7 @@ int64_t orc_simulate(const orc_netlist* nl, int mode, uint64_t seed,
                         if (y != 0 && y != 1) violations++;
                         v[base + g] = (uint8_t)(y & 1);
                     } else {
-                        v[base + g] = (uint8_t)((nl->gate_tt[g] >> idx) & 1u);
+                        v[base + g] = (uint8_t)tt_bit(nl, g, idx);
                     }
                 }
                 uint64_t word = 0;

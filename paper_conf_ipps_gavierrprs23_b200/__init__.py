@@ -24,6 +24,7 @@ GS_OK = 0
 GS_ERR_ARG, GS_ERR_ARITY, GS_ERR_UNDRIVEN, GS_ERR_COMB_LOOP = -1, -2, -3, -4
 GS_ERR_BUFFER_TOO_SMALL, GS_ERR_CUDA, GS_ERR_STATE, GS_ERR_NOMEM = -5, -6, -7, -8
 GS_MAX_K = 6
+GS_MAX_K_POLY = 8
 GS_SIM_NO_PDL = 1
 GS_KERNEL_AUTO, GS_KERNEL_LUT, GS_KERNEL_POLY, GS_KERNEL_AB, GS_KERNEL_DATAFLOW = 0, 1, 2, 3, 4
 GS_KERNEL_TILE = 5
@@ -42,7 +43,7 @@ class gs_netlist_arrays(C.Structure):
     _fields_ = [("n_pi", C.c_uint32), ("n_reg", C.c_uint32), ("n_gates", C.c_uint32),
                 ("n_po", C.c_uint32), ("reg_init", C.c_void_p), ("reg_d", C.c_void_p),
                 ("gate_k", C.c_void_p), ("gate_in_off", C.c_void_p), ("gate_in", C.c_void_p),
-                ("gate_tt", C.c_void_p), ("po", C.c_void_p)]
+                ("gate_tt", C.c_void_p), ("po", C.c_void_p), ("gate_tt_hi", C.c_void_p)]
 
 
 class gs_netlist_counts(C.Structure):
@@ -58,7 +59,7 @@ class gs_program_info(C.Structure):
     _fields_ = [("n_pi", C.c_uint32), ("n_reg", C.c_uint32), ("n_po", C.c_uint32),
                 ("n_gates", C.c_uint32), ("n_eval_gates", C.c_uint32), ("n_levels", C.c_uint32),
                 ("max_width", C.c_uint32), ("min_width", C.c_uint32),
-                ("k_hist", C.c_uint32 * (GS_MAX_K + 1)), ("n_edges", C.c_uint64),
+                ("k_hist", C.c_uint32 * (GS_MAX_K_POLY + 1)), ("n_edges", C.c_uint64),
                 ("nnz_coeffs", C.c_uint64), ("hidden_neurons", C.c_uint64), ("n_rows", C.c_uint64),
                 ("program_hash", C.c_uint64)]
 
@@ -101,6 +102,7 @@ _SIGS = {
     "gs_add_input": (C.c_int32, [_P, _P]),
     "gs_add_const": (C.c_int32, [_P, C.c_int, _P]),
     "gs_add_gate": (C.c_int32, [_P, C.c_uint32, _P, C.c_uint64, _P]),
+    "gs_add_gate_wide": (C.c_int32, [_P, C.c_uint32, _P, _P, _P]),
     "gs_add_register": (C.c_int32, [_P, C.c_int, _P]),
     "gs_set_register_d": (C.c_int32, [_P, C.c_uint32, C.c_uint32]),
     "gs_mark_output": (C.c_int32, [_P, C.c_uint32, _P]),
@@ -194,6 +196,8 @@ class Netlist:
                 np.ascontiguousarray(nl.gate_in, dtype=np.uint32),
                 np.ascontiguousarray(nl.gate_tt, dtype=np.uint64),
                 np.ascontiguousarray(nl.po, dtype=np.uint32)]
+        hi = getattr(nl, "gate_tt_hi", None)
+        keep.append(None if hi is None else np.ascontiguousarray(hi, dtype=np.uint64))
         a = gs_netlist_arrays(nl.n_pi, nl.n_reg, nl.n_gates, nl.n_po, *[_p(x) for x in keep])
         _call("gs_netlist_load_arrays", self.h, C.byref(a))
         return self
@@ -209,9 +213,14 @@ class Netlist:
         return n.value
 
     def add_gate(self, ins, tt: int) -> int:
+        """k-input LUT; tt is the LSB-first table as a Python int (up to 2^8 bits)."""
         arr = np.ascontiguousarray(list(ins), dtype=np.uint32)
         n = C.c_uint32()
-        _call("gs_add_gate", self.h, len(arr), _p(arr) if len(arr) else None, int(tt), C.byref(n))
+        if len(arr) <= GS_MAX_K:
+            _call("gs_add_gate", self.h, len(arr), _p(arr) if len(arr) else None, int(tt), C.byref(n))
+        else:
+            words = np.array([(int(tt) >> (64 * i)) & (2**64 - 1) for i in range(4)], dtype=np.uint64)
+            _call("gs_add_gate_wide", self.h, len(arr), _p(arr), _p(words), C.byref(n))
         return n.value
 
     def add_register(self, init: int = 0) -> int:
@@ -262,12 +271,12 @@ class Program:
         return lv[:self.info["n_gates"]]
 
     def gate_lut(self, gate: int) -> tuple[list[int], int]:
-        """(input nets, truth table) of the LUT evaluated for netlist gate `gate`."""
+        """(input nets, truth table as a Python int) of the LUT evaluated for netlist gate `gate`."""
         k = C.c_uint32()
-        ins = np.zeros(GS_MAX_K, dtype=np.uint32)
-        tt = C.c_uint64()
-        _call("gs_program_gate_lut", self.h, int(gate), C.byref(k), _p(ins), C.byref(tt))
-        return ins[:k.value].tolist(), tt.value
+        ins = np.zeros(GS_MAX_K_POLY, dtype=np.uint32)
+        tt = np.zeros(4, dtype=np.uint64)
+        _call("gs_program_gate_lut", self.h, int(gate), C.byref(k), _p(ins), _p(tt))
+        return ins[:k.value].tolist(), sum(int(w) << (64 * i) for i, w in enumerate(tt))
 
     def tile_slots(self) -> int:
         v = C.c_uint32()

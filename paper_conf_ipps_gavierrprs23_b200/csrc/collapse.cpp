@@ -14,6 +14,7 @@
 // PIs and register Qs on every net that is still read, so simulation results are
 // identical (tested against the oracle on the original netlist).
 #include <algorithm>
+#include <array>
 #include <vector>
 
 #include "internal.h"
@@ -23,7 +24,10 @@ namespace gs {
 gs_status collapse_luts(const Netlist& nl, uint32_t L, Netlist& out) {
     const uint32_t N = nl.n_nets(), G = (uint32_t)nl.gate_net.size();
     std::vector<std::vector<uint32_t>> ins(G);
-    std::vector<uint64_t> tt(nl.gate_tt);
+    typedef std::array<uint64_t, 4> T4;                       // tables of up to 2^8 bits
+    std::vector<T4> tt(G);
+    for (uint32_t g = 0; g < G; ++g) nl.table(g, tt[g].data());
+    auto bit = [](const T4& t, uint32_t m) -> uint32_t { return (uint32_t)((t[m >> 6] >> (m & 63)) & 1u); };
     for (uint32_t g = 0; g < G; ++g) {
         ins[g].assign(nl.gate_in.begin() + nl.gate_in_off[g], nl.gate_in.begin() + nl.gate_in_off[g + 1]);
         for (uint32_t n : ins[g])
@@ -73,7 +77,7 @@ gs_status collapse_luts(const Netlist& nl, uint32_t L, Netlist& out) {
             dead[g] = 1;
             for (uint32_t x : distinct(ins[g])) stack.push_back(x);
             ins[g].clear();
-            tt[g] = 0;
+            tt[g] = T4{0, 0, 0, 0};
         }
     };
     for (uint32_t c : order) {
@@ -98,7 +102,7 @@ gs_status collapse_luts(const Netlist& nl, uint32_t L, Netlist& out) {
             const uint32_t gnet = nl.gate_net[best];
             const std::vector<uint32_t>& gi = ins[best];
             const uint32_t K = (uint32_t)best_merged.size();
-            uint64_t nt = 0;
+            T4 nt{0, 0, 0, 0};
             for (uint32_t m = 0; m < (1u << K); ++m) {
                 auto val = [&](uint32_t net) -> uint32_t {
                     const size_t j = std::lower_bound(best_merged.begin(), best_merged.end(), net) - best_merged.begin();
@@ -106,10 +110,10 @@ gs_status collapse_luts(const Netlist& nl, uint32_t L, Netlist& out) {
                 };
                 uint32_t gx = 0;
                 for (size_t i = 0; i < gi.size(); ++i) gx |= val(gi[i]) << i;
-                const uint32_t gv = (uint32_t)((tt[best] >> gx) & 1u);
+                const uint32_t gv = bit(tt[best], gx);
                 uint32_t cx = 0;
                 for (size_t i = 0; i < ins[c].size(); ++i) cx |= (ins[c][i] == gnet ? gv : val(ins[c][i])) << i;
-                nt |= ((tt[c] >> cx) & 1ull) << m;
+                nt[m >> 6] |= (uint64_t)bit(tt[c], cx) << (m & 63);
             }
             // reader bookkeeping: c now reads best_merged instead of its old inputs
             const std::vector<uint32_t> old = distinct(ins[c]);
@@ -128,11 +132,16 @@ gs_status collapse_luts(const Netlist& nl, uint32_t L, Netlist& out) {
     out.gate_k.assign(G, 0);
     out.gate_in_off.assign(G + 1, 0);
     out.gate_in.clear();
+    bool wide = false;
+    for (uint32_t g = 0; g < G; ++g) wide = wide || ins[g].size() > GS_MAX_K;
+    out.gate_tt_hi.assign(wide ? (size_t)G * 3 : 0, 0);
     for (uint32_t g = 0; g < G; ++g) {
         out.gate_k[g] = (uint8_t)ins[g].size();
         out.gate_in.insert(out.gate_in.end(), ins[g].begin(), ins[g].end());
         out.gate_in_off[g + 1] = (uint32_t)out.gate_in.size();
-        out.gate_tt[g] = dead[g] ? 0 : tt[g];
+        out.gate_tt[g] = dead[g] ? 0 : tt[g][0];
+        if (wide && !dead[g])
+            for (int j = 0; j < 3; ++j) out.gate_tt_hi[(size_t)g * 3 + j] = tt[g][1 + j];
     }
     return GS_OK;
 }

@@ -23,9 +23,9 @@ namespace gs {
 // for different variables act on different index bits and commute, so k stages give
 // the same coefficients as the recursion (<= k 2^(k-1) subtractions).  Index
 // bit i <-> x_i in S (LSB-first, reading R1).
-void mobius_butterfly(uint64_t tt, uint32_t k, int32_t* w) {
+void mobius_butterfly(const uint64_t* tt4, uint32_t k, int32_t* w) {
     const uint32_t n = 1u << k;
-    for (uint32_t m = 0; m < n; ++m) w[m] = (int32_t)((tt >> m) & 1u);
+    for (uint32_t m = 0; m < n; ++m) w[m] = (int32_t)((tt4[m >> 6] >> (m & 63)) & 1u);
     for (uint32_t i = 0; i < k; ++i) {
         const uint32_t b = 1u << i;
         for (uint32_t m = 0; m < n; ++m)
@@ -168,16 +168,16 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
 
     // counting sort by (level, k), stable in gate id
     pr.level_off.assign(D + 1, 0);
-    std::vector<uint64_t> bucket((uint64_t)D * (GS_MAX_K + 1) + 1, 0);
+    std::vector<uint64_t> bucket((uint64_t)D * (GS_MAX_K_POLY + 1) + 1, 0);
     for (uint32_t g = 0; g < G; ++g)
-        if (nl.gate_k[g] > 0) bucket[(uint64_t)(level[g] - 1) * (GS_MAX_K + 1) + nl.gate_k[g] + 1]++;
+        if (nl.gate_k[g] > 0) bucket[(uint64_t)(level[g] - 1) * (GS_MAX_K_POLY + 1) + nl.gate_k[g] + 1]++;
     for (size_t i = 1; i < bucket.size(); ++i) bucket[i] += bucket[i - 1];
-    for (uint32_t l = 0; l <= D; ++l) pr.level_off[l] = (uint32_t)bucket[(uint64_t)l * (GS_MAX_K + 1)];
+    for (uint32_t l = 0; l <= D; ++l) pr.level_off[l] = (uint32_t)bucket[(uint64_t)l * (GS_MAX_K_POLY + 1)];
     std::vector<uint32_t> exec_pos(G, NONE32);
     pr.exec_gate.assign(n_eval, 0);
     for (uint32_t g = 0; g < G; ++g)
         if (nl.gate_k[g] > 0) {
-            uint64_t b = (uint64_t)(level[g] - 1) * (GS_MAX_K + 1) + nl.gate_k[g];
+            uint64_t b = (uint64_t)(level[g] - 1) * (GS_MAX_K_POLY + 1) + nl.gate_k[g];
             uint32_t pos = (uint32_t)bucket[b]++;
             exec_pos[g] = pos;
             pr.exec_gate[pos] = g;
@@ -199,16 +199,17 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
     pr.aux.resize(n_eval);
     for (uint32_t g = 0; g < G; ++g)
         if (nl.gate_k[g] > 4) pr.any_wide = true;
-    if (pr.any_wide) pr.in_hi.assign((size_t)n_eval * 2, 0);
+    if (pr.any_wide) pr.in_hi.assign((size_t)n_eval * 4, 0);
     for (uint32_t pos = 0; pos < n_eval; ++pos) {
         uint32_t g = pr.exec_gate[pos];
         uint32_t k = nl.gate_k[g];
         for (uint32_t j = 0; j < k; ++j) {
             uint32_t rr = row_of(nl.gate_in[nl.gate_in_off[g] + j]);
             if (j < 4) pr.in_lo[(size_t)pos * 4 + j] = rr;
-            else pr.in_hi[(size_t)pos * 2 + (j - 4)] = rr;
+            else pr.in_hi[(size_t)pos * 4 + (j - 4)] = rr;
         }
         pr.aux[pos].tt = nl.gate_tt[g];
+        pr.max_k = std::max(pr.max_k, k);
         pr.aux[pos].qdst = NONE32;
         pr.aux[pos].k = k;
     }
@@ -242,6 +243,7 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
     pr.lut_in_off = nl.gate_in_off;
     pr.lut_in = nl.gate_in;
     pr.lut_tt = nl.gate_tt;
+    pr.lut_tt_hi = nl.gate_tt_hi;
 
     // ---------------------------------------------------------------- coefficients
     pr.gate_level.assign(G, 0);
@@ -251,7 +253,11 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
         pr.coeff_off[g + 1] = pr.coeff_off[g] + (1u << nl.gate_k[g]);
     }
     pr.coeffs.assign(pr.coeff_off[G], 0);
-    for (uint32_t g = 0; g < G; ++g) mobius_butterfly(nl.gate_tt[g], nl.gate_k[g], &pr.coeffs[pr.coeff_off[g]]);
+    for (uint32_t g = 0; g < G; ++g) {
+        uint64_t t4[4];
+        nl.table(g, t4);
+        mobius_butterfly(t4, nl.gate_k[g], &pr.coeffs[pr.coeff_off[g]]);
+    }
     pr.term_off.assign(n_eval + 1, 0);
     uint64_t nnz = 0, hidden = 0, edges = 0;
     for (uint32_t pos = 0; pos < n_eval; ++pos) {
@@ -292,6 +298,7 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
     for (uint32_t v : pr.level_off) h = hmix(h, v);
     for (uint32_t v : pr.in_lo) h = hmix(h, v);
     for (uint32_t v : pr.in_hi) h = hmix(h, v);
+    for (uint64_t v : nl.gate_tt_hi) h = hmix(h, v);
     for (const GateAux& a : pr.aux) h = hmix(hmix(h, a.tt), ((uint64_t)a.qdst << 32) | a.k);
     for (uint32_t v : pr.po_rows) h = hmix(h, v);
     for (size_t i = 0; i < pr.latch_src.size(); ++i) h = hmix(h, ((uint64_t)pr.latch_src[i] << 32) | pr.latch_dst[i]);

@@ -31,8 +31,14 @@ struct Netlist {
     std::vector<uint32_t> gate_in_off{0};
     std::vector<uint32_t> gate_in;      // net ids
     std::vector<uint64_t> gate_tt;
+    std::vector<uint64_t> gate_tt_hi;   // [n_gates * 3] table bits 64..255, empty if no k > 6
     std::vector<uint32_t> po_net;
     uint32_t n_nets() const { return (uint32_t)net_kind.size(); }
+    // the 4-word table of gate g (bits beyond 2^k are zero)
+    void table(uint32_t g, uint64_t* t4) const {
+        t4[0] = gate_tt[g];
+        for (int j = 0; j < 3; ++j) t4[1 + j] = gate_tt_hi.empty() ? 0 : gate_tt_hi[(size_t)g * 3 + j];
+    }
 };
 
 // ---------------------------------------------------------------- program
@@ -52,11 +58,12 @@ struct Program {
     uint32_t row_pi0 = 2, row_q0 = 0, row_gate0 = 0;
     uint64_t n_rows = 0;
     bool any_wide = false;                    // some gate has k > 4
+    uint32_t max_k = 0;                       // widest evaluated gate
 
     // execution order = level by level, k-grouped within a level
     std::vector<uint32_t> level_off;          // [n_levels + 1] into exec order
     std::vector<uint32_t> in_lo;              // [n_eval * 4] row refs (QFLAG for Q rows)
-    std::vector<uint32_t> in_hi;              // [n_eval * 2] (inputs 4, 5) if any_wide
+    std::vector<uint32_t> in_hi;              // [n_eval * 4] (inputs 4..7) if any_wide
     std::vector<GateAux> aux;                 // [n_eval]
     std::vector<uint8_t> hot;                 // [n_eval] a gate of the next level reads it
     std::vector<uint32_t> term_off;           // [n_eval + 1] kernel B nonzero terms
@@ -73,6 +80,7 @@ struct Program {
     std::vector<uint8_t> lut_k;               // evaluated LUT of every netlist gate (after
     std::vector<uint32_t> lut_in_off, lut_in; //   optional cone collapsing): k, inputs (net
     std::vector<uint64_t> lut_tt;             //   ids) and truth table
+    std::vector<uint64_t> lut_tt_hi;          //   (bits 64..255, empty if no k > 6)
     std::vector<uint32_t> exec_gate;          // exec index -> netlist gate (for G count / debug)
     gs_program_info info{};
 };
@@ -104,8 +112,9 @@ struct TilePlan {
 
 gs_status tile_plan(const Program& p, TilePlan& t);
 
-// Möbius transform of one LSB-first truth table (Algorithm 1 as an iterative butterfly)
-void mobius_butterfly(uint64_t tt, uint32_t k, int32_t* w);
+// Möbius transform of one LSB-first truth table of up to 2^8 bits (4 words; Algorithm 1
+// as an iterative butterfly)
+void mobius_butterfly(const uint64_t* tt4, uint32_t k, int32_t* w);
 
 }  // namespace gs
 

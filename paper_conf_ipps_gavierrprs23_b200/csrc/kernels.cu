@@ -32,7 +32,7 @@ __device__ __forceinline__ void lut_gate_vec16(const LevelArgs& a, uint32_t gate
     uint32_t r[6];
     r[0] = in.x; r[1] = in.y; r[2] = in.z; r[3] = in.w;
     if (K > 4) {
-        const uint2 hi = __ldg(a.dhi + gate);
+        const uint4 hi = __ldg(a.dhi + gate);
         r[4] = hi.x; r[5] = hi.y;
     }
     uint4 x[K];
@@ -53,7 +53,7 @@ __device__ __forceinline__ void lut_gate_vec8(const LevelArgs& a, uint32_t gate,
     uint32_t r[6];
     r[0] = in.x; r[1] = in.y; r[2] = in.z; r[3] = in.w;
     if (K > 4) {
-        const uint2 hi = __ldg(a.dhi + gate);
+        const uint4 hi = __ldg(a.dhi + gate);
         r[4] = hi.x; r[5] = hi.y;
     }
     uint2 x[K];
@@ -122,7 +122,7 @@ __device__ __forceinline__ void lut_gate_u(const LevelArgs& a, uint32_t gate, ui
     uint32_t r[6];
     r[0] = in.x; r[1] = in.y; r[2] = in.z; r[3] = in.w;
     if (K > 4) {
-        const uint2 hi = __ldg(a.dhi + gate);
+        const uint4 hi = __ldg(a.dhi + gate);
         r[4] = hi.x; r[5] = hi.y;
     }
     const uint4* src[K];
@@ -261,7 +261,7 @@ __device__ __forceinline__ void df_gate(const DfArgs& a, uint32_t gate, uint4 in
     uint32_t r[6];
     r[0] = in.x; r[1] = in.y; r[2] = in.z; r[3] = in.w;
     if (K > 4) {
-        const uint2 hi = __ldg(a.dhi + gate);
+        const uint4 hi = __ldg(a.dhi + gate);
         r[4] = hi.x; r[5] = hi.y;
     }
     const uint4* src[K];
@@ -428,47 +428,49 @@ __global__ void __launch_bounds__(256) k_level_poly(LevelArgs a, uint32_t words3
     const bool valid = j < words32;
     const uint4 in = __ldg(a.din + gate);
     const uint4 au = __ldg(reinterpret_cast<const uint4*>(a.aux) + gate);
-    const uint32_t qdst = au.z, k = au.w & 0xFFu;
-    uint32_t r[6] = {in.x, in.y, in.z, in.w, 0u, 0u};
+    const uint32_t qdst = au.z, k = au.w & 0xFFu;             // k <= GS_MAX_K_POLY = 8
+    uint32_t r[8] = {in.x, in.y, in.z, in.w, 0u, 0u, 0u, 0u};
     if (k > 4) {
-        const uint2 hi = __ldg(a.dhi + gate);
-        r[4] = hi.x; r[5] = hi.y;
+        const uint4 hi = __ldg(a.dhi + gate);
+        r[4] = hi.x; r[5] = hi.y; r[6] = hi.z; r[7] = hi.w;
     }
-    uint32_t x[6];
+    uint32_t x[8];
 #pragma unroll
-    for (int i = 0; i < 6; ++i) {
+    for (int i = 0; i < 8; ++i) {
         x[i] = 0u;
         if (i < (int)k && valid)
             x[i] = __ldg(reinterpret_cast<const uint32_t*>(a.state + (uint64_t)resolve(r[i], a.qcur) * a.stride) + j);
     }
-    // idx[b]: input point of stimulus `lane` in word b
+    // idx[b]: input point of stimulus `lane` in word b (bit i = x_i)
     uint32_t idx[32];
 #pragma unroll
     for (int b = 0; b < 32; ++b) idx[b] = 0u;
 #pragma unroll
-    for (int i = 0; i < 6; ++i) {
+    for (int i = 0; i < 8; ++i) {
         if (i < (int)k) {
 #pragma unroll
             for (int b = 0; b < 32; ++b) idx[b] |= ((__shfl_sync(FULL, x[i], b) >> lane) & 1u) << i;
         }
     }
-    // nonzero terms of this gate: lane t holds terms t and t + 32 (k <= 6 -> <= 64)
+    // nonzero terms of this gate (sparse), 32 at a time: lane t holds term base + t
     const uint32_t t0 = __ldg(a.term_off + gate), nt = __ldg(a.term_off + gate + 1) - t0;
-    const uint32_t myterm0 = lane < nt ? __ldg(a.terms + t0 + lane) : 0u;
-    const uint32_t myterm1 = lane + 32 < nt ? __ldg(a.terms + t0 + 32 + lane) : 0u;
     int acc[32];
 #pragma unroll
     for (int b = 0; b < 32; ++b) acc[b] = 0;
-    for (uint32_t i = 0; i < nt; ++i) {
-        const uint32_t tm = __shfl_sync(FULL, i < 32 ? myterm0 : myterm1, i & 31);
-        const uint32_t S = tm & 0xFFu;                         // monomial S (bit s <-> x_s)
-        const int bias = (int)(int8_t)((tm >> 8) & 0xFFu);     // |S| - 1   (Eq. 3)
-        const int w = (int)(int16_t)(tm >> 16);                // w_S       (Eq. 1)
+    for (uint32_t base = 0; base < nt; base += 32) {
+        const uint32_t myterm = base + lane < nt ? __ldg(a.terms + t0 + base + lane) : 0u;
+        const uint32_t cnt = min(32u, nt - base);
+        for (uint32_t i = 0; i < cnt; ++i) {
+            const uint32_t tm = __shfl_sync(FULL, myterm, i);
+            const uint32_t S = tm & 0xFFu;                         // monomial S (bit s <-> x_s)
+            const int bias = (int)(int8_t)((tm >> 8) & 0xFFu);     // |S| - 1   (Eq. 3)
+            const int w = (int)(int16_t)(tm >> 16);                // w_S       (Eq. 1)
 #pragma unroll
-        for (int b = 0; b < 32; ++b) {
-            // hidden neuron: Theta(sum_{s in S} x_s - |S| + 1) = [popc(idx & S) > |S| - 1]
-            const int h = __popc(idx[b] & S) > bias ? 1 : 0;
-            acc[b] += w * h;
+            for (int b = 0; b < 32; ++b) {
+                // hidden neuron: Theta(sum_{s in S} x_s - |S| + 1) = [popc(idx & S) > |S| - 1]
+                const int h = __popc(idx[b] & S) > bias ? 1 : 0;
+                acc[b] += w * h;
+            }
         }
     }
     uint32_t y = 0u, bad = 0u;

@@ -25,7 +25,7 @@ struct Ctl {
 struct LevelArgs {
     const uint4* din;
     const GateAux* aux;
-    const uint2* dhi;
+    const uint4* dhi;                 // inputs 4..7 (gates with k > 4)
     const uint32_t* term_off;
     const uint32_t* terms;
     uint32_t g0, ng;                  // exec-order gate range of the level
@@ -68,7 +68,7 @@ struct EndArgs {
 struct DfArgs {
     const uint4* din;
     const GateAux* aux;
-    const uint2* dhi;
+    const uint4* dhi;                 // inputs 4..7 (gates with k > 4)
     uint8_t* state;
     uint64_t stride;
     uint32_t row_gate0, qcur, qnext;

@@ -80,7 +80,29 @@ gs_status gs_add_gate(gs_netlist* h, uint32_t k, const gs_net* in, uint64_t tt, 
         for (uint32_t i = 0; i < k; ++i) n.gate_in.push_back(in[i]);
         n.gate_in_off.push_back((uint32_t)n.gate_in.size());
         n.gate_tt.push_back(tt);
+        if (!n.gate_tt_hi.empty()) n.gate_tt_hi.insert(n.gate_tt_hi.end(), 3, 0);
         *out = id;
+        clear_error();
+        return GS_OK;
+    })
+}
+
+gs_status gs_add_gate_wide(gs_netlist* h, uint32_t k, const gs_net* in, const uint64_t* tt_words, gs_net* out) {
+    if (!h || !out || (k && !in) || !tt_words) return fail(GS_ERR_ARG, "gs_add_gate_wide: NULL argument");
+    if (k > GS_MAX_K_POLY) return fail(GS_ERR_ARITY, "gs_add_gate_wide: k > GS_MAX_K_POLY");
+    if (k <= GS_MAX_K) return gs_add_gate(h, k, in, tt_words[0], out);
+    GS_TRY({
+        Netlist& n = h->nl;
+        const uint32_t words = (1u << k) / 64;
+        gs_status st = gs_add_gate(h, 0, nullptr, 0, out);   // allocate the net, then fill it in
+        if (st != GS_OK) return st;
+        n.gate_tt_hi.resize(n.gate_tt.size() * 3, 0);       // from now on 3 words per gate
+        const uint32_t g = (uint32_t)n.gate_net.size() - 1;
+        n.gate_k[g] = (uint8_t)k;                              // k = 0 pushed no inputs
+        for (uint32_t i = 0; i < k; ++i) n.gate_in.push_back(in[i]);
+        n.gate_in_off[g + 1] = (uint32_t)n.gate_in.size();
+        n.gate_tt[g] = tt_words[0];
+        for (uint32_t j = 1; j < 4; ++j) n.gate_tt_hi[(size_t)g * 3 + j - 1] = j < words ? tt_words[j] : 0;
         clear_error();
         return GS_OK;
     })
@@ -143,7 +165,9 @@ gs_status gs_netlist_load_arrays(gs_netlist* h, const gs_netlist_arrays* a) {
         return fail(GS_ERR_ARG, "gs_netlist_load_arrays: gate_in_off[0] must be 0");
     for (uint32_t g = 0; g < a->n_gates; ++g) {
         uint32_t k = a->gate_k[g];
-        if (k > GS_MAX_K) return fail(GS_ERR_ARITY, "gs_netlist_load_arrays: gate with k > GS_MAX_K");
+        if (k > GS_MAX_K_POLY) return fail(GS_ERR_ARITY, "gs_netlist_load_arrays: gate with k > GS_MAX_K_POLY");
+        if (k > GS_MAX_K && !a->gate_tt_hi)
+            return fail(GS_ERR_ARG, "gs_netlist_load_arrays: gates with k > 6 need gate_tt_hi");
         if (a->gate_in_off[g + 1] != a->gate_in_off[g] + k)
             return fail(GS_ERR_ARG, "gs_netlist_load_arrays: gate_in_off inconsistent with gate_k");
         if (k < 6 && (a->gate_tt[g] >> (1u << k)) != 0)
@@ -183,6 +207,15 @@ gs_status gs_netlist_load_arrays(gs_netlist* h, const gs_netlist_arrays* a) {
         if (a->n_gates == 0) n.gate_in_off.assign(1, 0);
         n.gate_in.assign(a->gate_in, a->gate_in + E);
         n.gate_tt.assign(a->gate_tt, a->gate_tt + a->n_gates);
+        n.gate_tt_hi.clear();
+        bool wide = false;
+        for (uint32_t g = 0; g < a->n_gates && !wide; ++g) wide = a->gate_k[g] > GS_MAX_K;
+        if (wide) {
+            n.gate_tt_hi.assign(a->gate_tt_hi, a->gate_tt_hi + (size_t)a->n_gates * 3);
+            for (uint32_t g = 0; g < a->n_gates; ++g)        // bits beyond 2^k must not leak in
+                for (uint32_t j = 0; j < 3; ++j)
+                    if (a->gate_k[g] < 7 || (j + 1) * 64 >= (1u << a->gate_k[g])) n.gate_tt_hi[(size_t)g * 3 + j] = 0;
+        }
         n.po_net.assign(a->po, a->po + a->n_po);
         clear_error();
         return GS_OK;
@@ -207,7 +240,7 @@ gs_status gs_compile(const gs_netlist* h, const gs_compile_opts* opts, gs_progra
     if (!h || !out) return fail(GS_ERR_ARG, "gs_compile: NULL argument");
     gs_compile_opts o{1, 0, 0};
     if (opts) o = *opts;
-    if (o.max_k == 0 || o.max_k > GS_MAX_K) o.max_k = GS_MAX_K;
+    if (o.max_k == 0 || o.max_k > GS_MAX_K_POLY) o.max_k = GS_MAX_K_POLY;
     if (o.lut_k == 1 || o.lut_k > o.max_k)
         return fail(GS_ERR_ARG, "gs_compile: lut_k must be 0 or in [2, max_k]");
     Program* p = nullptr;
@@ -279,7 +312,8 @@ gs_status gs_program_gate_lut(const gs_program* prog, uint32_t gate, uint32_t* k
     if (gate >= p.n_gates) return fail(GS_ERR_ARG, "gs_program_gate_lut: gate out of range");
     *k = p.lut_k[gate];
     for (uint32_t j = 0; j < *k; ++j) in[j] = p.lut_in[p.lut_in_off[gate] + j];
-    *tt = p.lut_tt[gate];
+    tt[0] = p.lut_tt[gate];
+    for (uint32_t j = 0; j < 3; ++j) tt[1 + j] = p.lut_tt_hi.empty() ? 0 : p.lut_tt_hi[(size_t)gate * 3 + j];
     clear_error();
     return GS_OK;
 }

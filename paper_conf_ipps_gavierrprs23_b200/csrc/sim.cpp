@@ -116,6 +116,10 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
 gs_sim_opts resolve_auto(const Program& p, const gs_sim_opts& o) {
     gs_sim_opts r = o;
     if (o.kernel != GS_KERNEL_AUTO) return r;
+    if (p.max_k > GS_MAX_K) {                   // 7-8-input LUTs: only the polynomial network
+        r.kernel = GS_KERNEL_POLY;
+        return r;
+    }
     r.kernel = GS_KERNEL_TILE;
     Plans pl;
     const std::string saved = gs_last_error();
@@ -141,7 +145,7 @@ Layout make_layout(const Program& p, const gs_sim_opts& o, const Plans& pl) {
     L.state = take((size_t)p.n_rows * stride);
     L.din = take((size_t)p.n_eval * 16);
     L.aux = take((size_t)p.n_eval * 16);
-    L.dhi = take(p.any_wide ? (size_t)p.n_eval * 8 : 0);
+    L.dhi = take(p.any_wide ? (size_t)p.n_eval * 16 : 0);
     L.term_off = take(poly ? ((size_t)p.n_eval + 1) * 4 : 0);
     L.terms = take(poly ? p.terms.size() * 4 : 0);
     L.po_rows = take((size_t)p.n_po * 4);
@@ -215,7 +219,7 @@ static LevelArgs level_args(const gs_sim* s, uint32_t l, uint32_t parity) {
     LevelArgs a{};
     a.din = s->at<const uint4>(s->L.din);
     a.aux = s->at<const GateAux>(s->L.aux);
-    a.dhi = p.any_wide ? s->at<const uint2>(s->L.dhi) : nullptr;
+    a.dhi = p.any_wide ? s->at<const uint4>(s->L.dhi) : nullptr;
     a.term_off = s->at<const uint32_t>(s->L.term_off);
     a.terms = s->at<const uint32_t>(s->L.terms);
     a.g0 = p.level_off[l];
@@ -284,7 +288,7 @@ static cudaError_t dataflow_launch(const gs_sim* s, uint32_t parity, cudaStream_
     DfArgs a{};
     a.din = s->at<const uint4>(s->L.din);
     a.aux = s->at<const GateAux>(s->L.aux);
-    a.dhi = p.any_wide ? s->at<const uint2>(s->L.dhi) : nullptr;
+    a.dhi = p.any_wide ? s->at<const uint4>(s->L.dhi) : nullptr;
     a.state = s->state();
     a.stride = s->stride;
     a.row_gate0 = p.row_gate0;
@@ -423,6 +427,8 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
     if (!prog || !opts_in || !out || !dev_ws) return fail(GS_ERR_ARG, "gs_sim_create: NULL argument");
     const gs_sim_opts resolved = resolve_auto(*prog->p, *opts_in);
     const gs_sim_opts* opts = &resolved;
+    if (prog->p->max_k > GS_MAX_K && opts->kernel != GS_KERNEL_POLY)
+        return fail(GS_ERR_ARITY, "gs_sim_create: gates with k > 6 are evaluated only by kernel B (GS_KERNEL_POLY)");
     if (opts->lanes == 0 || opts->lanes % 64) return fail(GS_ERR_ARG, "gs_sim_create: lanes must be a positive multiple of 64");
     if (opts->lane_offset % 64) return fail(GS_ERR_ARG, "gs_sim_create: lane_offset must be a multiple of 64");
     if (opts->kernel < GS_KERNEL_AUTO || opts->kernel > GS_KERNEL_TILE) return fail(GS_ERR_ARG, "gs_sim_create: bad kernel");

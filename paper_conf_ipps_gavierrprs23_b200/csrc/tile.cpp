@@ -20,6 +20,7 @@ namespace gs {
 gs_status tile_plan(const Program& p, TilePlan& t) {
     const uint32_t P = p.n_pi, R = p.n_reg, G = p.n_eval, D = p.n_levels;
     t = TilePlan();
+    if (p.max_k > GS_MAX_K) return fail(GS_ERR_ARITY, "TILE: gates with k > 6 need kernel B (GS_KERNEL_POLY)");
     t.q0 = 2 + P;
     const uint32_t fixed = 2 + P + 2 * R;
     // row ref (state row, QFLAG for Q) -> which gate (exec index) it names, or NONE32
@@ -39,7 +40,7 @@ gs_status tile_plan(const Program& p, TilePlan& t) {
     };
     for (uint32_t g = 0; g < G; ++g) {
         const uint32_t k = p.aux[g].k;
-        for (uint32_t j = 0; j < k; ++j) use(j < 4 ? p.in_lo[(size_t)g * 4 + j] : p.in_hi[(size_t)g * 2 + j - 4], lvl[g]);
+        for (uint32_t j = 0; j < k; ++j) use(j < 4 ? p.in_lo[(size_t)g * 4 + j] : p.in_hi[(size_t)g * 4 + j - 4], lvl[g]);
     }
     for (uint32_t r : p.po_rows) use(r, D + 1);
     for (uint32_t r : p.latch_src) use(r, D + 1);
@@ -74,7 +75,7 @@ gs_status tile_plan(const Program& p, TilePlan& t) {
         const uint32_t k = p.aux[g].k;
         uint32_t in[6] = {0, 0, 0, 0, 0, 0};        // unused inputs read const0 (slot 0)
         for (uint32_t j = 0; j < k; ++j)
-            in[j] = slot_of(j < 4 ? p.in_lo[(size_t)g * 4 + j] : p.in_hi[(size_t)g * 2 + j - 4]);
+            in[j] = slot_of(j < 4 ? p.in_lo[(size_t)g * 4 + j] : p.in_hi[(size_t)g * 4 + j - 4]);
         const uint64_t tt = p.aux[g].tt;
         TileDesc d;
         d.in01 = in[0] | (in[1] << 16);

@@ -21,7 +21,7 @@ sys.path.insert(0, ROOT)
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--configs", default="C1,C2,C3")
-    ap.add_argument("--Ls", default="0,3,4,5,6")
+    ap.add_argument("--Ls", default="0,3,4,5,6,7,8")
     ap.add_argument("--kernels", default="lut,auto")
     ap.add_argument("--cycles", type=int, default=100)
     ap.add_argument("--steps", type=int, default=3)
@@ -39,7 +39,10 @@ def main():
             info = prog.info
             for kernel in a.kernels.split(","):
                 stream = torch.cuda.Stream()
-                sim = gs.Sim(prog, lanes, kernel=kernel, stream=stream)
+                try:
+                    sim = gs.Sim(prog, lanes, kernel=kernel, stream=stream)
+                except gs.GsError:               # k > 6 LUTs: kernel B only
+                    continue
                 sim.bind_generated(cfg.stim_seed)
                 sim.step(a.cycles)
                 sim.sync()
@@ -52,7 +55,8 @@ def main():
                 s = e0.elapsed_time(e1) / 1e3
                 evals = lanes * a.cycles * a.steps
                 print(json.dumps({"config": name, "L": L, "kernel": kernel,
-                                  "kernel_used": "tile" if sim.launches_per_cycle() == 1 else kernel,
+                                  "kernel_used": ("tile" if sim.launches_per_cycle() == 1 else
+                                                  "poly" if info["k_hist"][7] + info["k_hist"][8] else kernel),
                                   "levels": info["n_levels"], "luts": info["n_eval_gates"],
                                   "lut_inputs": info["n_edges"], "nnz_coeffs": info["nnz_coeffs"],
                                   "gates_original": g_orig, "lanes": lanes,

@@ -25,20 +25,24 @@ def collapsed_netlist(nl, L, balance=True):
         tts.append(t)
     off = np.zeros(nl.n_gates + 1, dtype=np.int64)
     off[1:] = np.cumsum(ks)
+    lo = np.array([t & (2**64 - 1) for t in tts], dtype=np.uint64)
+    hi = np.array([[(t >> (64 * j)) & (2**64 - 1) for j in (1, 2, 3)] for t in tts], dtype=np.uint64)
     c = workloads.Netlist(nl.n_pi, nl.reg_init, nl.reg_d, np.array(ks, dtype=np.uint8),
-                          off.astype(np.uint32), np.array(ins, dtype=np.uint32),
-                          np.array(tts, dtype=np.uint64), nl.po, name=nl.name + f"_L{L}", meta=nl.meta)
+                          off.astype(np.uint32), np.array(ins, dtype=np.uint32), lo, nl.po,
+                          name=nl.name + f"_L{L}", meta=nl.meta,
+                          gate_tt_hi=hi if max(ks, default=0) > 6 else None)
     return prog, c
 
 
 CASES = [("adder", lambda: workloads.adder(8)), ("mult8", lambda: workloads.array_multiplier(8)),
+         ("wide8", lambda: workloads.random_tiny(7, n_pi=6, n_reg=4, n_gates=80, n_po=10, max_k=8)),
          ("tiny3", lambda: workloads.random_tiny(3, n_pi=5, n_reg=4, n_gates=120, n_po=10)),
          ("tiny9", lambda: workloads.random_tiny(9, n_pi=6, n_reg=6, n_gates=200, n_po=12, max_k=3)),
          ("regs", workloads.register_edge_cases), ("probes", workloads.probes_circuit),
          ("synth", lambda: workloads.synthetic(3000, 120, 16, 40, 12, seed=9, name="s"))]
 
 
-@pytest.mark.parametrize("L", [2, 3, 4, 6])
+@pytest.mark.parametrize("L", [2, 3, 4, 6, 8])
 @pytest.mark.parametrize("name,make", CASES)
 def test_collapsed_netlist_simulates_identically(name, make, L):
     nl = make()
@@ -90,7 +94,7 @@ def test_collapse_depth_never_increases_and_multiplier_halves():
 
 def test_lut_k_argument_checks():
     nl = gs.Netlist.from_arrays(workloads.adder(4))
-    for bad in (1, 7):
+    for bad in (1, 9):
         with pytest.raises(gs.GsError) as e:
             nl.compile(lut_k=bad)
         assert e.value.code == gs.GS_ERR_ARG

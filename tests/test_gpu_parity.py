@@ -329,6 +329,55 @@ def test_collapsed_multiplier_all_lanes_equal_a_times_b():
     assert np.array_equal(prod, x * y)
 
 
+# ------------------------------------------------------------------ 7-8-input LUTs (kernel B)
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_wide_luts_kernel_b_all_lanes_vs_oracle(seed):
+    """Gates with k = 7, 8 (256-bit tables, up to 256 sparse terms per neuron group): only
+    the polynomial network evaluates them; AUTO selects it, the LUT kernels refuse."""
+    nl = workloads.random_tiny(seed, n_pi=8, n_reg=6, n_gates=250, n_po=14, max_k=8)
+    assert (nl.gate_k > 6).any()
+    prog = compile_nl(nl)
+    for kernel in ("poly", "auto"):
+        r = run_gpu(nl, 4096, 9, kernel, seed=31, prog=prog, trace_words=[0, 17, 63])
+        o = oracle.simulate(nl, np.arange(4096), 9, seed=31)
+        assert np.array_equal(gs.unpack_lanes(r["outputs"]).T, o["last"])
+        assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"])
+        assert np.array_equal(r["sigs"], o["sig"])
+        rows = np.concatenate([np.arange(0, 64), np.arange(17 * 64, 18 * 64), np.arange(63 * 64, 64 * 64)])
+        assert np.array_equal(gpu_trace_bits(r["trace"], None), o["trace"][rows])
+        assert r["signature"]["invariant_violations"] == 0
+    for kernel in ("lut", "ab", "tile", "df"):
+        with pytest.raises(gs.GsError) as e:
+            gs.Sim(prog, 4096, kernel=kernel)
+        assert e.value.code == gs.GS_ERR_ARITY
+
+
+@pytest.mark.parametrize("L", [7, 8])
+def test_collapsed_to_8_input_luts_closed_forms(L):
+    """The paper's L = 7 regime: the adder and the multiplier collapsed into <= L-input
+    LUTs and run on kernel B still give a+b (exhaustively) and a*b (1M lanes)."""
+    nl = workloads.adder(8)
+    prog = gs.Netlist.from_arrays(nl).compile(lut_k=L)
+    a = np.arange(1 << 16) & 0xFF
+    b = np.arange(1 << 16) >> 8
+    bits = np.concatenate([(a[None, :] >> np.arange(8)[:, None]) & 1,
+                           (b[None, :] >> np.arange(8)[:, None]) & 1]).astype(np.uint8)
+    words = np.packbits(bits, axis=1, bitorder="little").view(np.uint64)[None]
+    e = run_gpu(nl, 1 << 16, 1, "auto", host_stim=words, prog=prog)
+    out = gs.unpack_lanes(e["outputs"]).astype(np.int64)
+    assert np.array_equal((out << np.arange(9)[:, None]).sum(0), a + b)
+    cfg = workloads.CONFIGS["C2"]
+    prog = gs.Netlist.from_arrays(cfg.netlist()).compile(lut_k=L)
+    r = run_gpu(cfg.netlist(), cfg.lanes, 1, "auto", seed=cfg.stim_seed, prog=prog)
+    assert r["signature"]["invariant_violations"] == 0
+    bits = gs.unpack_lanes(r["outputs"]).astype(np.uint64)
+    prod = (bits << np.arange(64, dtype=np.uint64)[:, None]).sum(0, dtype=np.uint64)
+    pis = _ref.pi_lanes_np(cfg.stim_seed, 64, 0, cfg.lanes).astype(np.uint64)
+    x = (pis[:32] << np.arange(32, dtype=np.uint64)[:, None]).sum(0, dtype=np.uint64)
+    y = (pis[32:] << np.arange(32, dtype=np.uint64)[:, None]).sum(0, dtype=np.uint64)
+    assert np.array_equal(prod, x * y)
+
+
 # ------------------------------------------------------------------ DATAFLOW schedule
 DF_CASES = [  # (lanes, lane_slabs, interleave, gates per warp)
     (4096, 0, 0, 0), (8192, 0, 1, 1), (16384, 0, 3, 7), (16384, 2, 2, 4), (32768, 2, 1, 32),

@@ -58,6 +58,23 @@ def test_mobius_other_arities_match_definition(k):
         assert prog.coeffs(g, k) == oracle.mobius_def(tt, k)
 
 
+@pytest.mark.parametrize("k", [7, 8])
+def test_mobius_wide_gates_match_definition(k):
+    """k = 7, 8 (kernel B only): library Möbius butterfly vs the oracle's definition."""
+    rng = np.random.default_rng(k)
+    n = gs.Netlist()
+    x = [n.add_input() for _ in range(k)]
+    tts = []
+    for _ in range(20):
+        words = rng.integers(0, np.iinfo(np.uint64).max, size=(1 << k) // 64, dtype=np.uint64, endpoint=True)
+        tts.append(words)
+        g = n.add_gate(x, sum(int(w) << (64 * i) for i, w in enumerate(words)))
+        n.mark_output(g)
+    prog = n.compile()
+    for g, words in enumerate(tts):
+        assert prog.coeffs(g, k) == oracle.mobius_def_wide(words, k)
+
+
 def _alap(nl, asap, depth):
     G = nl.n_gates
     base = nl.n_pi + nl.n_reg
@@ -118,8 +135,11 @@ def test_program_info_counts():
     assert inf["n_rows"] == 2 + nl.n_pi + 2 * nl.n_reg + inf["n_eval_gates"]
 
 
-def test_incremental_equals_bulk_load():
-    nl = workloads.register_edge_cases()
+@pytest.mark.parametrize("make", [workloads.register_edge_cases,
+                                  lambda: workloads.random_tiny(5, n_pi=6, n_reg=4, n_gates=60, n_po=8,
+                                                                max_k=8)])
+def test_incremental_equals_bulk_load(make):
+    nl = make()
     bulk = _compile(nl)
     n = gs.Netlist()
     pis = [n.add_input() for _ in range(nl.n_pi)]
@@ -129,10 +149,13 @@ def test_incremental_equals_bulk_load():
     # gates are created in netlist order; constants via gs_add_const
     for g in range(nl.n_gates):
         k = int(nl.gate_k[g])
+        tt = int(nl.gate_tt[g])
+        if nl.gate_tt_hi is not None:
+            tt |= sum(int(w) << (64 * (j + 1)) for j, w in enumerate(nl.gate_tt_hi[g]))
         if k == 0:
-            ids.append(n.add_const(int(nl.gate_tt[g])))
+            ids.append(n.add_const(tt))
         else:
-            ids.append(n.add_gate([ids[x] for x in nl.inputs_of(g)], int(nl.gate_tt[g])))
+            ids.append(n.add_gate([ids[x] for x in nl.inputs_of(g)], tt))
     for r, d in enumerate(nl.reg_d):
         n.set_register_d(qs[r], ids[int(d)])
     for o in nl.po:
@@ -160,13 +183,19 @@ def test_errors():
     assert e.value.code == gs.GS_ERR_UNDRIVEN
     # arity
     n = gs.Netlist()
-    x = [n.add_input() for _ in range(7)]
+    x = [n.add_input() for _ in range(9)]
     with pytest.raises(gs.GsError) as e:
-        n.add_gate(x, 1)
+        n.add_gate(x, 1)                                  # k = 9 > GS_MAX_K_POLY
     assert e.value.code == gs.GS_ERR_ARITY
     n.add_gate(x[:5], 1)
     with pytest.raises(gs.GsError) as e:
         n.compile(max_k=4)
+    assert e.value.code == gs.GS_ERR_ARITY
+    g7 = n.add_gate(x[:7], (1 << 127) | 1)               # k = 7: a 128-bit table
+    n.mark_output(g7)
+    assert n.compile().info["k_hist"][7] == 1
+    with pytest.raises(gs.GsError) as e:
+        n.compile(max_k=6)
     assert e.value.code == gs.GS_ERR_ARITY
     # truth table wider than 2^k
     with pytest.raises(gs.GsError) as e:

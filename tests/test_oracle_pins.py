@@ -122,6 +122,31 @@ def test_algorithm1_literal_equals_definition():
         assert mobius.coeffs_alg1(int(tt), 6) == oracle.mobius_def(int(tt), 6)
 
 
+@pytest.mark.parametrize("k", [7, 8])
+def test_wide_gates_algorithm1_definition_and_eq1(k):
+    """k = 7, 8 (the paper's L = 7 regime, Table I): Algorithm 1 read literally equals the
+    inclusion-exclusion definition, Eq. 1 reproduces the table at all 2^k points, the
+    coefficients obey |w_S| <= 2^{|S|-1} (so int16 holds them) and the Theta network of
+    Eq. 2-3 outputs exactly f."""
+    rng = np.random.default_rng(k)
+    n = 1 << k
+    for trial in range(4):
+        words = rng.integers(0, np.iinfo(np.uint64).max, size=n // 64, dtype=np.uint64, endpoint=True)
+        tt = sum(int(w) << (64 * i) for i, w in enumerate(words))
+        w = oracle.mobius_def_wide(words, k)
+        assert mobius.coeffs_alg1(tt, k) == w
+        for x in range(n):
+            assert sum(w[S] for S in range(n) if (S & ~x) == 0) == (tt >> x) & 1
+        assert all(abs(w[S]) <= max(1, 2 ** (bin(S).count("1") - 1)) for S in range(n))
+        for x in rng.integers(0, n, size=40):
+            assert oracle.poly_eval(w, k, int(x)) == (tt >> int(x)) & 1
+    # parity_8 attains the bound: w_S = (-1)^{|S|+1} 2^{|S|-1}
+    par = sum(((bin(m).count("1") & 1) << m) for m in range(n))
+    wp = oracle.mobius_def_wide([(par >> (64 * i)) & (2**64 - 1) for i in range(n // 64)], k)
+    assert all(wp[S] == (0 if S == 0 else (-1) ** (bin(S).count("1") + 1) * 2 ** (bin(S).count("1") - 1))
+               for S in range(n))
+
+
 def test_algorithm1_operation_count():
     # P:183: "our algorithm requires at most 2^L L operations"
     for L in range(0, 12):
@@ -256,6 +281,15 @@ def test_register_edge_cases_closed_forms():
 
 # ---------------------------------------------------------------- brute force, different algorithm
 
+def _full_tt(nl, g):
+    """The whole truth table of gate g as one Python int (k <= 8: up to 4 words)."""
+    t = int(nl.gate_tt[g])
+    if nl.gate_tt_hi is not None:
+        for j in range(3):
+            t |= int(nl.gate_tt_hi[g, j]) << (64 * (j + 1))
+    return t
+
+
 def _recursive_eval(nl, pis, q):
     """Value of every net by memoised recursion on the definition (no topological sort)."""
     base = nl.n_pi + nl.n_reg
@@ -272,7 +306,7 @@ def _recursive_eval(nl, pis, q):
         idx = 0
         for j, x in enumerate(nl.inputs_of(g).tolist()):
             idx |= val(x) << j
-        memo[n] = (int(nl.gate_tt[g]) >> idx) & 1
+        memo[n] = (_full_tt(nl, g) >> idx) & 1
         return memo[n]
     return val
 
@@ -280,7 +314,7 @@ def _recursive_eval(nl, pis, q):
 @pytest.mark.parametrize("seed", range(12))
 def test_tiny_netlists_bruteforce(seed):
     nl = workloads.random_tiny(seed, n_pi=4, n_reg=3, n_gates=25, n_po=6,
-                               max_k=4 if seed % 3 else 6)
+                               max_k=(4, 6, 8)[seed % 3])
     cycles = 5
     lanes = np.arange(64, dtype=np.uint64)
     stim = workloads.random_host_stimulus(100 + seed, cycles, nl.n_pi, 1)

@@ -13,10 +13,13 @@ include/gsim.h):
 * net ids ``[n_pi, n_pi + n_reg)``      register outputs Q (the FF "pseudo-inputs",
                                         PAPER.md P:237-241)
 * net ids ``[n_pi + n_reg, ...)``       gate outputs, gate g is net n_pi + n_reg + g
-* ``gate_k[g]``                         fan-in k of gate g (0 <= k <= 6; L of P:167)
+* ``gate_k[g]``                         fan-in k of gate g (0 <= k <= 8; L of P:167)
 * ``gate_in[gate_in_off[g]:gate_in_off[g+1]]`` input nets x_0..x_{k-1}
 * ``gate_tt[g]``                        truth table, LSB-first: bit m = f(x) with
-                                        x_i = bit i of m (reading R1)
+                                        x_i = bit i of m (DESIGN.md reading R1);
+                                        bits 0..63
+* ``gate_tt_hi[g]`` (optional)          bits 64..255 of the table as 3 more uint64
+                                        words, for gates with k = 7, 8 (None if none)
 * ``reg_init[r]``, ``reg_d[r]``         initial Q and the net feeding D (the FF
                                         "pseudo-output", P:241)
 * ``po[o]``                             primary-output nets
@@ -87,6 +90,7 @@ class Netlist:
     po: np.ndarray                # uint32 [n_po]
     name: str = ""
     meta: dict = field(default_factory=dict)
+    gate_tt_hi: np.ndarray | None = None   # uint64 [n_gates][3] (k = 7, 8) or None
 
     @property
     def n_reg(self) -> int:
@@ -137,7 +141,8 @@ class Netlist:
             ins[off[j]:off[j + 1]] = self.inputs_of(int(perm[j]))
         return Netlist(self.n_pi, self.reg_init.copy(), remap(self.reg_d), k.copy(),
                        off.astype(U32), remap(ins), self.gate_tt[perm].copy(), remap(self.po),
-                       name=self.name + "+perm", meta=dict(self.meta))
+                       name=self.name + "+perm", meta=dict(self.meta),
+                       gate_tt_hi=None if self.gate_tt_hi is None else self.gate_tt_hi[perm].copy())
 
 
 class Builder:
@@ -516,11 +521,13 @@ def synthetic(n_gates: int, n_reg: int, n_pi: int, n_po: int, depth: int, seed: 
 
 def random_tiny(seed: int, n_pi: int = 4, n_reg: int = 3, n_gates: int = 30,
                 n_po: int = 6, max_k: int = 4) -> Netlist:
-    """Tiny random sequential netlist (brute-force tests): gates only read earlier nets."""
+    """Tiny random sequential netlist (brute-force tests): gates only read earlier nets.
+    max_k up to 8: tables of k = 7, 8 gates spill into ``gate_tt_hi``."""
     rng = np.random.default_rng(seed)
     base = n_pi + n_reg
     ks = rng.integers(0, max_k + 1, size=n_gates).astype(np.uint8)
     ins, tts = [], []
+    hi = np.zeros((n_gates, 3), dtype=np.uint64)
     for g in range(n_gates):
         k = int(ks[g])
         avail = base + g
@@ -528,11 +535,17 @@ def random_tiny(seed: int, n_pi: int = 4, n_reg: int = 3, n_gates: int = 30,
             k = 0
             ks[g] = 0
         ins.extend(int(x) for x in rng.integers(0, avail, size=k))
-        tts.append(int(rng.integers(0, 1 << (1 << k), dtype=np.uint64)) if k < 6 else
-                   int(rng.integers(0, 2**63, dtype=np.int64)))
+        if k < 6:
+            tts.append(int(rng.integers(0, 1 << (1 << k), dtype=np.uint64)))
+        else:
+            words = rng.integers(0, np.iinfo(np.uint64).max, size=4, dtype=np.uint64, endpoint=True)
+            nw = (1 << k) // 64
+            tts.append(int(words[0]))
+            hi[g, :nw - 1] = words[1:nw]
     off = np.zeros(n_gates + 1, dtype=np.int64)
     off[1:] = np.cumsum(ks.astype(np.int64))
     return Netlist(n_pi, rng.integers(0, 2, size=n_reg).astype(np.uint8),
                    rng.integers(0, base + n_gates, size=n_reg).astype(U32), ks,
                    off.astype(U32), np.array(ins, dtype=U32), np.array(tts, dtype=np.uint64),
-                   rng.integers(0, base + n_gates, size=n_po).astype(U32), name=f"tiny{seed}")
+                   rng.integers(0, base + n_gates, size=n_po).astype(U32), name=f"tiny{seed}",
+                   gate_tt_hi=hi if max_k > 6 else None)
