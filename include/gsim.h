@@ -280,6 +280,19 @@ gs_status gs_sim_reset(gs_sim* sim);
  * host/device stimulus would run past its bound cycles. */
 gs_status gs_sim_step(gs_sim* sim, uint32_t ncycles);
 gs_status gs_sim_sync(gs_sim* sim);
+
+/* Paper-style streamed run (the binary inputs are transferred to the GPU and the
+ * binary outputs read back, inside the timed region): step `ncycles` cycles with stimuli
+ * taken from host_stim [ncycles][n_pi][W] and EVERY output of EVERY cycle written to
+ * host_out [ncycles][n_po][W] (NULL = no output stream), W = lanes/64.  Chunks of
+ * `chunk` cycles (0 = 25) are pipelined: the host->device copy of chunk i+1 and the
+ * device->host copy of chunk i-1 run on a library-owned copy stream while chunk i is
+ * computed (pinned host buffers required for overlap).  Uses a library-owned device
+ * staging buffer (2 x chunk of inputs and outputs, freed by gs_sim_destroy).  Asynchronous
+ * on the sim's stream: host_out is complete after gs_sim_sync.  Afterwards the stimulus
+ * binding is the last chunk (bind again before gs_sim_step). */
+gs_status gs_sim_run_streamed(gs_sim* sim, const uint64_t* host_stim, uint64_t* host_out, uint32_t ncycles,
+                              uint32_t chunk);
 gs_status gs_sim_get_cycle(const gs_sim* sim, uint64_t* cycle);
 
 /* Readback (synchronous).  Layouts, with W = lanes/64 local words:

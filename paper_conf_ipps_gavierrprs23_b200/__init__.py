@@ -125,6 +125,7 @@ _SIGS = {
     "gs_sim_reset": (C.c_int32, [_P]),
     "gs_sim_step": (C.c_int32, [_P, C.c_uint32]),
     "gs_sim_sync": (C.c_int32, [_P]),
+    "gs_sim_run_streamed": (C.c_int32, [_P, _P, _P, C.c_uint32, C.c_uint32]),
     "gs_sim_get_cycle": (C.c_int32, [_P, _P]),
     "gs_sim_read_outputs": (C.c_int32, [_P, _P, C.c_size_t]),
     "gs_sim_read_registers": (C.c_int32, [_P, _P, C.c_size_t]),
@@ -353,6 +354,15 @@ class Sim:
 
     def sync(self):
         _call("gs_sim_sync", self.h)
+
+    def run_streamed(self, stim: np.ndarray, out: np.ndarray | None = None, chunk: int = 0):
+        """Stream stim [cycles][n_pi][W] in and every output [cycles][n_po][W] out (async;
+        pinned arrays for overlap; call sync() before reading `out`)."""
+        assert stim.dtype == np.uint64 and stim.flags.c_contiguous and stim.shape[2] == self.words
+        if out is not None:
+            assert out.dtype == np.uint64 and out.flags.c_contiguous and out.shape == (stim.shape[0], self.n_po, self.words)
+        self._stim_keep = (stim, out)
+        _call("gs_sim_run_streamed", self.h, _p(stim), _p(out), int(stim.shape[0]), int(chunk))
 
     @property
     def cycle(self) -> int:

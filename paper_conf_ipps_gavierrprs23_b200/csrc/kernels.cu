@@ -579,6 +579,10 @@ __global__ void __launch_bounds__(256) k_end_cycle(EndArgs a, uint32_t latch_blo
         if (t < (uint64_t)64 * a.words) {
             const uint32_t j = (uint32_t)(t / a.words), w = (uint32_t)(t - (uint64_t)j * a.words);
             const int32_t slot = (a.trace && c < a.trace_cap) ? __ldg(a.trace_slot + w) : -1;
+            unsigned long long* sink = nullptr;                  // full per-cycle output stream
+            if (a.ctl->sink_ptr && c - a.ctl->sink_base < a.ctl->sink_cycles)
+                sink = reinterpret_cast<unsigned long long*>(a.ctl->sink_ptr) +
+                       (c - a.ctl->sink_base) * a.n_po * (uint64_t)a.words;
             unsigned long long v = 0;
             for (uint32_t o = j; o < a.n_po; o += 64) {
                 const uint32_t row = resolve(__ldg(a.po_rows + o), a.qcur);
@@ -586,6 +590,7 @@ __global__ void __launch_bounds__(256) k_end_cycle(EndArgs a, uint32_t latch_blo
                 v ^= x;
                 pop += __popcll(x);
                 if (slot >= 0) a.trace[((uint64_t)c * a.n_po + o) * a.ntw + slot] = x;
+                if (sink) sink[(uint64_t)o * a.words + w] = x;
             }
             const unsigned long long prev = j ? a.misr_cur[(uint64_t)(j - 1) * a.words + w] : 0ULL;
             const unsigned long long fb = ((MISR_POLY >> j) & 1ULL) ? a.misr_cur[(uint64_t)63 * a.words + w] : 0ULL;
@@ -616,6 +621,26 @@ cudaError_t launch_end_cycle(const EndArgs& a, cudaStream_t s) {
 }
 
 // --------------------------------------------------------------------- utilities
+// Rebinds the stimulus source and the output sink from kernel parameters (no host memory
+// whose lifetime the asynchronous copy would depend on): gs_sim_run_streamed's chunks.
+__global__ void k_set_binding(Ctl* ctl, unsigned long long stim_ptr, unsigned long long stim_base,
+                              unsigned int stim_mode, unsigned long long sink_ptr, unsigned long long sink_base,
+                              unsigned long long sink_cycles) {
+    ctl->stim_ptr = stim_ptr;
+    ctl->stim_base = stim_base;
+    ctl->stim_mode = stim_mode;
+    ctl->sink_ptr = sink_ptr;
+    ctl->sink_base = sink_base;
+    ctl->sink_cycles = sink_cycles;
+}
+
+cudaError_t launch_set_binding(Ctl* ctl, unsigned long long stim_ptr, unsigned long long stim_base,
+                               unsigned int stim_mode, unsigned long long sink_ptr, unsigned long long sink_base,
+                               unsigned long long sink_cycles, cudaStream_t s) {
+    k_set_binding<<<1, 1, 0, s>>>(ctl, stim_ptr, stim_base, stim_mode, sink_ptr, sink_base, sink_cycles);
+    return cudaGetLastError();
+}
+
 __global__ void k_fill_rows(uint8_t* state, uint64_t stride, uint32_t words, uint32_t row0, uint32_t nrows,
                             const uint8_t* init, int value) {
     const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;

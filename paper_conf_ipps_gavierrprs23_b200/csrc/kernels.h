@@ -20,6 +20,9 @@ struct Ctl {
     unsigned long long sig_sum;      // scratch for gs_sim_read_signature
     unsigned int stim_mode;          // 0 generated, 1 bound buffer
     unsigned int done;               // last-block counter of the end-of-cycle kernel
+    unsigned long long sink_ptr;     // 0, or device [cycle - sink_base][po][word] every output
+    unsigned long long sink_base;    //   of every cycle is written to (gs_sim_run_streamed)
+    unsigned long long sink_cycles;  //   capacity in cycles
 };
 
 struct LevelArgs {
@@ -126,6 +129,9 @@ cudaError_t launch_level_poly(const LevelArgs& a, int check_only, cudaStream_t s
 cudaError_t launch_stim(Ctl* ctl, uint8_t* state, uint64_t stride, uint32_t words, uint32_t row_pi0,
                         uint32_t n_pi, uint64_t word_off, uint32_t pdl, cudaStream_t s);
 cudaError_t launch_end_cycle(const EndArgs& a, cudaStream_t s);
+cudaError_t launch_set_binding(Ctl* ctl, unsigned long long stim_ptr, unsigned long long stim_base,
+                               unsigned int stim_mode, unsigned long long sink_ptr, unsigned long long sink_base,
+                               unsigned long long sink_cycles, cudaStream_t s);
 cudaError_t launch_fill_rows(uint8_t* state, uint64_t stride, uint32_t words, uint32_t row0, uint32_t nrows,
                              const uint8_t* init, int value, cudaStream_t s);
 cudaError_t launch_gather_rows(const uint8_t* state, uint64_t stride, uint32_t words, const uint32_t* rows,

@@ -192,6 +192,11 @@ struct gs_sim {
     uint32_t bind_mode = 0;
     void* host_stage = nullptr;       // library-owned device copy of host stimulus
     size_t host_stage_bytes = 0;
+    // gs_sim_run_streamed: library-owned double-buffered device staging + a copy stream
+    void* stream_buf = nullptr;
+    size_t stream_buf_bytes = 0;
+    cudaStream_t copy = nullptr;
+    cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
     cudaGraphExec_t exec[2] = {nullptr, nullptr};
     DfPlan df;
     uint32_t df_grid = 0;
@@ -556,6 +561,11 @@ gs_status gs_sim_destroy(gs_sim* s) {
         if (x) cudaGraphExecDestroy(x);
     if (s->cap) cudaStreamDestroy(s->cap);
     if (s->host_stage) cudaFree(s->host_stage);
+    if (s->copy) cudaStreamSynchronize(s->copy);
+    if (s->stream_buf) cudaFree(s->stream_buf);
+    for (auto& e : s->ev)
+        if (e) cudaEventDestroy(e);
+    if (s->copy) cudaStreamDestroy(s->copy);
     delete s;
     return GS_OK;
 }
@@ -654,6 +664,83 @@ gs_status gs_sim_step(gs_sim* s, uint32_t n) {
         }
         s->cycle++;
     }
+    clear_error();
+    return GS_OK;
+}
+
+gs_status gs_sim_run_streamed(gs_sim* s, const uint64_t* host_stim, uint64_t* host_out, uint32_t ncycles,
+                              uint32_t chunk) {
+    if (gs_status st = check_sim(s, "gs_sim_run_streamed")) return st;
+    if (!host_stim && ncycles) return fail(GS_ERR_ARG, "gs_sim_run_streamed: NULL host_stim");
+    if (!ncycles) return GS_OK;
+    const Program& p = *s->prog;
+    if (!chunk) chunk = 25;
+    chunk = std::min(chunk, ncycles);
+    const size_t w = s->words;
+    const size_t in_b = (size_t)chunk * p.n_pi * w * 8, out_b = host_out ? (size_t)chunk * p.n_po * w * 8 : 0;
+    const size_t in_b2 = (in_b + 255) & ~(size_t)255, out_b2 = (out_b + 255) & ~(size_t)255;
+    CU(cudaSetDevice(s->opts.device));
+    if (2 * (in_b2 + out_b2) > s->stream_buf_bytes) {
+        CU(cudaStreamSynchronize(s->stream));
+        if (s->copy) CU(cudaStreamSynchronize(s->copy));
+        if (s->stream_buf) cudaFree(s->stream_buf);
+        s->stream_buf = nullptr;
+        s->stream_buf_bytes = 0;
+        CU(cudaMalloc(&s->stream_buf, 2 * (in_b2 + out_b2)));
+        s->stream_buf_bytes = 2 * (in_b2 + out_b2);
+    }
+    if (!s->copy) {
+        CU(cudaStreamCreateWithFlags(&s->copy, cudaStreamNonBlocking));
+        for (auto& e : s->ev) CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    }
+    uint8_t* buf = static_cast<uint8_t*>(s->stream_buf);
+    auto in_slot = [&](uint32_t i) { return buf + (i & 1) * in_b2; };
+    auto out_slot = [&](uint32_t i) { return buf + 2 * in_b2 + (i & 1) * out_b2; };
+    cudaEvent_t* ev_in = s->ev;          // H2D of the slot's stimuli done
+    cudaEvent_t* ev_comp = s->ev + 2;    // compute that read / wrote the slot done
+    cudaEvent_t* ev_out = s->ev + 4;     // D2H of the slot's outputs done
+    const uint32_t nch = (ncycles + chunk - 1) / chunk;
+    const uint64_t c_start = s->cycle;
+    // the copy stream may not start before everything already queued on the sim's stream
+    CU(cudaEventRecord(ev_comp[0], s->stream));
+    CU(cudaEventRecord(ev_comp[1], s->stream));
+    CU(cudaEventRecord(ev_out[0], s->stream));
+    CU(cudaEventRecord(ev_out[1], s->stream));
+    auto h2d = [&](uint32_t i) -> gs_status {
+        const uint32_t cc = std::min<uint32_t>(chunk, ncycles - i * chunk);
+        CU(cudaStreamWaitEvent(s->copy, ev_comp[i & 1], 0));          // slot no longer read
+        CU(cudaMemcpyAsync(in_slot(i), host_stim + (size_t)i * chunk * p.n_pi * w, (size_t)cc * p.n_pi * w * 8,
+                           cudaMemcpyHostToDevice, s->copy));
+        CU(cudaEventRecord(ev_in[i & 1], s->copy));
+        return GS_OK;
+    };
+    if (gs_status st = h2d(0)) return st;
+    for (uint32_t i = 0; i < nch; ++i) {
+        const uint32_t cc = std::min<uint32_t>(chunk, ncycles - i * chunk);
+        const uint64_t c0 = c_start + (uint64_t)i * chunk;
+        if (i + 1 < nch)
+            if (gs_status st = h2d(i + 1)) return st;                  // overlaps chunk i's compute
+        CU(cudaStreamWaitEvent(s->stream, ev_in[i & 1], 0));
+        CU(cudaStreamWaitEvent(s->stream, ev_out[i & 1], 0));          // output slot drained
+        CU(launch_set_binding(s->ctl(), reinterpret_cast<uint64_t>(in_slot(i)), c0, 1u,
+                              host_out ? reinterpret_cast<uint64_t>(out_slot(i)) : 0ull, c0, cc, s->stream));
+        s->bound = 2;
+        s->bound_ptr = reinterpret_cast<uint64_t>(in_slot(i));
+        s->bound_base = c0;
+        s->bound_cycles = cc;
+        if (gs_status st = gs_sim_step(s, cc)) return st;
+        CU(cudaEventRecord(ev_comp[i & 1], s->stream));
+        if (host_out) {
+            CU(cudaStreamWaitEvent(s->copy, ev_comp[i & 1], 0));
+            CU(cudaMemcpyAsync(host_out + (size_t)i * chunk * p.n_po * w, out_slot(i), (size_t)cc * p.n_po * w * 8,
+                               cudaMemcpyDeviceToHost, s->copy));
+            CU(cudaEventRecord(ev_out[i & 1], s->copy));
+        }
+    }
+    // detach the sink; the sim's stream completes only after the last output copy
+    CU(launch_set_binding(s->ctl(), s->bound_ptr, s->bound_base, 1u, 0ull, 0ull, 0ull, s->stream));
+    CU(cudaEventRecord(ev_in[0], s->copy));
+    CU(cudaStreamWaitEvent(s->stream, ev_in[0], 0));
     clear_error();
     return GS_OK;
 }
