@@ -52,6 +52,7 @@ def parse():
     ap.add_argument("--lane-slabs", type=int, default=0, help="L2 lane slabs (0 = library default)")
     ap.add_argument("--lut-unroll", type=int, default=0, help="vectors per thread (0 = auto)")
     ap.add_argument("--no-pdl", action="store_true", help="disable programmatic dependent launch")
+    ap.add_argument("--no-grid-stride", action="store_true", help="kernel A: one CTA per work chunk")
     ap.add_argument("--l2-hints", type=int, default=0, help="kernel A L2 hints: 0 off, 1 stores, 2 +loads")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
@@ -244,7 +245,8 @@ def main():
                  lane_slabs=args.lane_slabs, lut_unroll=args.lut_unroll,
                  df_interleave=args.df_interleave, df_gates_per_warp=args.df_gpw, pdl=not args.no_pdl,
                  tile_words=args.tile_words, tile_groups=args.tile_groups,
-                 flags=(2 if args.l2_hints >= 1 else 0) | (4 if args.l2_hints >= 2 else 0))
+                 flags=(2 if args.l2_hints >= 1 else 0) | (4 if args.l2_hints >= 2 else 0) |
+                 (8 if args.no_grid_stride else 0))
     sim.bind_generated(cfg.stim_seed)
     C = args.cycles_per_step
     launches_per_cycle = sim.launches_per_cycle()
@@ -348,6 +350,7 @@ def main():
                        "df_interleave": args.df_interleave, "df_gpw": args.df_gpw,
                        "pdl": not args.no_pdl, "tile_words": args.tile_words,
                        "tile_groups": args.tile_groups, "l2_hints": args.l2_hints, "lut_k": args.lut_k,
+                       "grid_stride": not args.no_grid_stride,
                        "l2": "inputs larger than L2 (state %.1f GB per GPU)" % (info["n_rows"] * lanes / 8 / 1e9),
                        "parallelism": f"dp{world} (stimulus sharding)" + (" TEST: all ranks on cuda:0"
                                                                               if args.same_device else ""),

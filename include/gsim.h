@@ -250,6 +250,9 @@ typedef struct {
 #define GS_SIM_L2_HINTS 2u
 /* flags: with GS_SIM_L2_HINTS, also load gate inputs with L2 evict_first. */
 #define GS_SIM_L2_HINT_LOADS 4u
+/* flags: kernel A launches one CTA per work chunk instead of a grid-stride grid sized to
+ * the resident capacity (A/B measurement only). */
+#define GS_SIM_NO_GRID_STRIDE 8u
 
 /* Device workspace bytes required for (prog, opts). */
 gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts, size_t* bytes);

@@ -44,6 +44,7 @@ struct LevelArgs {
     uint32_t min_warps;               // auto U: prefer smaller U below this many warps
     uint32_t hint;                    // L2 eviction-priority stores (aux.k bit 8 = read next level)
     uint32_t hint_ld;                 // ... and evict_first input loads
+    uint32_t grid_blocks;             // wide path: cap the grid at the resident capacity (0 = off)
 };
 
 struct EndArgs {
@@ -123,6 +124,7 @@ cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_ev
 cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s);
 
 cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s);
+uint32_t level_lut_resident_blocks(int device);   // CTAs of k_level_lut_wide resident on the GPU
 cudaError_t launch_dataflow(const DfArgs& a, uint32_t grid, cudaStream_t s);
 cudaError_t dataflow_grid(uint32_t slab_vec, int device, uint32_t* grid);
 cudaError_t launch_level_poly(const LevelArgs& a, int check_only, cudaStream_t s);

@@ -206,6 +206,8 @@ struct gs_sim {
     uint32_t tile_groups = 1;
     uint32_t pdl = 1;                 // programmatic dependent launch between cycle kernels
     uint32_t min_warps = 0;           // kernel A auto-U threshold (2 waves of resident warps)
+    uint32_t resident_blocks = 0;     // kernel A wide path: CTAs resident on the GPU
+    uint32_t grid_waves = 1;          // grid-stride grid = resident_blocks x this
 
     Ctl* ctl() const { return reinterpret_cast<Ctl*>(ws + L.ctl); }
     uint8_t* state() const { return ws + L.state; }
@@ -240,6 +242,7 @@ static LevelArgs level_args(const gs_sim* s, uint32_t l, uint32_t parity) {
     a.min_warps = s->min_warps;
     a.hint = (s->opts.flags & GS_SIM_L2_HINTS) ? 1u : 0u;
     a.hint_ld = (s->opts.flags & GS_SIM_L2_HINT_LOADS) ? 1u : 0u;
+    a.grid_blocks = (s->opts.flags & GS_SIM_NO_GRID_STRIDE) ? 0u : s->resident_blocks * s->grid_waves;
     return a;
 }
 
@@ -468,6 +471,7 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
         int sms = 148;
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, opts->device);
         s->min_warps = (uint32_t)sms * 32u * 2u;   // 4 CTAs x 8 warps per SM, two waves
+        s->resident_blocks = level_lut_resident_blocks(opts->device);
     }
     s->slabs = (opts->lane_slabs && s->opts.kernel != GS_KERNEL_DATAFLOW) ? opts->lane_slabs : 1;
     if (s->slabs > 1) {

@@ -283,7 +283,7 @@ def test_errors_on_device():
     sim.close()
 
 
-@pytest.mark.parametrize("flags", [gs.GS_SIM_NO_PDL, 2, 6])
+@pytest.mark.parametrize("flags", [gs.GS_SIM_NO_PDL, 2, 6, 8])
 def test_launch_and_cache_options_do_not_change_results(flags):
     """PDL off, L2 eviction hints on stores, hints on stores and loads: bit-identical."""
     cfg = workloads.CONFIGS["C3"]
