@@ -200,8 +200,9 @@ gs_status gs_program_tile_slots(const gs_program* prog, uint32_t* slots);
 
 /* ======================================================================= simulate */
 enum {
-    GS_KERNEL_AUTO = 0,   /* GS_KERNEL_TILE when one tile's live state and every gate
-                             descriptor fit shared memory, else GS_KERNEL_LUT             */
+    GS_KERNEL_AUTO = 0,   /* GS_KERNEL_POLY if some LUT has k > 6; else GS_KERNEL_TILE when
+                             one tile's live state fits shared memory next to the gate
+                             descriptors (resident or TMA-streamed); else GS_KERNEL_LUT   */
     GS_KERNEL_LUT = 1,    /* kernel A: bit-sliced LUT evaluation, 64 stimuli per word      */
     GS_KERNEL_POLY = 2,   /* kernel B: the paper's network, sum_S w_S Theta(sum x - |S| + 1)
                              per stimulus in int32, ballot-packed (Eq. 1-3)                */
@@ -253,6 +254,11 @@ typedef struct {
 /* flags: kernel A launches one CTA per work chunk instead of a grid-stride grid sized to
  * the resident capacity (A/B measurement only). */
 #define GS_SIM_NO_GRID_STRIDE 8u
+/* flags (kernel T): force the descriptor source — global memory (L2), or a TMA bulk-copy
+ * stream of one level at a time into a shared-memory double buffer.  Default: resident in
+ * shared memory if the whole table fits, else the TMA stream, else global. */
+#define GS_SIM_TILE_DESC_GLOBAL 16u
+#define GS_SIM_TILE_DESC_TMA 32u
 
 /* Device workspace bytes required for (prog, opts). */
 gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts, size_t* bytes);

@@ -158,7 +158,7 @@ __device__ __forceinline__ void lut_gate_u(const LevelArgs& a, uint32_t gate, ui
 // resident capacity (148 SMs x CTAs per SM, a.grid_blocks), so no level ends with a
 // partially filled wave of CTAs.
 template <int U, bool HINT>
-__global__ void __launch_bounds__(256, 4) k_level_lut_wide(LevelArgs a, uint32_t cpg_shift, uint32_t vec0) {
+__global__ void __launch_bounds__(256, U > 4 ? 2 : 4) k_level_lut_wide(LevelArgs a, uint32_t cpg_shift, uint32_t vec0) {
     pdl_entry();
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t total = a.ng << cpg_shift;
@@ -182,11 +182,15 @@ __global__ void __launch_bounds__(256, 4) k_level_lut_wide(LevelArgs a, uint32_t
                     if (U > 1) lut_gate_u<5, 1, HINT>(a, gate, in, v0 + 32, tt, qdst, hot);
                     if (U > 2) { lut_gate_u<5, 1, HINT>(a, gate, in, v0 + 64, tt, qdst, hot);
                                  lut_gate_u<5, 1, HINT>(a, gate, in, v0 + 96, tt, qdst, hot); }
+                    if (U > 4)
+                        for (int u = 4; u < U; ++u) lut_gate_u<5, 1, HINT>(a, gate, in, v0 + 32 * u, tt, qdst, hot);
                     break;
             default: lut_gate_u<6, 1, HINT>(a, gate, in, v0, tt, qdst, hot);
                     if (U > 1) lut_gate_u<6, 1, HINT>(a, gate, in, v0 + 32, tt, qdst, hot);
                     if (U > 2) { lut_gate_u<6, 1, HINT>(a, gate, in, v0 + 64, tt, qdst, hot);
                                  lut_gate_u<6, 1, HINT>(a, gate, in, v0 + 96, tt, qdst, hot); }
+                    if (U > 4)
+                        for (int u = 4; u < U; ++u) lut_gate_u<6, 1, HINT>(a, gate, in, v0 + 32 * u, tt, qdst, hot);
                     break;
         }
     }
@@ -205,7 +209,8 @@ cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s) {
     // slab: 16-byte vectors [a.vec0, a.vec0 + a.vslab) of every row (whole row if vslab == 0)
     if ((a.words % 2) == 0) {
         const uint32_t vrow = a.vslab ? a.vslab : a.words / 2;
-        for (uint32_t U : {4u, 2u, 1u}) {
+        for (uint32_t U : {8u, 4u, 2u, 1u}) {
+            if (U == 8 && a.unroll != 8) continue;              // U = 8 only on request
             if (a.unroll && U > a.unroll) continue;
             const uint32_t cpg = vrow / (32 * U);
             if (vrow % (32 * U) || cpg == 0 || (cpg & (cpg - 1))) continue;
@@ -221,6 +226,7 @@ cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s) {
             // partial last wave would idle SMs for a large share of the launch; measured: C3
             // +8.5 %); deep levels (C4: 12 waves, C5: 41) keep one CTA per chunk (-1 % otherwise)
             if (a.grid_blocks && blocks > a.grid_blocks && blocks <= 4 * a.grid_blocks) blocks = a.grid_blocks;
+            if (U == 8) return launch_k(k_level_lut_wide<8, false>, blocks, s, a.pdl, a, sh, a.vec0);
             if (a.hint) {
                 if (U == 4) return launch_k(k_level_lut_wide<4, true>, blocks, s, a.pdl, a, sh, a.vec0);
                 if (U == 2) return launch_k(k_level_lut_wide<2, true>, blocks, s, a.pdl, a, sh, a.vec0);

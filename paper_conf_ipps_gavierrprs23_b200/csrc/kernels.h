@@ -96,7 +96,9 @@ struct TileArgs {
     const uint4* desc_hi;             // [n_eval] (k > 4 only)
     const uint32_t* level_off;        // [n_levels + 1]
     uint32_t n_eval, n_levels;
-    uint32_t desc_smem;               // 1: copy desc + level_off into shared memory once
+    uint32_t desc_smem;               // 0: descriptors read from global; 1: resident in shared
+                                      // memory; 2: TMA-streamed level by level (double buffer)
+    uint32_t max_width;               // widest level (mode 2 buffer size, in descriptors)
     const uint32_t* po_slot;
     uint32_t n_po;
     const uint32_t* latch_src;
@@ -118,9 +120,9 @@ struct TileArgs {
     uint32_t ncycles, n_tiles;
 };
 size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
-                       int desc_smem);
+                       int desc_mode, uint32_t max_width);
 cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
-                       int desc_smem, uint32_t has_q, uint32_t* per_sm);
+                       int desc_smem, uint32_t max_width, uint32_t has_q, uint32_t* per_sm);
 cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s);
 
 cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s);

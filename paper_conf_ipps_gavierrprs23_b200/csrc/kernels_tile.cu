@@ -23,12 +23,49 @@ namespace gs {
 constexpr uint32_t TILE_CTA = 512;                   // threads per CTA (one CTA per SM)
 constexpr unsigned long long TILE_MISR_POLY = 0x42F0E1EBA9EA3693ULL;   // CRC-64/ECMA-182
 
-// Shared memory: [desc: 16 B x n_eval (if desc_smem)] [level_off: 4 B x (n_levels + 1),
-// padded to 16 B] then per thread group: [slots: n_slots x TW words] [MISR: 64 x TW words].
+// Shared memory by descriptor mode:
+//   1 (resident): [desc: 16 B x n_eval] [level_off: 4 B x (n_levels + 1), padded to 16 B]
+//   2 (TMA-streamed): [level_off] then per group [2 mbarriers, 16 B][2 x max_width x 16 B]
+//   0 (global): nothing
+// then per thread group: [slots: n_slots x TW words] [MISR: 64 x TW words].
+static size_t lvl_bytes(uint32_t n_levels) { return (((size_t)n_levels + 1) * 4 + 15) / 16 * 16; }
+
 size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
-                       int desc_smem) {
-    size_t b = desc_smem ? (size_t)n_eval * 16 + (((size_t)n_levels + 1) * 4 + 15) / 16 * 16 : 0;
-    return b + (size_t)ng * ((size_t)n_slots + 64) * 4 * tw;
+                       int desc_mode, uint32_t max_width) {
+    size_t b = 0, g = ((size_t)n_slots + 64) * 4 * tw;
+    if (desc_mode == 1) b = (size_t)n_eval * 16 + lvl_bytes(n_levels);
+    if (desc_mode == 2) {
+        b = lvl_bytes(n_levels);
+        g += 16 + 2 * (size_t)max_width * 16;
+    }
+    return b + (size_t)ng * g;
+}
+
+// ---- TMA bulk copy (cp.async.bulk) of a level's descriptors into shared memory, completion
+// signalled on an mbarrier (expect_tx / complete_tx), consumers wait on the phase parity
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // prior generic reads of dst
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    uint32_t done = 0;
+    while (!done) {
+        asm volatile(
+            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+            : "=r"(done)
+            : "r"(smem_u32(bar)), "r"(parity)
+            : "memory");
+    }
 }
 
 // One gate on one 16-byte group (4 words = 128 lanes) of its slots.  HASQ: the circuit has
@@ -75,21 +112,35 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     constexpr uint32_t V = TW / 4;                       // uint4 per slot
     constexpr uint32_t GT = TILE_CTA / NG;               // threads per group
     extern __shared__ uint4 smem[];
-    const uint4* dsm = a.desc_smem ? smem : reinterpret_cast<const uint4*>(a.desc);
+    const uint4* dsm = a.desc_smem == 1 ? smem : reinterpret_cast<const uint4*>(a.desc);
     const uint32_t* lvl = a.level_off;
     uint4* base = smem;
-    if (a.desc_smem) {
+    if (a.desc_smem == 1) {
         uint32_t* lv = reinterpret_cast<uint32_t*>(smem + a.n_eval);
         const uint4* gd = reinterpret_cast<const uint4*>(a.desc);
         for (uint32_t i = threadIdx.x; i < a.n_eval; i += blockDim.x) smem[i] = __ldg(gd + i);
         for (uint32_t i = threadIdx.x; i <= a.n_levels; i += blockDim.x) lv[i] = __ldg(a.level_off + i);
         lvl = lv;
         base = smem + a.n_eval + ((a.n_levels + 1) * 4 + 15) / 16;
+    } else if (a.desc_smem == 2) {
+        uint32_t* lv = reinterpret_cast<uint32_t*>(smem);
+        for (uint32_t i = threadIdx.x; i <= a.n_levels; i += blockDim.x) lv[i] = __ldg(a.level_off + i);
+        lvl = lv;
+        base = smem + ((a.n_levels + 1) * 4 + 15) / 16;
     }
-    __syncthreads();
     const uint32_t gid = threadIdx.x / GT, tid = threadIdx.x % GT, bd = GT;
     const uint32_t bar = 1 + gid;
-    uint4* sl = base + (size_t)gid * (a.n_slots + 64) * V;   // this group's slots
+    // group region: [mbarriers + descriptor double buffer (mode 2)] [slots] [MISR]
+    uint4* greg = base + (size_t)gid * ((a.n_slots + 64) * V + (a.desc_smem == 2 ? 1 + 2 * a.max_width : 0));
+    uint64_t* mbar = reinterpret_cast<uint64_t*>(greg);
+    uint4* dbuf = greg + 1;                                   // [2][max_width]
+    uint4* sl = a.desc_smem == 2 ? greg + 1 + 2 * a.max_width : greg;   // this group's slots
+    if (a.desc_smem == 2 && tid == 0) {
+        mbar_init(mbar, 1);
+        mbar_init(mbar + 1, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
     uint32_t* sw = reinterpret_cast<uint32_t*>(sl);          // slots as 32-bit words
     uint32_t* mp = sw + (size_t)a.n_slots * TW;               // MISR planes [64][TW]
     const unsigned long long c0 = a.ctl->cycle;
@@ -102,8 +153,15 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     const uint32_t* misr_in = reinterpret_cast<const uint32_t*>(a.misr + (size_t)(c0 & 1) * 64 * a.words);
     uint32_t* misr_out = reinterpret_cast<uint32_t*>(a.misr + (size_t)((c0 + a.ncycles) & 1) * 64 * a.words);
     unsigned long long pop = 0;
+    // mode 2: the group's descriptor stream, one level per step, double-buffered: while
+    // level l is evaluated from buffer (step & 1), the TMA engine fetches the next level
+    // (the same sequence repeats every cycle and every tile)
+    uint32_t step = 0;
+    if (a.desc_smem == 2 && tid == 0 && blockIdx.x * NG + gid < a.n_tiles)
+        tma_load_1d(dbuf, a.desc + lvl[0], (lvl[1] - lvl[0]) * 16, mbar);
 
     for (uint32_t tile = blockIdx.x * NG + gid; tile < a.n_tiles; tile += gridDim.x * NG) {
+        const bool last_tile = tile + gridDim.x * NG >= a.n_tiles;
         const uint32_t t0 = tile * TW;                    // first 32-bit word of the tile (shard-local)
         // ---- load: constants, both register banks, MISR planes
         for (uint32_t u = tid; u < TW; u += bd) {
@@ -139,10 +197,22 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
             // ---- levels: every (gate, 16-byte group) unit of the level, then a barrier
             for (uint32_t l = 0; l < a.n_levels; ++l) {
                 const uint32_t g0 = lvl[l], n = (lvl[l + 1] - g0) * V;
+                const uint4* dl = dsm + g0;
+                if (a.desc_smem == 2) {
+                    const uint32_t b = step & 1;
+                    if (tid == 0 && !(last_tile && c + 1 == a.ncycles && l + 1 == a.n_levels)) {
+                        const uint32_t ln = l + 1 == a.n_levels ? 0 : l + 1;
+                        tma_load_1d(dbuf + (b ^ 1) * a.max_width, a.desc + lvl[ln], (lvl[ln + 1] - lvl[ln]) * 16,
+                                    mbar + (b ^ 1));
+                    }
+                    mbar_wait(mbar + b, (step >> 1) & 1);
+                    dl = dbuf + b * a.max_width;
+                    ++step;
+                }
                 for (uint32_t u = tid; u < n; u += bd) {
                     const uint32_t gi = u / V, v = u % V;
                     const uint32_t g = g0 + gi;
-                    const uint4 d = dsm[g];
+                    const uint4 d = dl[gi];
                     switch (d.w & 15u) {                       // k: warp-uniform except at k-group edges
                         case 1: tile_gate<1, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
                         case 2: tile_gate<2, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
@@ -241,8 +311,8 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     }
 
 cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
-                       int desc_smem, uint32_t has_q, uint32_t* per_sm) {
-    const size_t smem = tile_smem_bytes(tw, ng, n_slots, n_eval, n_levels, desc_smem);
+                       int desc_smem, uint32_t max_width, uint32_t has_q, uint32_t* per_sm) {
+    const size_t smem = tile_smem_bytes(tw, ng, n_slots, n_eval, n_levels, desc_smem, max_width);
     cudaError_t e = cudaSuccess;
     int per = 0;
 #define TILE_PREP(T, Q, G)                                                                                        \
@@ -256,7 +326,7 @@ cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_ev
 
 cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s) {
     if (a.n_tiles == 0 || a.ncycles == 0) return cudaSuccess;
-    const size_t smem = tile_smem_bytes(tw, ng, a.n_slots, a.n_eval, a.n_levels, a.desc_smem);
+    const size_t smem = tile_smem_bytes(tw, ng, a.n_slots, a.n_eval, a.n_levels, a.desc_smem, a.max_width);
 #define TILE_LAUNCH(T, Q, G) k_tile<T, Q, G><<<grid, TILE_CTA, smem, s>>>(a)
     TILE_SWITCH(tw, a.n_reg > 0, ng, TILE_LAUNCH)
 #undef TILE_LAUNCH

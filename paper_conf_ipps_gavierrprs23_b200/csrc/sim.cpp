@@ -69,7 +69,8 @@ struct Plans {
     TilePlan tile;
     uint32_t tw = 0;                  // kernel T: 32-bit words per slot
     uint32_t ng = 0;                  // kernel T: thread groups (tiles) per CTA
-    int desc_smem = 0;                // kernel T: descriptors resident in shared memory
+    int desc_smem = 0;                // kernel T: descriptors 0 global, 1 resident, 2 TMA-streamed
+    uint32_t max_width = 0;           // kernel T: widest level
 };
 
 constexpr size_t TILE_SMEM_MAX = 232448;   // 227 KB opt-in shared memory per CTA (sm_100a)
@@ -78,8 +79,16 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
     if (gs_status st = df_plan(p, o, pl.df)) return st;
     if (o.kernel != GS_KERNEL_TILE) return GS_OK;
     if (gs_status st = tile_plan(p, pl.tile)) return st;
+    uint32_t maxw = 0;
+    bool empty_level = false;
+    for (uint32_t l = 0; l < p.n_levels; ++l) {
+        maxw = std::max(maxw, p.level_off[l + 1] - p.level_off[l]);
+        empty_level = empty_level || p.level_off[l + 1] == p.level_off[l];
+    }
+    pl.max_width = maxw;
     auto smem = [&](uint32_t tw, uint32_t ng, int ds) {
-        return tile_smem_bytes(tw, ng, pl.tile.n_slots, p.n_eval, p.n_levels, ds);
+        if (ds == 2 && empty_level) return (size_t)-1;             // TMA stream needs non-empty levels
+        return tile_smem_bytes(tw, ng, pl.tile.n_slots, p.n_eval, p.n_levels, ds, maxw);
     };
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, o.device);
@@ -89,30 +98,35 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
         return fail(GS_ERR_ARG, "TILE: tile_groups must be 1, 2 or 4");
     if (o.tile_words && o.lanes % (32ull * o.tile_words))
         return fail(GS_ERR_ARG, "TILE: lanes must be a multiple of 32 * tile_words");
-    // choose (tile words, groups per CTA): descriptors resident if possible, then the most
-    // lanes in flight on the GPU (groups x tile lanes x SMs, capped by the batch), then
-    // fewer groups and wider tiles (measured best on C2: one group of 32 words)
+    // choose (descriptor mode, tile words, groups per CTA): the most lanes in flight on the
+    // GPU (groups x tile lanes x SMs, capped by the batch) first — measured: a 10k-gate
+    // circuit runs 1.33x faster with TMA-streamed descriptors and 4x wider tiles than with a
+    // resident table and narrow tiles — then resident > TMA stream > global descriptors,
+    // then fewer groups and wider tiles (measured best on C2: one group of 32 words)
+    const int forced = (o.flags & GS_SIM_TILE_DESC_GLOBAL) ? 0 : (o.flags & GS_SIM_TILE_DESC_TMA) ? 2 : -1;
     uint64_t best = 0;
-    for (int ds : {1, 0}) {
+    for (int ds : {1, 2, 0}) {
+        if (forced >= 0 && ds != forced) continue;
         for (uint32_t ng : {4u, 2u, 1u}) {
             if (o.tile_groups && ng != o.tile_groups) continue;
             for (uint32_t tw : {4u, 8u, 16u, 32u}) {
                 if (o.tile_words && tw != o.tile_words) continue;
                 if (o.lanes % (32ull * tw) || smem(tw, ng, ds) > TILE_SMEM_MAX) continue;
                 const uint64_t inflight = std::min<uint64_t>((uint64_t)ng * tw * 32 * sms, o.lanes);
-                const uint64_t score = (inflight << 8) | ((8 - ng) << 4) | tw;
-                if (score > best) { best = score; pl.tw = tw; pl.ng = ng; }
+                const uint64_t pref = ds == 1 ? 2 : ds == 2 ? 1 : 0;
+                const uint64_t score = (inflight << 16) | (pref << 12) | ((8 - ng) << 8) | tw;
+                if (score > best) { best = score; pl.tw = tw; pl.ng = ng; pl.desc_smem = ds; }
             }
         }
-        if (best) { pl.desc_smem = ds; break; }
     }
     if (!best) return fail(GS_ERR_ARG, "TILE: live state of a 128-lane tile exceeds shared memory (or lanes % 128)");
     return GS_OK;
 }
 
-// GS_KERNEL_AUTO: kernel T when one tile's live state AND the whole descriptor table fit
-// shared memory (small, deep circuits: measured 1.8x kernel A on C2, 5.8x on C1), else
-// kernel A (large circuits are HBM-bound; kernel T cannot hold them).
+// GS_KERNEL_AUTO: kernel T when one tile's live state fits shared memory next to either the
+// whole descriptor table or the TMA descriptor double buffer (small and mid-size circuits:
+// measured 1.8x kernel A on C2, 5.8x on C1, 2.6x / 1.4x / 1.1x on 5k / 10k / 20k-gate
+// synthetic circuits), else kernel A (large circuits are HBM-bound; T cannot hold them).
 gs_sim_opts resolve_auto(const Program& p, const gs_sim_opts& o) {
     gs_sim_opts r = o;
     if (o.kernel != GS_KERNEL_AUTO) return r;
@@ -123,7 +137,7 @@ gs_sim_opts resolve_auto(const Program& p, const gs_sim_opts& o) {
     r.kernel = GS_KERNEL_TILE;
     Plans pl;
     const std::string saved = gs_last_error();
-    if (p.n_eval == 0 || make_plans(p, r, pl) != GS_OK || !pl.desc_smem) r.kernel = GS_KERNEL_LUT;
+    if (p.n_eval == 0 || make_plans(p, r, pl) != GS_OK || pl.desc_smem == 0) r.kernel = GS_KERNEL_LUT;
     set_error(saved);
     return r;
 }
@@ -204,6 +218,7 @@ struct gs_sim {
     uint32_t tw = 0, tile_grid = 0;
     int desc_smem = 0;
     uint32_t tile_groups = 1;
+    uint32_t tile_max_width = 0;
     uint32_t pdl = 1;                 // programmatic dependent launch between cycle kernels
     uint32_t min_warps = 0;           // kernel A auto-U threshold (2 waves of resident warps)
     uint32_t resident_blocks = 0;     // kernel A wide path: CTAs resident on the GPU
@@ -329,6 +344,7 @@ static cudaError_t tile_launch(const gs_sim* s, uint32_t ncycles, cudaStream_t s
     a.n_eval = p.n_eval;
     a.n_levels = p.n_levels;
     a.desc_smem = (uint32_t)s->desc_smem;
+    a.max_width = s->tile_max_width;
     a.po_slot = s->at<const uint32_t>(s->L.t_po);
     a.n_po = p.n_po;
     a.latch_src = s->at<const uint32_t>(s->L.t_lsrc);
@@ -466,6 +482,7 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
     s->tile = pls.tile;
     s->tw = pls.tw;
     s->desc_smem = pls.desc_smem;
+    s->tile_max_width = pls.max_width;
     s->pdl = (opts->flags & GS_SIM_NO_PDL) ? 0u : 1u;
     {
         int sms = 148;
@@ -500,8 +517,8 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
         uint32_t per = 0;
         int sms = 148;
         s->tile_groups = pls.ng;
-        e = tile_setup(s->tw, s->tile_groups, s->tile.n_slots, p.n_eval, p.n_levels, s->desc_smem, p.n_reg > 0,
-                       &per);
+        e = tile_setup(s->tw, s->tile_groups, s->tile.n_slots, p.n_eval, p.n_levels, s->desc_smem,
+                       s->tile_max_width, p.n_reg > 0, &per);
         if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, opts->device);
         if (e != cudaSuccess || per == 0) {
             delete s;

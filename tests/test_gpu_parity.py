@@ -545,6 +545,27 @@ def test_tile_sequential_synthetic_all_lanes_probes_resume(tw, ng):
     sim.close()
 
 
+@pytest.mark.parametrize("flags", [16, 32])
+def test_tile_descriptor_sources_global_and_tma_stream(flags):
+    """Kernel T with descriptors read from global memory (16) or streamed one level at a time
+    by TMA bulk copies into a shared-memory double buffer (32): every lane vs the oracle,
+    steps split over several launches (the TMA stream restarts at each tile and step)."""
+    nl = workloads.synthetic(8000, 300, 32, 48, 24, seed=21, name="t8k")
+    prog = compile_nl(nl)
+    lanes = 4096
+    sim = gs.Sim(prog, lanes, kernel="tile", flags=flags, trace_words=[0, 31, 63], trace_cycles=20)
+    sim.bind_generated(5)
+    for n in (1, 6, 13):
+        sim.step(n)
+    o = oracle.simulate(nl, np.arange(lanes), 20, seed=5)
+    assert np.array_equal(sim.read_lane_signatures(), o["sig"])
+    assert np.array_equal(gs.unpack_lanes(sim.read_registers()).T, o["regs"])
+    assert np.array_equal(gs.unpack_lanes(sim.read_outputs()).T, o["last"])
+    rows = np.concatenate([np.arange(0, 64), np.arange(31 * 64, 32 * 64), np.arange(63 * 64, 64 * 64)])
+    assert np.array_equal(gpu_trace_bits(sim.read_trace(), None), o["trace"][rows])
+    sim.close()
+
+
 def test_auto_kernel_selection():
     """AUTO = kernel T (one launch per step) when the circuit fits shared memory, else A."""
     for name, lanes, tile in (("C1", 1024, True), ("C2", 1 << 14, True), ("C3", 4096, False)):
