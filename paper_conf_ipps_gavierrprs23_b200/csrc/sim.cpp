@@ -99,10 +99,11 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
     if (o.tile_words && o.lanes % (32ull * o.tile_words))
         return fail(GS_ERR_ARG, "TILE: lanes must be a multiple of 32 * tile_words");
     // choose (descriptor mode, tile words, groups per CTA): the most lanes in flight on the
-    // GPU (groups x tile lanes x SMs, capped by the batch) first — measured: a 10k-gate
-    // circuit runs 1.33x faster with TMA-streamed descriptors and 4x wider tiles than with a
-    // resident table and narrow tiles — then resident > TMA stream > global descriptors,
-    // then fewer groups and wider tiles (measured best on C2: one group of 32 words)
+    // GPU (groups x tile lanes x SMs, capped by the batch), counting a resident descriptor
+    // table as worth 2x the lanes (measured: C2 runs 1.08x faster with one group and a
+    // resident table than with two groups and TMA-streamed descriptors, while a 10k-gate
+    // circuit runs 1.33x faster with TMA and 4x wider tiles than resident with narrow
+    // ones), then wider tiles, then resident > TMA stream > global, then fewer groups
     const int forced = (o.flags & GS_SIM_TILE_DESC_GLOBAL) ? 0 : (o.flags & GS_SIM_TILE_DESC_TMA) ? 2 : -1;
     uint64_t best = 0;
     for (int ds : {1, 2, 0}) {
@@ -114,7 +115,8 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
                 if (o.lanes % (32ull * tw) || smem(tw, ng, ds) > TILE_SMEM_MAX) continue;
                 const uint64_t inflight = std::min<uint64_t>((uint64_t)ng * tw * 32 * sms, o.lanes);
                 const uint64_t pref = ds == 1 ? 2 : ds == 2 ? 1 : 0;
-                const uint64_t score = (inflight << 16) | (pref << 12) | ((8 - ng) << 8) | tw;
+                const uint64_t score = ((inflight << (ds == 1 ? 1 : 0)) << 24) | ((uint64_t)tw << 16) | (pref << 12) |
+                                       ((8 - ng) << 8);
                 if (score > best) { best = score; pl.tw = tw; pl.ng = ng; pl.desc_smem = ds; }
             }
         }
