@@ -107,22 +107,22 @@ __device__ __forceinline__ void group_sync(uint32_t id, uint32_t nthreads) {
 // group simulates its own tile and synchronises only with itself (named barrier 1 + gid),
 // so one group's level barrier overlaps the other groups' work.  All groups share the
 // descriptor table in shared memory.
-template <int TW, bool HASQ, int NG>
+template <int TW, bool HASQ, int NG, int DM>
 __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     constexpr uint32_t V = TW / 4;                       // uint4 per slot
     constexpr uint32_t GT = TILE_CTA / NG;               // threads per group
     extern __shared__ uint4 smem[];
-    const uint4* dsm = a.desc_smem == 1 ? smem : reinterpret_cast<const uint4*>(a.desc);
+    const uint4* dsm = DM == 1 ? smem : reinterpret_cast<const uint4*>(a.desc);
     const uint32_t* lvl = a.level_off;
     uint4* base = smem;
-    if (a.desc_smem == 1) {
+    if (DM == 1) {
         uint32_t* lv = reinterpret_cast<uint32_t*>(smem + a.n_eval);
         const uint4* gd = reinterpret_cast<const uint4*>(a.desc);
         for (uint32_t i = threadIdx.x; i < a.n_eval; i += blockDim.x) smem[i] = __ldg(gd + i);
         for (uint32_t i = threadIdx.x; i <= a.n_levels; i += blockDim.x) lv[i] = __ldg(a.level_off + i);
         lvl = lv;
         base = smem + a.n_eval + ((a.n_levels + 1) * 4 + 15) / 16;
-    } else if (a.desc_smem == 2) {
+    } else if (DM == 2) {
         uint32_t* lv = reinterpret_cast<uint32_t*>(smem);
         for (uint32_t i = threadIdx.x; i <= a.n_levels; i += blockDim.x) lv[i] = __ldg(a.level_off + i);
         lvl = lv;
@@ -131,11 +131,11 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     const uint32_t gid = threadIdx.x / GT, tid = threadIdx.x % GT, bd = GT;
     const uint32_t bar = 1 + gid;
     // group region: [mbarriers + descriptor double buffer (mode 2)] [slots] [MISR]
-    uint4* greg = base + (size_t)gid * ((a.n_slots + 64) * V + (a.desc_smem == 2 ? 1 + 2 * a.max_width : 0));
+    uint4* greg = base + (size_t)gid * ((a.n_slots + 64) * V + (DM == 2 ? 1 + 2 * a.max_width : 0));
     uint64_t* mbar = reinterpret_cast<uint64_t*>(greg);
     uint4* dbuf = greg + 1;                                   // [2][max_width]
-    uint4* sl = a.desc_smem == 2 ? greg + 1 + 2 * a.max_width : greg;   // this group's slots
-    if (a.desc_smem == 2 && tid == 0) {
+    uint4* sl = DM == 2 ? greg + 1 + 2 * a.max_width : greg;   // this group's slots
+    if (DM == 2 && tid == 0) {
         mbar_init(mbar, 1);
         mbar_init(mbar + 1, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -157,7 +157,7 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     // level l is evaluated from buffer (step & 1), the TMA engine fetches the next level
     // (the same sequence repeats every cycle and every tile)
     uint32_t step = 0;
-    if (a.desc_smem == 2 && tid == 0 && blockIdx.x * NG + gid < a.n_tiles)
+    if (DM == 2 && tid == 0 && blockIdx.x * NG + gid < a.n_tiles)
         tma_load_1d(dbuf, a.desc + lvl[0], (lvl[1] - lvl[0]) * 16, mbar);
 
     for (uint32_t tile = blockIdx.x * NG + gid; tile < a.n_tiles; tile += gridDim.x * NG) {
@@ -198,7 +198,7 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
             for (uint32_t l = 0; l < a.n_levels; ++l) {
                 const uint32_t g0 = lvl[l], n = (lvl[l + 1] - g0) * V;
                 const uint4* dl = dsm + g0;
-                if (a.desc_smem == 2) {
+                if (DM == 2) {
                     const uint32_t b = step & 1;
                     if (tid == 0 && !(last_tile && c + 1 == a.ncycles && l + 1 == a.n_levels)) {
                         const uint32_t ln = l + 1 == a.n_levels ? 0 : l + 1;
@@ -298,12 +298,20 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     }
 }
 
-// instantiations: TW in {4, 8, 16, 32} x registers present x groups {1, 2, 4}
+// instantiations: TW in {4, 8, 16, 32} x registers present x groups {1, 2, 4} x descriptor
+// source {global, resident, TMA stream} (a compile-time source lets ptxas emit LDS for
+// shared-memory descriptors instead of generic loads)
+#define TILE_CASES_DM(T, Q, G, CALL)                                                                  \
+    switch (dmv) {                                                                                   \
+        case 0: CALL(T, Q, G, 0); break;                                                             \
+        case 1: CALL(T, Q, G, 1); break;                                                             \
+        default: CALL(T, Q, G, 2); break;                                                            \
+    }
 #define TILE_CASES_TW(T, CALL)                                                                        \
-    case T * 16 + 0: CALL(T, false, 1); break; case T * 16 + 1: CALL(T, false, 2); break;           \
-    case T * 16 + 2: CALL(T, false, 4); break;                                                       \
-    case T * 16 + 8: CALL(T, true, 1); break;  case T * 16 + 9: CALL(T, true, 2); break;            \
-    case T * 16 + 10: CALL(T, true, 4); break;
+    case T * 16 + 0: TILE_CASES_DM(T, false, 1, CALL) break; case T * 16 + 1: TILE_CASES_DM(T, false, 2, CALL) break; \
+    case T * 16 + 2: TILE_CASES_DM(T, false, 4, CALL) break;                                          \
+    case T * 16 + 8: TILE_CASES_DM(T, true, 1, CALL) break;  case T * 16 + 9: TILE_CASES_DM(T, true, 2, CALL) break;  \
+    case T * 16 + 10: TILE_CASES_DM(T, true, 4, CALL) break;
 #define TILE_SWITCH(TWV, Q, NGV, CALL)                                                                \
     switch ((TWV) * 16 + ((Q) ? 8 : 0) + ((NGV) == 1 ? 0 : (NGV) == 2 ? 1 : (NGV) == 4 ? 2 : 7)) {  \
         TILE_CASES_TW(4, CALL) TILE_CASES_TW(8, CALL) TILE_CASES_TW(16, CALL) TILE_CASES_TW(32, CALL)  \
@@ -315,9 +323,10 @@ cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_ev
     const size_t smem = tile_smem_bytes(tw, ng, n_slots, n_eval, n_levels, desc_smem, max_width);
     cudaError_t e = cudaSuccess;
     int per = 0;
-#define TILE_PREP(T, Q, G)                                                                                        \
-    e = cudaFuncSetAttribute(k_tile<T, Q, G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);           \
-    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_tile<T, Q, G>, TILE_CTA, smem)
+    const int dmv = desc_smem;
+#define TILE_PREP(T, Q, G, D)                                                                                     \
+    e = cudaFuncSetAttribute(k_tile<T, Q, G, D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);        \
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_tile<T, Q, G, D>, TILE_CTA, smem)
     TILE_SWITCH(tw, has_q, ng, TILE_PREP)
 #undef TILE_PREP
     *per_sm = (uint32_t)per;
@@ -327,7 +336,8 @@ cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_ev
 cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s) {
     if (a.n_tiles == 0 || a.ncycles == 0) return cudaSuccess;
     const size_t smem = tile_smem_bytes(tw, ng, a.n_slots, a.n_eval, a.n_levels, a.desc_smem, a.max_width);
-#define TILE_LAUNCH(T, Q, G) k_tile<T, Q, G><<<grid, TILE_CTA, smem, s>>>(a)
+    const int dmv = (int)a.desc_smem;
+#define TILE_LAUNCH(T, Q, G, D) k_tile<T, Q, G, D><<<grid, TILE_CTA, smem, s>>>(a)
     TILE_SWITCH(tw, a.n_reg > 0, ng, TILE_LAUNCH)
 #undef TILE_LAUNCH
     return cudaGetLastError();
