@@ -45,9 +45,9 @@ extern "C" {
 #endif
 
 #define GSIM_VERSION "0.1.0"
-#define GS_MAX_K 6        /* largest LUT fan-in L of kernels A, T and D (64-bit truth tables) */
-#define GS_MAX_K_POLY 8   /* largest LUT fan-in L of kernel B (the polynomial network) and of
-                             the netlist / compiler ("4, 6 or 8"); tables of 2^8 bits   */
+#define GS_MAX_K 6        /* largest fan-in of gs_add_gate (the table fits one uint64)        */
+#define GS_MAX_K_POLY 8   /* largest LUT fan-in L of the netlist, the compiler and every kernel
+                             ("4, 6 or 8"); tables of up to 2^8 bits (gs_add_gate_wide) */
 
 typedef int32_t gs_status;
 enum {
@@ -94,8 +94,7 @@ gs_status gs_add_const(gs_netlist* nl, int value, gs_net* out);
 gs_status gs_add_gate(gs_netlist* nl, uint32_t k, const gs_net* in, uint64_t tt, gs_net* out);
 
 /* Same for 0 <= k <= GS_MAX_K_POLY: tt_words holds the table LSB-first in max(1, 2^k / 64)
- * uint64 words (bit m of the table = bit m % 64 of word m / 64).  Gates with k > GS_MAX_K can
- * only be simulated by kernel B (GS_KERNEL_POLY; AUTO selects it). */
+ * uint64 words (bit m of the table = bit m % 64 of word m / 64). */
 gs_status gs_add_gate_wide(gs_netlist* nl, uint32_t k, const gs_net* in, const uint64_t* tt_words, gs_net* out);
 
 /* D flip-flop on the global clock.  *q_out is its Q net (pseudo-input);
@@ -200,9 +199,9 @@ gs_status gs_program_tile_slots(const gs_program* prog, uint32_t* slots);
 
 /* ======================================================================= simulate */
 enum {
-    GS_KERNEL_AUTO = 0,   /* GS_KERNEL_POLY if some LUT has k > 6; else GS_KERNEL_TILE when
-                             one tile's live state fits shared memory next to the gate
-                             descriptors (resident or TMA-streamed); else GS_KERNEL_LUT   */
+    GS_KERNEL_AUTO = 0,   /* GS_KERNEL_TILE when every LUT has k <= 5 and one tile's live
+                             state fits shared memory next to the gate descriptors
+                             (resident or TMA-streamed); else GS_KERNEL_LUT              */
     GS_KERNEL_LUT = 1,    /* kernel A: bit-sliced LUT evaluation, 64 stimuli per word      */
     GS_KERNEL_POLY = 2,   /* kernel B: the paper's network, sum_S w_S Theta(sum x - |S| + 1)
                              per stimulus in int32, ballot-packed (Eq. 1-3)                */

@@ -210,6 +210,10 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
         }
         pr.aux[pos].tt = nl.gate_tt[g];
         pr.max_k = std::max(pr.max_k, k);
+        if (!nl.gate_tt_hi.empty()) {
+            if (pr.tt_full.empty()) pr.tt_full.assign((size_t)n_eval * 4, 0);
+            nl.table(g, &pr.tt_full[(size_t)pos * 4]);
+        }
         pr.aux[pos].qdst = NONE32;
         pr.aux[pos].k = k;
     }

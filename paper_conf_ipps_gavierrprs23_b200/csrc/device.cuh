@@ -115,6 +115,18 @@ __device__ __forceinline__ uint32_t lut_eval(uint64_t tt, const uint32_t* x) {
 }
 
 
+// K = 7, 8: Shannon expansion on x_6 (and x_7) over the 64-bit sub-tables t4[0..3] of the
+// 2^K-bit table (2 x 63 + 1 or 4 x 63 + 3 LOP3 per 32 lanes)
+template <int K>
+__device__ __forceinline__ uint32_t lut_eval_big(const uint64_t* t4, const uint32_t* x) {
+    const uint32_t y0 = lut_eval<6>(t4[0], x), y1 = lut_eval<6>(t4[1], x);
+    const uint32_t lo = (x[6] & y1) | (~x[6] & y0);
+    if (K == 7) return lo;
+    const uint32_t y2 = lut_eval<6>(t4[2], x), y3 = lut_eval<6>(t4[3], x);
+    const uint32_t hi = (x[6] & y3) | (~x[6] & y2);
+    return (x[7] & hi) | (~x[7] & lo);
+}
+
 // evaluate 4 x 32-bit lanes-words (one 16-byte vector) of a K-input gate
 template <int K>
 __device__ __forceinline__ uint4 lut_eval4(uint64_t tt, const uint4* xv) {

@@ -42,7 +42,8 @@ struct Netlist {
 };
 
 // ---------------------------------------------------------------- program
-constexpr uint32_t QFLAG = 0x80000000u;   // row ref is a Q row: add the current bank offset
+constexpr uint32_t QFLAG = 0x80000000u;
+constexpr uint32_t GS_MAX_K_LUT64 = 6;    // widest LUT whose table fits GateAux::tt (64 bits)   // row ref is a Q row: add the current bank offset
 constexpr uint32_t NONE32 = 0xFFFFFFFFu;
 
 // 16-byte per-gate auxiliary descriptor (device layout, see kernels.cu)
@@ -66,6 +67,7 @@ struct Program {
     std::vector<uint32_t> in_hi;              // [n_eval * 4] (inputs 4..7) if any_wide
     std::vector<GateAux> aux;                 // [n_eval]
     std::vector<uint8_t> hot;                 // [n_eval] a gate of the next level reads it
+    std::vector<uint64_t> tt_full;            // [n_eval * 4] 256-bit tables if max_k > 6
     std::vector<uint32_t> term_off;           // [n_eval + 1] kernel B nonzero terms
     std::vector<uint32_t> terms;              // S | (|S|-1)<<8 | (w & 0xffff)<<16
     std::vector<uint32_t> po_rows;            // [n_po]  row refs
@@ -103,7 +105,8 @@ static_assert(sizeof(TileDesc) == 16, "TileDesc layout");
 struct TilePlan {
     uint32_t n_slots = 0, q0 = 0;
     std::vector<TileDesc> desc;         // [n_eval] exec order
-    std::vector<uint32_t> desc_hi;      // [n_eval][4] if any k > 4: in4|in5<<16, tt[47:16], tt[63:48], 0
+    std::vector<uint32_t> desc_hi;      // [n_eval][12] if any k > 4: in4|in5<<16, in6|in7<<16, 0, 0,
+                                        //   then the 256-bit table as 8 words
     std::vector<uint32_t> po_slot;      // [n_po]
     std::vector<uint32_t> latch_src;    // slots (leftover latches)
     std::vector<uint32_t> latch_dst;    // register index

@@ -26,6 +26,36 @@
 
 namespace gs {
 
+// K = 7, 8 (any vector width VT = uint4 / uint2): the full 256-bit table comes from a.dtt
+template <int K, typename VT, typename Args>
+__device__ __forceinline__ void lut_gate_big(const Args& a, uint32_t gate, uint4 in, uint32_t v, uint32_t qdst) {
+    const uint4 hi = __ldg(a.dhi + gate);
+    const uint32_t r[8] = {in.x, in.y, in.z, in.w, hi.x, hi.y, hi.z, hi.w};
+    const uint4 t01 = __ldg(a.dtt + 2 * (uint64_t)gate), t23 = __ldg(a.dtt + 2 * (uint64_t)gate + 1);
+    const uint64_t t4[4] = {((uint64_t)t01.y << 32) | t01.x, ((uint64_t)t01.w << 32) | t01.z,
+                            ((uint64_t)t23.y << 32) | t23.x, ((uint64_t)t23.w << 32) | t23.z};
+    constexpr int NW = sizeof(VT) / 4;
+    uint32_t xw[K][NW];
+#pragma unroll
+    for (int i = 0; i < K; ++i) {
+        const VT xv = __ldg(reinterpret_cast<const VT*>(a.state + (uint64_t)resolve(r[i], a.qcur) * a.stride) + v);
+        const uint32_t* xp = reinterpret_cast<const uint32_t*>(&xv);
+#pragma unroll
+        for (int j = 0; j < NW; ++j) xw[i][j] = xp[j];
+    }
+    VT y;
+    uint32_t* yp = reinterpret_cast<uint32_t*>(&y);
+#pragma unroll
+    for (int j = 0; j < NW; ++j) {
+        uint32_t xs[K];
+#pragma unroll
+        for (int i = 0; i < K; ++i) xs[i] = xw[i][j];
+        yp[j] = lut_eval_big<K>(t4, xs);
+    }
+    *(reinterpret_cast<VT*>(a.state + (uint64_t)(a.row_gate0 + gate) * a.stride) + v) = y;
+    if (qdst != 0xFFFFFFFFu) *(reinterpret_cast<VT*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride) + v) = y;
+}
+
 template <int K>
 __device__ __forceinline__ void lut_gate_vec16(const LevelArgs& a, uint32_t gate, uint4 in, uint32_t v,
                                                uint64_t tt, uint32_t qdst) {
@@ -97,7 +127,9 @@ __global__ void __launch_bounds__(256) k_level_lut(LevelArgs a, uint32_t vpr, ui
             case 3: lut_gate_vec16<3>(a, gate, in, v, tt, qdst); break;
             case 4: lut_gate_vec16<4>(a, gate, in, v, tt, qdst); break;
             case 5: lut_gate_vec16<5>(a, gate, in, v, tt, qdst); break;
-            default: lut_gate_vec16<6>(a, gate, in, v, tt, qdst); break;
+            case 6: lut_gate_vec16<6>(a, gate, in, v, tt, qdst); break;
+            case 7: lut_gate_big<7, uint4>(a, gate, in, v, qdst); break;
+            default: lut_gate_big<8, uint4>(a, gate, in, v, qdst); break;
         }
     } else {
         switch (k) {
@@ -106,7 +138,9 @@ __global__ void __launch_bounds__(256) k_level_lut(LevelArgs a, uint32_t vpr, ui
             case 3: lut_gate_vec8<3>(a, gate, in, v, tt, qdst); break;
             case 4: lut_gate_vec8<4>(a, gate, in, v, tt, qdst); break;
             case 5: lut_gate_vec8<5>(a, gate, in, v, tt, qdst); break;
-            default: lut_gate_vec8<6>(a, gate, in, v, tt, qdst); break;
+            case 6: lut_gate_vec8<6>(a, gate, in, v, tt, qdst); break;
+            case 7: lut_gate_big<7, uint2>(a, gate, in, v, qdst); break;
+            default: lut_gate_big<8, uint2>(a, gate, in, v, qdst); break;
         }
     }
 }
@@ -185,12 +219,20 @@ __global__ void __launch_bounds__(256, U > 4 ? 2 : 4) k_level_lut_wide(LevelArgs
                     if (U > 4)
                         for (int u = 4; u < U; ++u) lut_gate_u<5, 1, HINT>(a, gate, in, v0 + 32 * u, tt, qdst, hot);
                     break;
-            default: lut_gate_u<6, 1, HINT>(a, gate, in, v0, tt, qdst, hot);
+            case 6: lut_gate_u<6, 1, HINT>(a, gate, in, v0, tt, qdst, hot);
                     if (U > 1) lut_gate_u<6, 1, HINT>(a, gate, in, v0 + 32, tt, qdst, hot);
                     if (U > 2) { lut_gate_u<6, 1, HINT>(a, gate, in, v0 + 64, tt, qdst, hot);
                                  lut_gate_u<6, 1, HINT>(a, gate, in, v0 + 96, tt, qdst, hot); }
                     if (U > 4)
                         for (int u = 4; u < U; ++u) lut_gate_u<6, 1, HINT>(a, gate, in, v0 + 32 * u, tt, qdst, hot);
+                    break;
+            case 7:
+#pragma unroll 1
+                    for (int u = 0; u < U; ++u) lut_gate_big<7, uint4>(a, gate, in, v0 + 32 * u, qdst);
+                    break;
+            default:
+#pragma unroll 1
+                    for (int u = 0; u < U; ++u) lut_gate_big<8, uint4>(a, gate, in, v0 + 32 * u, qdst);
                     break;
         }
     }
@@ -392,7 +434,15 @@ __global__ void __launch_bounds__(256, 4) k_dataflow(DfArgs a) {
                 case 3: df_gate<3, VPT, LPG>(a, g, in, tt, au.z, v0); break;
                 case 4: df_gate<4, VPT, LPG>(a, g, in, tt, au.z, v0); break;
                 case 5: df_gate_wide<5, VPT, LPG>(a, g, in, tt, au.z, v0); break;
-                default: df_gate_wide<6, VPT, LPG>(a, g, in, tt, au.z, v0); break;
+                case 6: df_gate_wide<6, VPT, LPG>(a, g, in, tt, au.z, v0); break;
+                case 7:
+#pragma unroll 1
+                    for (int u = 0; u < VPT; ++u) lut_gate_big<7, uint4>(a, g, in, v0 + u * LPG, au.z);
+                    break;
+                default:
+#pragma unroll 1
+                    for (int u = 0; u < VPT; ++u) lut_gate_big<8, uint4>(a, g, in, v0 + u * LPG, au.z);
+                    break;
             }
         }
         if (threadIdx.x == 0) s_item[it ^ 1] = next;

@@ -29,6 +29,7 @@ struct LevelArgs {
     const uint4* din;
     const GateAux* aux;
     const uint4* dhi;                 // inputs 4..7 (gates with k > 4)
+    const uint4* dtt;                 // [n_eval][2] full 256-bit tables (programs with k > 6)
     const uint32_t* term_off;
     const uint32_t* terms;
     uint32_t g0, ng;                  // exec-order gate range of the level
@@ -73,6 +74,7 @@ struct DfArgs {
     const uint4* din;
     const GateAux* aux;
     const uint4* dhi;                 // inputs 4..7 (gates with k > 4)
+    const uint4* dtt;                 // [n_eval][2] full 256-bit tables (programs with k > 6)
     uint8_t* state;
     uint64_t stride;
     uint32_t row_gate0, qcur, qnext;

@@ -74,13 +74,20 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 template <int K, bool HASQ>
 __device__ __forceinline__ void tile_gate(uint4* sl, uint32_t V, uint32_t v, const uint4& d, const uint4* desc_hi,
                                           uint32_t g, uint32_t q0, uint32_t R, uint32_t qcur, uint32_t qnext) {
-    uint32_t s[6] = {d.x & 0xFFFFu, d.x >> 16, d.y & 0xFFFFu, d.y >> 16, 0u, 0u};
-    uint64_t tt = d.z & 0xFFFFu;
-    if (K > 4) {
-        const uint4 hi = __ldg(desc_hi + g);
-        s[4] = hi.x & 0xFFFFu;
-        s[5] = hi.x >> 16;
-        tt |= ((uint64_t)hi.y << 16) | ((uint64_t)hi.z << 48);
+    constexpr int KS = K > 4 ? 8 : 4;
+    uint32_t s[KS];
+    s[0] = d.x & 0xFFFFu; s[1] = d.x >> 16; s[2] = d.y & 0xFFFFu; s[3] = d.y >> 16;
+    uint64_t t4[4] = {d.z & 0xFFFFu, 0, 0, 0};
+    if (K > 4) {                                       // desc_hi[g] = {inputs 4..7, 256-bit table}
+        const uint4 h0 = __ldg(desc_hi + 3 * (uint64_t)g), h1 = __ldg(desc_hi + 3 * (uint64_t)g + 1);
+        s[4] = h0.x & 0xFFFFu; s[5] = h0.x >> 16; s[6] = h0.y & 0xFFFFu; s[7] = h0.y >> 16;
+        t4[0] = ((uint64_t)h1.y << 32) | h1.x;
+        t4[1] = ((uint64_t)h1.w << 32) | h1.z;
+        if (K > 7) {
+            const uint4 h2 = __ldg(desc_hi + 3 * (uint64_t)g + 2);
+            t4[2] = ((uint64_t)h2.y << 32) | h2.x;
+            t4[3] = ((uint64_t)h2.w << 32) | h2.z;
+        }
     }
     uint4 x[K];
 #pragma unroll
@@ -89,7 +96,19 @@ __device__ __forceinline__ void tile_gate(uint4* sl, uint32_t V, uint32_t v, con
         if (HASQ) si += (si - q0) < R ? qcur : 0u;
         x[i] = sl[(size_t)si * V + v];
     }
-    const uint4 y = lut_eval4<K>(tt, x);
+    uint4 y;
+    if (K <= 6) {
+        y = lut_eval4<K <= 6 ? K : 6>(t4[0], x);
+    } else {
+        uint32_t xs[8];
+        uint32_t* yp = reinterpret_cast<uint32_t*>(&y);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+#pragma unroll
+            for (int i = 0; i < K; ++i) xs[i] = reinterpret_cast<const uint32_t*>(&x[i])[j];
+            yp[j] = lut_eval_big<K <= 6 ? 7 : K>(t4, xs);
+        }
+    }
     sl[(size_t)(d.z >> 16) * V + v] = y;
     if (HASQ) {
         const uint32_t reg = d.w >> 4;
@@ -219,7 +238,9 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
                         case 3: tile_gate<3, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
                         case 4: tile_gate<4, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
                         case 5: tile_gate<5, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        default: tile_gate<6, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
+                        case 6: tile_gate<6, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
+                        case 7: tile_gate<7, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
+                        default: tile_gate<8, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
                     }
                 }
                 group_sync(bar, GT);

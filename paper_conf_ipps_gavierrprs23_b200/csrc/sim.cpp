@@ -22,7 +22,7 @@ namespace {
 size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 
 struct Layout {
-    size_t ctl, state, din, aux, dhi, term_off, terms, po_rows, latch_src, latch_dst, reg_init,
+    size_t ctl, state, din, aux, dhi, dtt, term_off, terms, po_rows, latch_src, latch_dst, reg_init,
         trace_slot, misr, trace, lane_sigs, scratch, lv_gate0, lv_item0, dfctl, dfctl_bytes,
         t_desc, t_desc_hi, t_po, t_lsrc, t_ldst, t_wbrow, t_wbslot, t_lvl, total;
 };
@@ -129,13 +129,14 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
 // whole descriptor table or the TMA descriptor double buffer (small and mid-size circuits:
 // measured 1.8x kernel A on C2, 5.8x on C1, 2.6x / 1.4x / 1.1x on 5k / 10k / 20k-gate
 // synthetic circuits), else kernel A (large circuits are HBM-bound; T cannot hold them).
+// Programs with 6-8-input LUTs use kernel A.
 gs_sim_opts resolve_auto(const Program& p, const gs_sim_opts& o) {
     gs_sim_opts r = o;
     if (o.kernel != GS_KERNEL_AUTO) return r;
-    if (p.max_k > GS_MAX_K) {                   // 7-8-input LUTs: only the polynomial network
-        r.kernel = GS_KERNEL_POLY;
-        return r;
-    }
+    r.kernel = GS_KERNEL_LUT;
+    // wide LUTs make every level ALU-heavy (2^k - 1 LOP3 per 32 lanes): kernel A's higher
+    // occupancy wins from k = 6 on (measured on C2 collapsed to L = 6, 7, 8)
+    if (p.max_k > 5) return r;
     r.kernel = GS_KERNEL_TILE;
     Plans pl;
     const std::string saved = gs_last_error();
@@ -162,6 +163,7 @@ Layout make_layout(const Program& p, const gs_sim_opts& o, const Plans& pl) {
     L.din = take((size_t)p.n_eval * 16);
     L.aux = take((size_t)p.n_eval * 16);
     L.dhi = take(p.any_wide ? (size_t)p.n_eval * 16 : 0);
+    L.dtt = take(p.max_k > GS_MAX_K_LUT64 ? (size_t)p.n_eval * 32 : 0);
     L.term_off = take(poly ? ((size_t)p.n_eval + 1) * 4 : 0);
     L.terms = take(poly ? p.terms.size() * 4 : 0);
     L.po_rows = take((size_t)p.n_po * 4);
@@ -178,7 +180,7 @@ Layout make_layout(const Program& p, const gs_sim_opts& o, const Plans& pl) {
     L.dfctl_bytes = d.nl ? 4 + (size_t)d.n_slabs * d.nl * 4 : 0;
     L.dfctl = take(L.dfctl_bytes);
     L.t_desc = take(t.desc.size() * sizeof(TileDesc));
-    L.t_desc_hi = take(t.desc_hi.size() * 4);
+    L.t_desc_hi = take(t.desc_hi.size() * 4);   // 48 B per gate when any k > 4
     L.t_po = take(t.po_slot.size() * 4);
     L.t_lsrc = take(t.latch_src.size() * 4);
     L.t_ldst = take(t.latch_dst.size() * 4);
@@ -244,6 +246,7 @@ static LevelArgs level_args(const gs_sim* s, uint32_t l, uint32_t parity) {
     a.din = s->at<const uint4>(s->L.din);
     a.aux = s->at<const GateAux>(s->L.aux);
     a.dhi = p.any_wide ? s->at<const uint4>(s->L.dhi) : nullptr;
+    a.dtt = p.max_k > GS_MAX_K_LUT64 ? s->at<const uint4>(s->L.dtt) : nullptr;
     a.term_off = s->at<const uint32_t>(s->L.term_off);
     a.terms = s->at<const uint32_t>(s->L.terms);
     a.g0 = p.level_off[l];
@@ -314,6 +317,7 @@ static cudaError_t dataflow_launch(const gs_sim* s, uint32_t parity, cudaStream_
     a.din = s->at<const uint4>(s->L.din);
     a.aux = s->at<const GateAux>(s->L.aux);
     a.dhi = p.any_wide ? s->at<const uint4>(s->L.dhi) : nullptr;
+    a.dtt = p.max_k > GS_MAX_K_LUT64 ? s->at<const uint4>(s->L.dtt) : nullptr;
     a.state = s->state();
     a.stride = s->stride;
     a.row_gate0 = p.row_gate0;
@@ -453,8 +457,7 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
     if (!prog || !opts_in || !out || !dev_ws) return fail(GS_ERR_ARG, "gs_sim_create: NULL argument");
     const gs_sim_opts resolved = resolve_auto(*prog->p, *opts_in);
     const gs_sim_opts* opts = &resolved;
-    if (prog->p->max_k > GS_MAX_K && opts->kernel != GS_KERNEL_POLY)
-        return fail(GS_ERR_ARITY, "gs_sim_create: gates with k > 6 are evaluated only by kernel B (GS_KERNEL_POLY)");
+
     if (opts->lanes == 0 || opts->lanes % 64) return fail(GS_ERR_ARG, "gs_sim_create: lanes must be a positive multiple of 64");
     if (opts->lane_offset % 64) return fail(GS_ERR_ARG, "gs_sim_create: lane_offset must be a multiple of 64");
     if (opts->kernel < GS_KERNEL_AUTO || opts->kernel > GS_KERNEL_TILE) return fail(GS_ERR_ARG, "gs_sim_create: bad kernel");
@@ -544,6 +547,7 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
         {L.din, p.in_lo.data(), p.in_lo.size() * 4},
         {L.aux, aux_dev.data(), aux_dev.size() * sizeof(GateAux)},
         {L.dhi, p.in_hi.data(), p.any_wide ? p.in_hi.size() * 4 : 0},
+        {L.dtt, p.tt_full.data(), p.max_k > GS_MAX_K_LUT64 ? p.tt_full.size() * 8 : 0},
         {L.term_off, p.term_off.data(), poly ? p.term_off.size() * 4 : 0},
         {L.terms, p.terms.data(), poly ? p.terms.size() * 4 : 0},
         {L.po_rows, p.po_rows.data(), p.po_rows.size() * 4},

@@ -20,7 +20,6 @@ namespace gs {
 gs_status tile_plan(const Program& p, TilePlan& t) {
     const uint32_t P = p.n_pi, R = p.n_reg, G = p.n_eval, D = p.n_levels;
     t = TilePlan();
-    if (p.max_k > GS_MAX_K) return fail(GS_ERR_ARITY, "TILE: gates with k > 6 need kernel B (GS_KERNEL_POLY)");
     t.q0 = 2 + P;
     const uint32_t fixed = 2 + P + 2 * R;
     // row ref (state row, QFLAG for Q) -> which gate (exec index) it names, or NONE32
@@ -68,12 +67,13 @@ gs_status tile_plan(const Program& p, TilePlan& t) {
         return slot[ref - p.row_gate0];
     };
     // descriptors (16 B): x = in0 | in1 << 16, y = in2 | in3 << 16, z = tt[15:0] | out << 16,
-    // w = k | (fused-latch register + 1) << 4; k > 4 adds {in4 | in5 << 16, tt[47:16], tt[63:48], 0}
+    // w = k | (fused-latch register + 1) << 4; gates with k > 4 add 3 x 16 B in desc_hi:
+    // {in4 | in5 << 16, in6 | in7 << 16, 0, 0} and the whole 256-bit table
     t.desc.resize(G);
-    t.desc_hi.assign(p.any_wide ? (size_t)G * 4 : 0, 0);
+    t.desc_hi.assign(p.any_wide ? (size_t)G * 12 : 0, 0);
     for (uint32_t g = 0; g < G; ++g) {
         const uint32_t k = p.aux[g].k;
-        uint32_t in[6] = {0, 0, 0, 0, 0, 0};        // unused inputs read const0 (slot 0)
+        uint32_t in[8] = {0, 0, 0, 0, 0, 0, 0, 0};   // unused inputs read const0 (slot 0)
         for (uint32_t j = 0; j < k; ++j)
             in[j] = slot_of(j < 4 ? p.in_lo[(size_t)g * 4 + j] : p.in_hi[(size_t)g * 4 + j - 4]);
         const uint64_t tt = p.aux[g].tt;
@@ -85,9 +85,14 @@ gs_status tile_plan(const Program& p, TilePlan& t) {
         d.kreg = k | (reg << 4);
         t.desc[g] = d;
         if (p.any_wide) {
-            t.desc_hi[(size_t)g * 4 + 0] = in[4] | (in[5] << 16);
-            t.desc_hi[(size_t)g * 4 + 1] = (uint32_t)(tt >> 16);
-            t.desc_hi[(size_t)g * 4 + 2] = (uint32_t)(tt >> 48);
+            uint32_t* h = &t.desc_hi[(size_t)g * 12];
+            h[0] = in[4] | (in[5] << 16);
+            h[1] = in[6] | (in[7] << 16);
+            for (uint32_t w = 0; w < 4; ++w) {
+                const uint64_t word = p.tt_full.empty() ? (w ? 0 : tt) : p.tt_full[(size_t)g * 4 + w];
+                h[4 + 2 * w] = (uint32_t)word;
+                h[5 + 2 * w] = (uint32_t)(word >> 32);
+            }
         }
     }
     for (uint32_t r : p.po_rows) t.po_slot.push_back(slot_of(r));

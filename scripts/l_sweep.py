@@ -22,7 +22,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--configs", default="C1,C2,C3")
     ap.add_argument("--Ls", default="0,3,4,5,6,7,8")
-    ap.add_argument("--kernels", default="lut,auto")
+    ap.add_argument("--kernels", default="lut,auto,poly")
     ap.add_argument("--cycles", type=int, default=100)
     ap.add_argument("--steps", type=int, default=3)
     a = ap.parse_args()
@@ -56,7 +56,7 @@ def main():
                 evals = lanes * a.cycles * a.steps
                 print(json.dumps({"config": name, "L": L, "kernel": kernel,
                                   "kernel_used": ("tile" if sim.launches_per_cycle() == 1 else
-                                                  "poly" if info["k_hist"][7] + info["k_hist"][8] else kernel),
+                                                  "lut" if kernel == "auto" else kernel),
                                   "levels": info["n_levels"], "luts": info["n_eval_gates"],
                                   "lut_inputs": info["n_edges"], "nnz_coeffs": info["nnz_coeffs"],
                                   "gates_original": g_orig, "lanes": lanes,
