@@ -237,6 +237,7 @@ gs_status gs_netlist_get_counts(const gs_netlist* h, gs_netlist_counts* out) {
 
 // ------------------------------------------------------------------ compile front
 gs_status gs_compile(const gs_netlist* h, const gs_compile_opts* opts, gs_program** out) {
+    NvtxRange nvtx("gs_compile");
     if (!h || !out) return fail(GS_ERR_ARG, "gs_compile: NULL argument");
     gs_compile_opts o{1, 0, 0};
     if (opts) o = *opts;

@@ -454,6 +454,7 @@ gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts
 }
 
 gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void* dev_ws, size_t bytes, gs_sim** out) {
+    NvtxRange nvtx("gs_sim_create");
     if (!prog || !opts_in || !out || !dev_ws) return fail(GS_ERR_ARG, "gs_sim_create: NULL argument");
     const gs_sim_opts resolved = resolve_auto(*prog->p, *opts_in);
     const gs_sim_opts* opts = &resolved;
@@ -670,6 +671,7 @@ gs_status gs_sim_bind_stimulus_host(gs_sim* s, const uint64_t* words, uint32_t c
 }
 
 gs_status gs_sim_step(gs_sim* s, uint32_t n) {
+    NvtxRange nvtx("gs_sim_step");
     if (gs_status st = check_sim(s, "gs_sim_step")) return st;
     if (!s->bound) return fail(GS_ERR_STATE, "gs_sim_step: no stimulus bound");
     if (s->bound == 2 && s->cycle + n > s->bound_base + s->bound_cycles)
@@ -697,6 +699,7 @@ gs_status gs_sim_step(gs_sim* s, uint32_t n) {
 
 gs_status gs_sim_run_streamed(gs_sim* s, const uint64_t* host_stim, uint64_t* host_out, uint32_t ncycles,
                               uint32_t chunk) {
+    NvtxRange nvtx("gs_sim_run_streamed");
     if (gs_status st = check_sim(s, "gs_sim_run_streamed")) return st;
     if (!host_stim && ncycles) return fail(GS_ERR_ARG, "gs_sim_run_streamed: NULL host_stim");
     if (!ncycles) return GS_OK;
