@@ -86,6 +86,7 @@ __device__ __forceinline__ uint32_t lut_eval(uint64_t tt, const uint32_t* x);
 // time, so the register footprint stays that of K = 4 (keeps occupancy up).
 template <int K>
 __device__ __forceinline__ uint32_t lut_eval_wide(uint64_t tt, const uint32_t* x) {
+    static_assert(K == 5 || K == 6, "lut_eval_wide: K = 5, 6");
     uint32_t y[4];
 #pragma unroll 1
     for (int j = 0; j < (1 << (K - 4)); ++j) y[j] = lut_eval<4>(tt >> (16 * j), x);
@@ -97,7 +98,7 @@ __device__ __forceinline__ uint32_t lut_eval_wide(uint64_t tt, const uint32_t* x
 
 template <int K>
 __device__ __forceinline__ uint32_t lut_eval(uint64_t tt, const uint32_t* x) {
-    if (K > 4) return lut_eval_wide<K>(tt, x);
+    if constexpr (K > 4) return lut_eval_wide<K>(tt, x);
     constexpr int KK = K > 4 ? 4 : K;
     uint32_t v[1 << (KK - 1)];
 #pragma unroll
