@@ -283,6 +283,18 @@ def test_errors_on_device():
     sim.close()
 
 
+@pytest.mark.parametrize("slabs", [2, 4])
+def test_lane_slabs_do_not_change_results(slabs):
+    """Kernel A run slab-major (all levels on 1/slabs of the lanes, then the next slab)."""
+    cfg = workloads.CONFIGS["C3"]
+    nl = cfg.netlist()
+    prog = compile_nl(nl)
+    a = run_gpu(nl, 16384, 12, "lut", seed=8, prog=prog)
+    b = run_gpu(nl, 16384, 12, "lut", seed=8, prog=prog, lane_slabs=slabs)
+    for key in ("outputs", "regs", "sigs"):
+        assert np.array_equal(a[key], b[key]), key
+
+
 @pytest.mark.parametrize("flags", [gs.GS_SIM_NO_PDL, 2, 6, 8])
 def test_launch_and_cache_options_do_not_change_results(flags):
     """PDL off, L2 eviction hints on stores, hints on stores and loads: bit-identical."""
