@@ -1,33 +1,9 @@
-// kernels_tile.cu — kernel T: tile-resident simulation in shared memory (sm_100a).
-//
-// Stimuli are independent, so a tile of 32*TW lanes can run every level of
-// every cycle of a step without ever synchronising with another tile.  One CTA owns a
-// tile at a time: its live state (slots of tile.cpp: constants, PIs, both register
-// banks, gate values by live range) sits in shared memory as TW 32-bit words per slot,
-// and each level (one merged NN layer) is one pass of the CTA over
-// (gate, word) units separated by __syncthreads.  HBM sees only the register rows and
-// MISR planes at the start and end of a step: no per-level launch, no per-level round
-// trip through HBM.  Narrow, deep circuits (the 32x32 multiplier has 184 levels of median
-// width 28) are latency-bound per tile, so many tiles run per SM at once.
-//
-// Semantics are exactly kernel A's: the same PI hash (R2), the same double-buffered
-// latch (R3), outputs sampled before the latch (R4), the same bit-sliced MISR (R5), so
-// lane signatures, outputs, registers and the trace are bit-identical.
-#include <cuda_runtime.h>
-
-#include "device.cuh"
-#include "kernels.h"
+// kernels_tile.cu — kernel T dispatch: plan-time setup and launch by tile width (the
+// template instantiations live in kernels_tile_tw{4,8,16,32}.cu).
+#include "kernels_tile.cuh"
 
 namespace gs {
 
-constexpr uint32_t TILE_CTA = 512;                   // threads per CTA (one CTA per SM)
-constexpr unsigned long long TILE_MISR_POLY = 0x42F0E1EBA9EA3693ULL;   // CRC-64/ECMA-182
-
-// Shared memory by descriptor mode:
-//   1 (resident): [desc: 16 B x n_eval] [level_off: 4 B x (n_levels + 1), padded to 16 B]
-//   2 (TMA-streamed): [level_off] then per group [2 mbarriers, 16 B][2 x max_width x 16 B]
-//   0 (global): nothing
-// then per thread group: [slots: n_slots x TW words] [MISR: 64 x TW words].
 static size_t lvl_bytes(uint32_t n_levels) { return (((size_t)n_levels + 1) * 4 + 15) / 16 * 16; }
 
 size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
@@ -41,315 +17,18 @@ size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_ev
     return b + (size_t)ng * g;
 }
 
-// ---- TMA bulk copy (cp.async.bulk) of a level's descriptors into shared memory, completion
-// signalled on an mbarrier (expect_tx / complete_tx), consumers wait on the phase parity
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-    return (uint32_t)__cvta_generic_to_shared(p);
-}
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // prior generic reads of dst
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-                 : "memory");
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
-                 : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-    uint32_t done = 0;
-    while (!done) {
-        asm volatile(
-            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
-            : "=r"(done)
-            : "r"(smem_u32(bar)), "r"(parity)
-            : "memory");
-    }
-}
-
-// One gate on one 16-byte group (4 words = 128 lanes) of its slots.  HASQ: the circuit has
-// registers, so an input slot may name a bank-0 register slot that must be moved to the
-// current bank.
-template <int K, bool HASQ>
-__device__ __forceinline__ void tile_gate(uint4* sl, uint32_t V, uint32_t v, const uint4& d, const uint4* desc_hi,
-                                          uint32_t g, uint32_t q0, uint32_t R, uint32_t qcur, uint32_t qnext) {
-    constexpr int KS = K > 4 ? 8 : 4;
-    uint32_t s[KS];
-    s[0] = d.x & 0xFFFFu; s[1] = d.x >> 16; s[2] = d.y & 0xFFFFu; s[3] = d.y >> 16;
-    uint64_t t4[4] = {d.z & 0xFFFFu, 0, 0, 0};
-    if (K > 4) {                                       // desc_hi[g] = {inputs 4..7, 256-bit table}
-        const uint4 h0 = __ldg(desc_hi + 3 * (uint64_t)g), h1 = __ldg(desc_hi + 3 * (uint64_t)g + 1);
-        s[4] = h0.x & 0xFFFFu; s[5] = h0.x >> 16; s[6] = h0.y & 0xFFFFu; s[7] = h0.y >> 16;
-        t4[0] = ((uint64_t)h1.y << 32) | h1.x;
-        t4[1] = ((uint64_t)h1.w << 32) | h1.z;
-        if (K > 7) {
-            const uint4 h2 = __ldg(desc_hi + 3 * (uint64_t)g + 2);
-            t4[2] = ((uint64_t)h2.y << 32) | h2.x;
-            t4[3] = ((uint64_t)h2.w << 32) | h2.z;
-        }
-    }
-    uint4 x[K];
-#pragma unroll
-    for (int i = 0; i < K; ++i) {
-        uint32_t si = s[i];
-        if (HASQ) si += (si - q0) < R ? qcur : 0u;
-        x[i] = sl[(size_t)si * V + v];
-    }
-    uint4 y;
-    if (K <= 6) {
-        y = lut_eval4<K <= 6 ? K : 6>(t4[0], x);
-    } else {
-        uint32_t xs[8];
-        uint32_t* yp = reinterpret_cast<uint32_t*>(&y);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-#pragma unroll
-            for (int i = 0; i < K; ++i) xs[i] = reinterpret_cast<const uint32_t*>(&x[i])[j];
-            yp[j] = lut_eval_big<K <= 6 ? 7 : K>(t4, xs);
-        }
-    }
-    sl[(size_t)(d.z >> 16) * V + v] = y;
-    if (HASQ) {
-        const uint32_t reg = d.w >> 4;
-        if (reg) sl[(size_t)(q0 + reg - 1 + qnext) * V + v] = y;      // fused latch
-    }
-}
-
-__device__ __forceinline__ void group_sync(uint32_t id, uint32_t nthreads) {
-    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
-}
-
-// TW = 32-bit words per slot (tile = 32 * TW lanes).  A thread evaluates one gate on one
-// 16-byte group of 4 words (128 lanes): k 16-byte shared-memory loads, 4 x (2^k - 1) LOP3,
-// one 16-byte store.  The CTA (TILE_CTA threads) is split into NG independent groups; each
-// group simulates its own tile and synchronises only with itself (named barrier 1 + gid),
-// so one group's level barrier overlaps the other groups' work.  All groups share the
-// descriptor table in shared memory.
-template <int TW, bool HASQ, int NG, int DM>
-__global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
-    constexpr uint32_t V = TW / 4;                       // uint4 per slot
-    constexpr uint32_t GT = TILE_CTA / NG;               // threads per group
-    extern __shared__ uint4 smem[];
-    const uint4* dsm = DM == 1 ? smem : reinterpret_cast<const uint4*>(a.desc);
-    const uint32_t* lvl = a.level_off;
-    uint4* base = smem;
-    if (DM == 1) {
-        uint32_t* lv = reinterpret_cast<uint32_t*>(smem + a.n_eval);
-        const uint4* gd = reinterpret_cast<const uint4*>(a.desc);
-        for (uint32_t i = threadIdx.x; i < a.n_eval; i += blockDim.x) smem[i] = __ldg(gd + i);
-        for (uint32_t i = threadIdx.x; i <= a.n_levels; i += blockDim.x) lv[i] = __ldg(a.level_off + i);
-        lvl = lv;
-        base = smem + a.n_eval + ((a.n_levels + 1) * 4 + 15) / 16;
-    } else if (DM == 2) {
-        uint32_t* lv = reinterpret_cast<uint32_t*>(smem);
-        for (uint32_t i = threadIdx.x; i <= a.n_levels; i += blockDim.x) lv[i] = __ldg(a.level_off + i);
-        lvl = lv;
-        base = smem + ((a.n_levels + 1) * 4 + 15) / 16;
-    }
-    const uint32_t gid = threadIdx.x / GT, tid = threadIdx.x % GT, bd = GT;
-    const uint32_t bar = 1 + gid;
-    // group region: [mbarriers + descriptor double buffer (mode 2)] [slots] [MISR]
-    uint4* greg = base + (size_t)gid * ((a.n_slots + 64) * V + (DM == 2 ? 1 + 2 * a.max_width : 0));
-    uint64_t* mbar = reinterpret_cast<uint64_t*>(greg);
-    uint4* dbuf = greg + 1;                                   // [2][max_width]
-    uint4* sl = DM == 2 ? greg + 1 + 2 * a.max_width : greg;   // this group's slots
-    if (DM == 2 && tid == 0) {
-        mbar_init(mbar, 1);
-        mbar_init(mbar + 1, 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    uint32_t* sw = reinterpret_cast<uint32_t*>(sl);          // slots as 32-bit words
-    uint32_t* mp = sw + (size_t)a.n_slots * TW;               // MISR planes [64][TW]
-    const unsigned long long c0 = a.ctl->cycle;
-    const uint32_t R = a.n_reg, q0 = a.q0;
-    const uint32_t w32_row = a.words * 2;                     // 32-bit words per state row
-    const uint32_t* st32 = reinterpret_cast<const uint32_t*>(a.state);
-    uint32_t* st32w = reinterpret_cast<uint32_t*>(a.state);
-    // MISR planes are double-buffered by cycle parity (as k_end_cycle): read the buffer of
-    // the first cycle, write the buffer of the cycle after the last
-    const uint32_t* misr_in = reinterpret_cast<const uint32_t*>(a.misr + (size_t)(c0 & 1) * 64 * a.words);
-    uint32_t* misr_out = reinterpret_cast<uint32_t*>(a.misr + (size_t)((c0 + a.ncycles) & 1) * 64 * a.words);
-    unsigned long long pop = 0;
-    // mode 2: the group's descriptor stream, one level per step, double-buffered: while
-    // level l is evaluated from buffer (step & 1), the TMA engine fetches the next level
-    // (the same sequence repeats every cycle and every tile)
-    uint32_t step = 0;
-    if (DM == 2 && tid == 0 && blockIdx.x * NG + gid < a.n_tiles)
-        tma_load_1d(dbuf, a.desc + lvl[0], (lvl[1] - lvl[0]) * 16, mbar);
-
-    for (uint32_t tile = blockIdx.x * NG + gid; tile < a.n_tiles; tile += gridDim.x * NG) {
-        const bool last_tile = tile + gridDim.x * NG >= a.n_tiles;
-        const uint32_t t0 = tile * TW;                    // first 32-bit word of the tile (shard-local)
-        // ---- load: constants, both register banks, MISR planes
-        for (uint32_t u = tid; u < TW; u += bd) {
-            sw[u] = 0u;
-            sw[TW + u] = 0xFFFFFFFFu;
-        }
-        for (uint32_t u = tid; u < 2 * R * TW; u += bd) {
-            const uint32_t r = u / TW, w = u % TW;
-            sw[(size_t)(q0 + r) * TW + w] = st32[(uint64_t)(a.row_q0 + r) * w32_row + t0 + w];
-        }
-        for (uint32_t u = tid; u < 64 * TW; u += bd) {
-            const uint32_t j = u / TW, w = u % TW;
-            mp[u] = misr_in[(uint64_t)j * w32_row + t0 + w];
-        }
-        group_sync(bar, GT);
-        for (uint32_t c = 0; c < a.ncycles; ++c) {
-            const unsigned long long cyc = c0 + c;
-            const uint32_t qcur = (cyc & 1) ? R : 0u, qnext = R - qcur;
-            // ---- primary inputs of this cycle (R2): one 64-bit hash per pair of words
-            for (uint32_t u = tid; u < a.n_pi * (TW / 2); u += bd) {
-                const uint32_t p = u / (TW / 2), w2 = u % (TW / 2);
-                const uint32_t g64 = (t0 >> 1) + w2;      // shard-local 64-bit word
-                unsigned long long v;
-                if (a.ctl->stim_mode == 0) {
-                    v = dmix64(dmix64(dmix64(a.ctl->seed ^ p) ^ cyc) ^ (a.word_off + g64));
-                } else {
-                    const unsigned long long* src = reinterpret_cast<const unsigned long long*>(a.ctl->stim_ptr);
-                    v = src[((cyc - a.ctl->stim_base) * a.n_pi + p) * a.words + g64];
-                }
-                reinterpret_cast<unsigned long long*>(sw + (size_t)(2 + p) * TW)[w2] = v;
-            }
-            group_sync(bar, GT);
-            // ---- levels: every (gate, 16-byte group) unit of the level, then a barrier
-            for (uint32_t l = 0; l < a.n_levels; ++l) {
-                const uint32_t g0 = lvl[l], n = (lvl[l + 1] - g0) * V;
-                const uint4* dl = dsm + g0;
-                if (DM == 2) {
-                    const uint32_t b = step & 1;
-                    if (tid == 0 && !(last_tile && c + 1 == a.ncycles && l + 1 == a.n_levels)) {
-                        const uint32_t ln = l + 1 == a.n_levels ? 0 : l + 1;
-                        tma_load_1d(dbuf + (b ^ 1) * a.max_width, a.desc + lvl[ln], (lvl[ln + 1] - lvl[ln]) * 16,
-                                    mbar + (b ^ 1));
-                    }
-                    mbar_wait(mbar + b, (step >> 1) & 1);
-                    dl = dbuf + b * a.max_width;
-                    ++step;
-                }
-                for (uint32_t u = tid; u < n; u += bd) {
-                    const uint32_t gi = u / V, v = u % V;
-                    const uint32_t g = g0 + gi;
-                    const uint4 d = dl[gi];
-                    switch (d.w & 15u) {                       // k: warp-uniform except at k-group edges
-                        case 1: tile_gate<1, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        case 2: tile_gate<2, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        case 3: tile_gate<3, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        case 4: tile_gate<4, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        case 5: tile_gate<5, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        case 6: tile_gate<6, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        case 7: tile_gate<7, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        default: tile_gate<8, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                    }
-                }
-                group_sync(bar, GT);
-            }
-            // ---- leftover latches into the next bank; MISR / popcount / trace of the POs
-            for (uint32_t u = tid; u < a.n_latch * V; u += bd) {
-                const uint32_t e = u / V, v = u % V;
-                uint32_t s = __ldg(a.latch_src + e);
-                s += (s - q0) < R ? qcur : 0u;
-                sl[(size_t)(q0 + __ldg(a.latch_dst + e) + qnext) * V + v] = sl[(size_t)s * V + v];
-            }
-            constexpr uint32_t NP = (64 * TW + GT - 1) / GT;    // MISR plane words per thread
-            uint32_t newp[NP];
-            const bool tr = a.trace && cyc < a.trace_cap;
-#pragma unroll
-            for (uint32_t i = 0; i < NP; ++i) {
-                const uint32_t u = tid + i * bd;
-                if (u >= 64 * TW) break;
-                const uint32_t j = u / TW, w = u % TW;
-                const uint32_t g32 = t0 + w;
-                const int32_t tslot = tr ? __ldg(a.trace_slot + (g32 >> 1)) : -1;
-                uint32_t* sink = nullptr;                          // full per-cycle output stream
-                if (a.ctl->sink_ptr && cyc - a.ctl->sink_base < a.ctl->sink_cycles)
-                    sink = reinterpret_cast<uint32_t*>(a.ctl->sink_ptr) +
-                           (cyc - a.ctl->sink_base) * a.n_po * (uint64_t)w32_row;
-                uint32_t vv = 0;
-                for (uint32_t o = j; o < a.n_po; o += 64) {
-                    uint32_t s = __ldg(a.po_slot + o);
-                    s += (s - q0) < R ? qcur : 0u;
-                    const uint32_t x = sw[(size_t)s * TW + w];
-                    vv ^= x;
-                    pop += __popc(x);
-                    if (tslot >= 0)
-                        reinterpret_cast<uint32_t*>(a.trace)[(((uint64_t)cyc * a.n_po + o) * a.ntw + tslot) * 2 +
-                                                             (g32 & 1)] = x;
-                    if (sink) sink[(uint64_t)o * w32_row + g32] = x;
-                }
-                const uint32_t prev = j ? mp[(j - 1) * TW + w] : 0u;
-                const uint32_t fb = ((TILE_MISR_POLY >> j) & 1ULL) ? mp[63 * TW + w] : 0u;
-                newp[i] = prev ^ fb ^ vv;
-            }
-            group_sync(bar, GT);
-#pragma unroll
-            for (uint32_t i = 0; i < NP; ++i)
-                if (tid + i * bd < 64 * TW) mp[tid + i * bd] = newp[i];
-            group_sync(bar, GT);
-        }
-        // ---- write back: both register banks, PO rows (read_outputs), MISR planes
-        for (uint32_t u = tid; u < 2 * R * TW; u += bd) {
-            const uint32_t r = u / TW, w = u % TW;
-            st32w[(uint64_t)(a.row_q0 + r) * w32_row + t0 + w] = sw[(size_t)(q0 + r) * TW + w];
-        }
-        for (uint32_t u = tid; u < a.n_wb * TW; u += bd) {
-            const uint32_t e = u / TW, w = u % TW;
-            st32w[(uint64_t)__ldg(a.wb_row + e) * w32_row + t0 + w] = sw[(size_t)__ldg(a.wb_slot + e) * TW + w];
-        }
-        for (uint32_t u = tid; u < 64 * TW; u += bd) {
-            const uint32_t j = u / TW, w = u % TW;
-            misr_out[(uint64_t)j * w32_row + t0 + w] = mp[u];
-        }
-        group_sync(bar, GT);                              // before the next tile reuses smem
-    }
-    // ---- counters; the last CTA advances the device clock
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) pop += __shfl_xor_sync(FULL, pop, o);
-    if ((threadIdx.x & 31) == 0 && pop) atomicAdd(&a.ctl->popcount, pop);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();
-        const unsigned int prev = atomicAdd(&a.ctl->done, 1u);
-        if (prev == gridDim.x - 1) {
-            a.ctl->done = 0u;
-            a.ctl->cycle = c0 + a.ncycles;
-            __threadfence();
-        }
-    }
-}
-
-// instantiations: TW in {4, 8, 16, 32} x registers present x groups {1, 2, 4} x descriptor
-// source {global, resident, TMA stream} (a compile-time source lets ptxas emit LDS for
-// shared-memory descriptors instead of generic loads)
-#define TILE_CASES_DM(T, Q, G, CALL)                                                                  \
-    switch (dmv) {                                                                                   \
-        case 0: CALL(T, Q, G, 0); break;                                                             \
-        case 1: CALL(T, Q, G, 1); break;                                                             \
-        default: CALL(T, Q, G, 2); break;                                                            \
-    }
-#define TILE_CASES_TW(T, CALL)                                                                        \
-    case T * 16 + 0: TILE_CASES_DM(T, false, 1, CALL) break; case T * 16 + 1: TILE_CASES_DM(T, false, 2, CALL) break; \
-    case T * 16 + 2: TILE_CASES_DM(T, false, 4, CALL) break;                                          \
-    case T * 16 + 8: TILE_CASES_DM(T, true, 1, CALL) break;  case T * 16 + 9: TILE_CASES_DM(T, true, 2, CALL) break;  \
-    case T * 16 + 10: TILE_CASES_DM(T, true, 4, CALL) break;
-#define TILE_SWITCH(TWV, Q, NGV, CALL)                                                                \
-    switch ((TWV) * 16 + ((Q) ? 8 : 0) + ((NGV) == 1 ? 0 : (NGV) == 2 ? 1 : (NGV) == 4 ? 2 : 7)) {  \
-        TILE_CASES_TW(4, CALL) TILE_CASES_TW(8, CALL) TILE_CASES_TW(16, CALL) TILE_CASES_TW(32, CALL)  \
-        default: return cudaErrorInvalidValue;                                                        \
-    }
-
 cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
                        int desc_smem, uint32_t max_width, uint32_t has_q, uint32_t* per_sm) {
     const size_t smem = tile_smem_bytes(tw, ng, n_slots, n_eval, n_levels, desc_smem, max_width);
-    cudaError_t e = cudaSuccess;
     int per = 0;
-    const int dmv = desc_smem;
-#define TILE_PREP(T, Q, G, D)                                                                                     \
-    e = cudaFuncSetAttribute(k_tile<T, Q, G, D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);        \
-    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_tile<T, Q, G, D>, TILE_CTA, smem)
-    TILE_SWITCH(tw, has_q, ng, TILE_PREP)
-#undef TILE_PREP
+    cudaError_t e;
+    switch (tw) {
+        case 4: e = tile_setup_tw<4>(ng, smem, desc_smem, has_q, &per); break;
+        case 8: e = tile_setup_tw<8>(ng, smem, desc_smem, has_q, &per); break;
+        case 16: e = tile_setup_tw<16>(ng, smem, desc_smem, has_q, &per); break;
+        case 32: e = tile_setup_tw<32>(ng, smem, desc_smem, has_q, &per); break;
+        default: return cudaErrorInvalidValue;
+    }
     *per_sm = (uint32_t)per;
     return e;
 }
@@ -357,11 +36,13 @@ cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_ev
 cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s) {
     if (a.n_tiles == 0 || a.ncycles == 0) return cudaSuccess;
     const size_t smem = tile_smem_bytes(tw, ng, a.n_slots, a.n_eval, a.n_levels, a.desc_smem, a.max_width);
-    const int dmv = (int)a.desc_smem;
-#define TILE_LAUNCH(T, Q, G, D) k_tile<T, Q, G, D><<<grid, TILE_CTA, smem, s>>>(a)
-    TILE_SWITCH(tw, a.n_reg > 0, ng, TILE_LAUNCH)
-#undef TILE_LAUNCH
-    return cudaGetLastError();
+    switch (tw) {
+        case 4: return launch_tile_tw<4>(a, ng, grid, smem, s);
+        case 8: return launch_tile_tw<8>(a, ng, grid, smem, s);
+        case 16: return launch_tile_tw<16>(a, ng, grid, smem, s);
+        case 32: return launch_tile_tw<32>(a, ng, grid, smem, s);
+        default: return cudaErrorInvalidValue;
+    }
 }
 
 }  // namespace gs
