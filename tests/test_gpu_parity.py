@@ -675,3 +675,31 @@ def test_fuzz_every_kernel_all_lanes_vs_oracle(case):
         assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"]), kernel
         assert np.array_equal(r["sigs"], o["sig"]), kernel
         assert r["signature"]["ab_mismatch"] == 0 and r["signature"]["invariant_violations"] == 0
+
+
+# ------------------------------------------------------------------ AES-128 core (FIPS-197)
+@pytest.mark.parametrize("kernel", ["auto", "lut", "tile", "poly", "ab"])
+def test_aes128_core_every_lane(kernel):
+    """A real circuit of the paper's Table I family: the iterative AES-128 core (8-input S-box
+    LUTs, 260 registers).  Ciphertexts on every lane equal the oracle's, the first 256 equal an
+    independent textbook AES, lane 0 is FIPS-197 Appendix C.1."""
+    from workloads import aes
+    from tests import _aes_ref
+    nl = aes.aes128_core()
+    prog = compile_nl(nl)
+    lanes = 4096
+    rng = np.random.default_rng(11)
+    keys = rng.integers(0, 256, size=(lanes, 16), dtype=np.uint8)
+    pts = rng.integers(0, 256, size=(lanes, 16), dtype=np.uint8)
+    keys[0] = np.frombuffer(bytes.fromhex("000102030405060708090a0b0c0d0e0f"), dtype=np.uint8)
+    pts[0] = np.frombuffer(bytes.fromhex("00112233445566778899aabbccddeeff"), dtype=np.uint8)
+    stim = aes.aes_stimulus(keys, pts)
+    r = run_gpu(nl, lanes, 12, kernel, host_stim=stim, prog=prog)
+    ct = aes.ciphertexts(gs.unpack_lanes(r["outputs"]).T)
+    assert bytes(ct[0]).hex() == "69c4e0d86a7b0430d8cdb78070b4c55a"
+    o = oracle.simulate(nl, np.arange(lanes), 12, host_stim=stim, want=("last", "sig"))
+    assert np.array_equal(ct, aes.ciphertexts(o["last"]))
+    assert np.array_equal(r["sigs"], o["sig"])
+    for s in range(256):
+        assert bytes(ct[s]) == _aes_ref.encrypt(bytes(keys[s]), bytes(pts[s]))
+    assert r["signature"]["ab_mismatch"] == 0 and r["signature"]["invariant_violations"] == 0

@@ -189,14 +189,18 @@ class Builder:
         off[1:] = np.cumsum(ks.astype(np.int64))
         ins = np.array([nid(r) for g, _ in self.gates for r in g], dtype=U32)
         assert all(d is not None for d in self.reg_d), "register without D"
+        M64 = (1 << 64) - 1
+        wide = any(len(g) > 6 for g, _ in self.gates)
+        hi = (np.array([[(tt >> (64 * j)) & M64 for j in (1, 2, 3)] for _, tt in self.gates], dtype=np.uint64)
+              if wide else None)
         return Netlist(
             n_pi=n_pi,
             reg_init=np.array(self.reg_init, dtype=np.uint8),
             reg_d=np.array([nid(d) for d in self.reg_d], dtype=U32),
             gate_k=ks, gate_in_off=off.astype(U32), gate_in=ins,
-            gate_tt=np.array([tt for _, tt in self.gates], dtype=np.uint64),
+            gate_tt=np.array([tt & M64 for _, tt in self.gates], dtype=np.uint64),
             po=np.array([nid(p) for p in self.pos], dtype=U32),
-            name=name, meta=meta or {})
+            name=name, meta=meta or {}, gate_tt_hi=hi)
 
 
 # ----------------------------------------------------------------------------
