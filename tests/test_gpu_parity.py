@@ -655,22 +655,24 @@ def _fuzz_netlist(rng, case):
                                  n_po=n_po, max_k=max_k)
 
 
-@pytest.mark.parametrize("case", range(24))
+@pytest.mark.parametrize("case", range(32))
 def test_fuzz_every_kernel_all_lanes_vs_oracle(case):
     """Seeded random netlists through every kernel / schedule / compile option, every lane and
     cycle against the oracle (outputs of the last cycle, registers, per-lane signatures)."""
     rng = np.random.default_rng(1000 + case)
     nl = _fuzz_netlist(rng, case)
-    lanes = int(rng.choice([128, 256, 1024, 4096, 8192]))
+    lanes = int(rng.choice([64, 192, 128, 256, 1024, 4096, 8192]))
+    offset = 64 * int(rng.integers(0, 1000))              # global lane of local lane 0
     cycles = int(rng.integers(1, 12))
     seed = int(rng.integers(0, 2**40))
     balance = bool(rng.integers(0, 2))
     lut_k = int(rng.choice([0, 0, 3, 4, 6, 8]))
     prog = gs.Netlist.from_arrays(nl).compile(balance=balance, lut_k=lut_k)
-    o = oracle.simulate(nl, np.arange(lanes), cycles, seed=seed, want=("last", "regs", "sig"))
-    kernels = ["lut", "poly", "ab", "tile", "auto"] + (["df"] if lanes % 4096 == 0 else [])
+    o = oracle.simulate(nl, np.arange(lanes) + offset, cycles, seed=seed, want=("last", "regs", "sig"))
+    kernels = ["lut", "poly", "ab", "auto"] + (["tile"] if lanes % 128 == 0 else []) + \
+        (["df"] if lanes % 4096 == 0 else [])
     for kernel in kernels:
-        r = run_gpu(nl, lanes, cycles, kernel, seed=seed, prog=prog)
+        r = run_gpu(nl, lanes, cycles, kernel, seed=seed, prog=prog, lane_offset=offset)
         assert np.array_equal(gs.unpack_lanes(r["outputs"]).T, o["last"]), kernel
         assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"]), kernel
         assert np.array_equal(r["sigs"], o["sig"]), kernel
