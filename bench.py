@@ -61,7 +61,7 @@ def parse():
                     help="test only: every rank uses cuda:0 (timings are NOT a scaling measurement)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-roofline", action="store_true")
-    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle CPU time")
+    ap.add_argument("--cpu-seconds", type=float, default=25.0, help="target oracle wall time (calibrated)")
     ap.add_argument("--quick", action="store_true", help="ncu mode: no e2e/cpu/roofline/clocks")
     return ap.parse_args()
 
