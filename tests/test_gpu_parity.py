@@ -705,3 +705,25 @@ def test_aes128_core_every_lane(kernel):
     for s in range(256):
         assert bytes(ct[s]) == _aes_ref.encrypt(bytes(keys[s]), bytes(pts[s]))
     assert r["signature"]["ab_mismatch"] == 0 and r["signature"]["invariant_violations"] == 0
+
+
+@pytest.mark.parametrize("kernel", ["lut", "tile"])
+def test_stimulus_hash_cuda_equals_python_every_word(kernel):
+    """The device counter hash (reading R2) against the independent Python implementation
+    (tests/_ref.py), word by word: primary outputs wired straight to the primary inputs,
+    every word of every cycle recorded by the trace; lane offset != 0."""
+    b = W.Builder()
+    pis = [b.pi() for _ in range(20)]
+    for p in pis:
+        b.out(p)
+    b.out(b.gate(W.NOT, pis[0]))
+    nl = b.build("pi_to_po")
+    lanes, cycles, offset, seed = 2048, 5, 64 * 777, 0xC0FFEE
+    W_ = lanes // 64
+    r = run_gpu(nl, lanes, cycles, kernel, seed=seed, trace_words=list(range(W_)), lane_offset=offset)
+    tr = r["trace"]                                        # [cycle][po][word]
+    words = np.arange(offset // 64, offset // 64 + W_, dtype=np.uint64)
+    for c in range(cycles):
+        for p in range(20):
+            assert np.array_equal(tr[c, p], _ref.stim_words_np(seed, p, c, words)), (c, p)
+        assert np.array_equal(tr[c, 20], ~_ref.stim_words_np(seed, 0, c, words))
