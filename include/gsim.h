@@ -318,7 +318,7 @@ gs_status gs_sim_read_lane_signatures(gs_sim* sim, uint64_t* host, size_t nlanes
 typedef struct {
     uint64_t lane_sig_sum;          /* sum_s mix64(sig_s ^ mix64(s)) mod 2^64 (R6)     */
     uint64_t out_popcount;          /* ones over all outputs, lanes and cycles        */
-    uint64_t ab_mismatch;           /* GS_KERNEL_AB: words where B != A               */
+    uint64_t ab_mismatch;           /* GS_KERNEL_AB: lane-cycles where B != A          */
     uint64_t invariant_violations;  /* kernel B outputs outside {0,1}         */
     uint64_t cycles;                /* cycles stepped since reset                     */
 } gs_signature;

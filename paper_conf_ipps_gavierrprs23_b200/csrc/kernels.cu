@@ -486,99 +486,106 @@ cudaError_t launch_dataflow(const DfArgs& a, uint32_t grid, cudaStream_t s) {
 }
 
 // ------------------------------------------------------------ kernel B: polynomial
-// One warp = one gate x 32 consecutive 32-bit words (1,024 stimuli).  Lane t owns
-// stimulus t of every word b; the words are transposed with shuffles so each lane
-// builds its own input point idx[b] (bit i = x_i), then evaluates the network.
-__global__ void __launch_bounds__(256) k_level_poly(LevelArgs a, uint32_t words32, uint32_t wpg, int check_only) {
-    pdl_entry();
-    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const uint32_t lane = threadIdx.x & 31;
-    const uint32_t gi = warp / wpg;
-    if (gi >= a.ng) return;                                   // warp-uniform
-    const uint32_t chunk = warp - gi * wpg;
-    const uint32_t gate = a.g0 + gi;
-    const uint32_t j = chunk * 32 + lane;                     // this lane's 32-bit word
-    const bool valid = j < words32;
-    const uint4 in = __ldg(a.din + gate);
-    const uint4 au = __ldg(reinterpret_cast<const uint4*>(a.aux) + gate);
-    const uint32_t qdst = au.z, k = au.w & 0xFFu;             // k <= GS_MAX_K_POLY = 8
-    uint32_t r[8] = {in.x, in.y, in.z, in.w, 0u, 0u, 0u, 0u};
-    if (k > 4) {
-        const uint4 hi = __ldg(a.dhi + gate);
-        r[4] = hi.x; r[5] = hi.y; r[6] = hi.z; r[7] = hi.w;
-    }
-    uint32_t x[8];
+// The paper's two-layer network per gate (Fig. 2; Eq. 1-3) in exact integer
+// arithmetic, BIT-SLICED: one thread holds 32 stimuli (one 32-bit word of every input row)
+// and evaluates, for every nonzero monomial S (the sparse polynomial):
+//   hidden neuron  h_S = Theta(sum_{s in S} x_s - |S| + 1): the sum is a 4-plane bit-sliced
+//                  counter of the selected inputs, compared with |S| - 1 (it cannot exceed
+//                  |S|, so "> |S| - 1" is "== |S|");
+//   output neuron  acc += w_S h_S: a two's-complement accumulator of B bit-planes
+//                  (|acc| <= sum |w_S| <= 3^k: B = 8 for k <= 4, 16 for k <= 8), the
+//                  constant w_S added under the mask h_S by a ripple of full adders.
+// The gate's output is [acc == 1]; lanes with acc outside {0, 1} are counted (P:224 says
+// there are none).  check_only: compare with the row kernel A wrote (GS_KERNEL_AB).
+template <int B, int KMAX>
+__device__ __forceinline__ void poly_word(const LevelArgs& a, uint32_t gate, uint32_t j, uint32_t k, uint32_t qdst,
+                                          const uint32_t* r, int check_only, uint32_t& bad) {
+    uint32_t x[KMAX];
 #pragma unroll
-    for (int i = 0; i < 8; ++i) {
-        x[i] = 0u;
-        if (i < (int)k && valid)
-            x[i] = __ldg(reinterpret_cast<const uint32_t*>(a.state + (uint64_t)resolve(r[i], a.qcur) * a.stride) + j);
-    }
-    // idx[b]: input point of stimulus `lane` in word b (bit i = x_i)
-    uint32_t idx[32];
+    for (int i = 0; i < KMAX; ++i)
+        x[i] = i < (int)k ? __ldg(reinterpret_cast<const uint32_t*>(a.state + (uint64_t)resolve(r[i], a.qcur) * a.stride) + j)
+                          : 0u;
+    uint32_t acc[B];
 #pragma unroll
-    for (int b = 0; b < 32; ++b) idx[b] = 0u;
+    for (int b = 0; b < B; ++b) acc[b] = 0u;
+    const uint32_t t0 = __ldg(a.term_off + gate), t1 = __ldg(a.term_off + gate + 1);
+    for (uint32_t ti = t0; ti < t1; ++ti) {
+        const uint32_t tm = __ldg(a.terms + ti);
+        const uint32_t S = tm & 0xFFu;                          // monomial S (bit s <-> x_s)
+        const uint32_t nS = (uint32_t)((int)(int8_t)((tm >> 8) & 0xFFu) + 1);   // |S| (bias + 1, Eq. 3)
+        const int w = (int)(int16_t)(tm >> 16);                 // w_S (Eq. 1)
+        // hidden neuron: bit-sliced sum of the selected inputs, then the threshold
+        uint32_t c0 = 0u, c1 = 0u, c2 = 0u, c3 = 0u;
 #pragma unroll
-    for (int i = 0; i < 8; ++i) {
-        if (i < (int)k) {
-#pragma unroll
-            for (int b = 0; b < 32; ++b) idx[b] |= ((__shfl_sync(FULL, x[i], b) >> lane) & 1u) << i;
-        }
-    }
-    // nonzero terms of this gate (sparse), 32 at a time: lane t holds term base + t
-    const uint32_t t0 = __ldg(a.term_off + gate), nt = __ldg(a.term_off + gate + 1) - t0;
-    int acc[32];
-#pragma unroll
-    for (int b = 0; b < 32; ++b) acc[b] = 0;
-    for (uint32_t base = 0; base < nt; base += 32) {
-        const uint32_t myterm = base + lane < nt ? __ldg(a.terms + t0 + base + lane) : 0u;
-        const uint32_t cnt = min(32u, nt - base);
-        for (uint32_t i = 0; i < cnt; ++i) {
-            const uint32_t tm = __shfl_sync(FULL, myterm, i);
-            const uint32_t S = tm & 0xFFu;                         // monomial S (bit s <-> x_s)
-            const int bias = (int)(int8_t)((tm >> 8) & 0xFFu);     // |S| - 1   (Eq. 3)
-            const int w = (int)(int16_t)(tm >> 16);                // w_S       (Eq. 1)
-#pragma unroll
-            for (int b = 0; b < 32; ++b) {
-                // hidden neuron: Theta(sum_{s in S} x_s - |S| + 1) = [popc(idx & S) > |S| - 1]
-                const int h = __popc(idx[b] & S) > bias ? 1 : 0;
-                acc[b] += w * h;
+        for (int i = 0; i < KMAX; ++i) {
+            if ((S >> i) & 1u) {
+                uint32_t cy = x[i], t;
+                t = c0 & cy; c0 ^= cy; cy = t;
+                t = c1 & cy; c1 ^= cy; cy = t;
+                t = c2 & cy; c2 ^= cy; cy = t;
+                c3 ^= cy;
             }
         }
-    }
-    uint32_t y = 0u, bad = 0u;
+        const uint32_t h = ((nS & 1u) ? c0 : ~c0) & ((nS & 2u) ? c1 : ~c1) & ((nS & 4u) ? c2 : ~c2) &
+                           ((nS & 8u) ? c3 : ~c3);
+        // output neuron: acc += w_S * h_S (two's complement, masked constant add)
+        uint32_t carry = 0u;
 #pragma unroll
-    for (int b = 0; b < 32; ++b) {
-        const uint32_t bal = __ballot_sync(FULL, acc[b] == 1);
-        if (lane == (uint32_t)b) y = bal;
-        bad += (acc[b] != 0 && acc[b] != 1) ? 1u : 0u;
+        for (int b = 0; b < B; ++b) {
+            const uint32_t add = ((w >> b) & 1) ? h : 0u;
+            const uint32_t sum = acc[b] ^ add ^ carry;
+            carry = (acc[b] & add) | (carry & (acc[b] ^ add));
+            acc[b] = sum;
+        }
     }
-    // counts only the stimuli this warp really owns
-    if (!valid) bad = 0u;
+    uint32_t hi = 0u;
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) bad += __shfl_xor_sync(FULL, bad, o);
-    if (lane == 0 && bad) atomicAdd(&a.ctl->violations, (unsigned long long)bad);
-    if (!valid) return;
+    for (int b = 1; b < B; ++b) hi |= acc[b];
+    const uint32_t one = acc[0] & ~hi, zero = ~(acc[0] | hi);
+    bad += __popc(~(one | zero));
     uint32_t* out = reinterpret_cast<uint32_t*>(a.state + (uint64_t)(a.row_gate0 + gate) * a.stride) + j;
     if (check_only) {
         const uint32_t ref = *out;
-        const uint32_t mism = __ballot_sync(__activemask(), ref != y);
-        if (mism && lane == __ffs(__activemask()) - 1) atomicAdd(&a.ctl->ab_mismatch, (unsigned long long)__popc(mism));
+        if (ref != one) atomicAdd(&a.ctl->ab_mismatch, (unsigned long long)__popc(ref ^ one));
     } else {
-        *out = y;
-        if (qdst != 0xFFFFFFFFu)
-            reinterpret_cast<uint32_t*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride)[j] = y;
+        *out = one;
+        if (qdst != 0xFFFFFFFFu) reinterpret_cast<uint32_t*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride)[j] = one;
     }
+}
+
+// one thread = one gate x one 32-bit word (32 stimuli); consecutive threads = consecutive
+// words of the same gate (coalesced loads, warp-uniform terms)
+__global__ void __launch_bounds__(256) k_level_poly(LevelArgs a, uint32_t words32, int check_only) {
+    pdl_entry();
+    const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint32_t gi = (uint32_t)(t / words32), j = (uint32_t)(t - (uint64_t)gi * words32);
+    uint32_t bad = 0u;
+    if (gi < a.ng) {
+        const uint32_t gate = a.g0 + gi;
+        const uint4 in = __ldg(a.din + gate);
+        const uint4 au = __ldg(reinterpret_cast<const uint4*>(a.aux) + gate);
+        const uint32_t qdst = au.z, k = au.w & 0xFFu;          // k <= GS_MAX_K_POLY = 8
+        uint32_t r[8] = {in.x, in.y, in.z, in.w, 0u, 0u, 0u, 0u};
+        if (k > 4) {
+            const uint4 hi = __ldg(a.dhi + gate);
+            r[4] = hi.x; r[5] = hi.y; r[6] = hi.z; r[7] = hi.w;
+            poly_word<16, 8>(a, gate, j, k, qdst, r, check_only, bad);
+        } else {
+            poly_word<8, 4>(a, gate, j, k, qdst, r, check_only, bad);
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) bad += __shfl_xor_sync(FULL, bad, o);
+    if ((threadIdx.x & 31) == 0 && bad) atomicAdd(&a.ctl->violations, (unsigned long long)bad);
 }
 
 cudaError_t launch_level_poly(const LevelArgs& a, int check_only, cudaStream_t s) {
     if (a.ng == 0) return cudaSuccess;
     const uint32_t words32 = a.words * 2;
-    const uint32_t wpg = (words32 + 31) / 32;
-    const uint64_t warps = (uint64_t)a.ng * wpg;
-    if (warps * 32 >= (1ull << 31)) return cudaErrorInvalidValue;
-    const uint32_t blocks = (uint32_t)((warps * 32 + 255) / 256);
-    return launch_k(k_level_poly, blocks, s, a.pdl, a, words32, wpg, check_only);
+    const uint64_t threads = (uint64_t)a.ng * words32;
+    const uint64_t blocks = (threads + 255) / 256;
+    if (blocks >= (1ull << 31)) return cudaErrorInvalidValue;
+    return launch_k(k_level_poly, (uint32_t)blocks, s, a.pdl, a, words32, check_only);
 }
 
 // --------------------------------------------------------------------- stimulus
