@@ -192,6 +192,13 @@ gs_status gs_program_coeffs(const gs_program* prog, uint32_t gate, int32_t* w, u
  * Without lut_k this is the gate as added; absorbed gates report k = 0. */
 gs_status gs_program_gate_lut(const gs_program* prog, uint32_t gate, uint32_t* k, gs_net* in, uint64_t* tt);
 
+/* Persist / restore a compiled program (the paper's saved network model, Fig. 1):
+ * a binary file of every table the simulator uses plus the query tables; loading checks the
+ * format and the program hash (GS_ERR_ARG on a foreign, truncated or edited file).  The
+ * loaded program behaves exactly like the one saved (same program_hash). */
+gs_status gs_program_save(const gs_program* prog, const char* path);
+gs_status gs_program_load(const char* path, gs_program** out);
+
 /* Shared-memory slots one lane tile of kernel T needs (constants, PIs, two register banks,
  * gate values reused by live range; tile.cpp).  A tile of 32*w lanes needs
  * (slots + 64) * 4 * w bytes of shared memory (<= 227 KB). */

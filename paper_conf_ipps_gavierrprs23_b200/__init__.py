@@ -115,6 +115,8 @@ _SIGS = {
     "gs_program_gate_levels": (C.c_int32, [_P, _P, C.c_uint32]),
     "gs_program_coeffs": (C.c_int32, [_P, C.c_uint32, _P, C.c_uint32]),
     "gs_program_tile_slots": (C.c_int32, [_P, _P]),
+    "gs_program_save": (C.c_int32, [_P, C.c_char_p]),
+    "gs_program_load": (C.c_int32, [C.c_char_p, _P]),
     "gs_program_gate_lut": (C.c_int32, [_P, C.c_uint32, _P, _P, _P]),
     "gs_sim_workspace_bytes": (C.c_int32, [_P, _P, _P]),
     "gs_sim_create": (C.c_int32, [_P, _P, _P, C.c_size_t, _P]),
@@ -247,14 +249,27 @@ class Netlist:
 
 
 class Program:
-    def __init__(self, netlist: Netlist, balance: bool = True, max_k: int = 0, lut_k: int = 0):
-        h = C.c_void_p()
-        o = gs_compile_opts(1 if balance else 0, max_k, lut_k)
-        _call("gs_compile", netlist.h, C.byref(o), C.byref(h))
+    def __init__(self, netlist: Netlist | None, balance: bool = True, max_k: int = 0, lut_k: int = 0,
+                 _handle=None):
+        if _handle is None:
+            h = C.c_void_p()
+            o = gs_compile_opts(1 if balance else 0, max_k, lut_k)
+            _call("gs_compile", netlist.h, C.byref(o), C.byref(h))
+        else:
+            h = _handle
         self.h = h
         inf = gs_program_info()
         _call("gs_program_get_info", self.h, C.byref(inf))
         self.info = inf.as_dict()
+
+    def save(self, path: str) -> None:
+        _call("gs_program_save", self.h, os.fsencode(path))
+
+    @classmethod
+    def load(cls, path: str) -> "Program":
+        h = C.c_void_p()
+        _call("gs_program_load", os.fsencode(path), C.byref(h))
+        return cls(None, _handle=h)
 
     def __del__(self):
         if getattr(self, "h", None) and _lib is not None:

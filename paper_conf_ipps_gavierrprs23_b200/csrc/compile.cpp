@@ -38,6 +38,23 @@ static inline uint64_t hmix(uint64_t h, uint64_t v) {
     return h * 0xff51afd7ed558ccdULL;
 }
 
+// Hash of everything the device evaluates (multi-rank consistency, program files): rows,
+// levels, descriptors, tables, terms, register and output maps.
+uint64_t program_hash(const Program& pr) {
+    uint64_t h = hmix(0, pr.n_rows);
+    h = hmix(h, ((uint64_t)pr.n_pi << 32) | pr.n_reg);
+    for (uint32_t v : pr.level_off) h = hmix(h, v);
+    for (uint32_t v : pr.in_lo) h = hmix(h, v);
+    for (uint32_t v : pr.in_hi) h = hmix(h, v);
+    for (uint64_t v : pr.tt_full) h = hmix(h, v);
+    for (const GateAux& a : pr.aux) h = hmix(hmix(h, a.tt), ((uint64_t)a.qdst << 32) | a.k);
+    for (uint32_t v : pr.terms) h = hmix(h, v);
+    for (uint32_t v : pr.po_rows) h = hmix(h, v);
+    for (size_t i = 0; i < pr.latch_src.size(); ++i) h = hmix(h, ((uint64_t)pr.latch_src[i] << 32) | pr.latch_dst[i]);
+    for (uint8_t v : pr.reg_init) h = hmix(h, v);
+    return h;
+}
+
 gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out) {
     const uint32_t N = nl.n_nets();
     const uint32_t P = (uint32_t)nl.pi_net.size();
@@ -297,17 +314,7 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
     in.nnz_coeffs = nnz;
     in.hidden_neurons = hidden;
     in.n_rows = pr.n_rows;
-    uint64_t h = hmix(0, pr.n_rows);
-    h = hmix(h, ((uint64_t)P << 32) | R);
-    for (uint32_t v : pr.level_off) h = hmix(h, v);
-    for (uint32_t v : pr.in_lo) h = hmix(h, v);
-    for (uint32_t v : pr.in_hi) h = hmix(h, v);
-    for (uint64_t v : nl.gate_tt_hi) h = hmix(h, v);
-    for (const GateAux& a : pr.aux) h = hmix(hmix(h, a.tt), ((uint64_t)a.qdst << 32) | a.k);
-    for (uint32_t v : pr.po_rows) h = hmix(h, v);
-    for (size_t i = 0; i < pr.latch_src.size(); ++i) h = hmix(h, ((uint64_t)pr.latch_src[i] << 32) | pr.latch_dst[i]);
-    for (uint8_t v : pr.reg_init) h = hmix(h, v);
-    in.program_hash = h;
+    in.program_hash = program_hash(pr);
     out = p;
     return GS_OK;
 }

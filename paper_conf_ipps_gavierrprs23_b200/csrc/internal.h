@@ -98,6 +98,7 @@ struct Program {
 };
 
 gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out);
+uint64_t program_hash(const Program& p);
 
 // Cone collapsing into LUTs of <= L inputs (collapse.cpp; the paper's LUT mapping)
 gs_status collapse_luts(const Netlist& nl, uint32_t L, Netlist& out);

@@ -266,6 +266,21 @@ def test_negative_flipped_truth_table_bit_is_detected():
     assert np.array_equal(r["sigs"], ob["sig"])
 
 
+def test_loaded_program_simulates_identically(tmp_path):
+    """A program saved to a file and loaded back runs bit-identically (kernels A and T)."""
+    cfg = workloads.CONFIGS["C3"]
+    nl = cfg.netlist()
+    prog = compile_nl(nl)
+    f = str(tmp_path / "c3.gsp")
+    prog.save(f)
+    loaded = gs.Program.load(f)
+    for kernel in ("lut", "auto"):
+        a = run_gpu(nl, 4096, 15, kernel, seed=3, prog=prog)
+        b = run_gpu(nl, 4096, 15, kernel, seed=3, prog=loaded)
+        for key in ("outputs", "regs", "sigs"):
+            assert np.array_equal(a[key], b[key]), (kernel, key)
+
+
 def test_errors_on_device():
     prog = compile_nl(workloads.adder(8))
     sim = gs.Sim(prog, 128)

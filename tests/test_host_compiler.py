@@ -240,3 +240,34 @@ def test_permuted_netlist_same_asap_widths():
     a = _compile(nl, balance=False).level_widths()
     b = _compile(nl.permuted(3), balance=False).level_widths()
     assert np.array_equal(a, b)
+
+
+def test_program_save_load_round_trip(tmp_path):
+    """gs_program_save / gs_program_load: same hash, info, levels, coefficients and LUTs;
+    foreign and truncated files are rejected."""
+    for nl, L in ((workloads.build_netlist("C3"), 0), (workloads.random_tiny(5, max_k=8, n_gates=80), 0),
+                  (workloads.adder(8), 4)):
+        p = gs.Netlist.from_arrays(nl).compile(lut_k=L)
+        f = str(tmp_path / f"{nl.name}.gsp")
+        p.save(f)
+        q = gs.Program.load(f)
+        assert q.info == p.info
+        assert np.array_equal(q.level_widths(), p.level_widths())
+        assert np.array_equal(q.gate_levels(), p.gate_levels())
+        for g in range(0, nl.n_gates, max(1, nl.n_gates // 50)):
+            k = len(p.gate_lut(g)[0])
+            assert q.coeffs(g, k) == p.coeffs(g, k) and q.gate_lut(g) == p.gate_lut(g)
+    bad = tmp_path / "bad.gsp"
+    bad.write_bytes(b"not a program")
+    with pytest.raises(gs.GsError):
+        gs.Program.load(str(bad))
+    data = open(f, "rb").read()
+    (tmp_path / "trunc.gsp").write_bytes(data[:len(data) // 2])
+    with pytest.raises(gs.GsError):
+        gs.Program.load(str(tmp_path / "trunc.gsp"))
+    for pos in (20, len(data) // 3, len(data) // 2, len(data) - 20):   # any edited byte
+        flipped = bytearray(data)
+        flipped[pos] ^= 0x5A
+        (tmp_path / "flip.gsp").write_bytes(bytes(flipped))
+        with pytest.raises(gs.GsError):
+            gs.Program.load(str(tmp_path / "flip.gsp"))
