@@ -84,7 +84,6 @@ __device__ __forceinline__ void tile_gate(uint4* sl, uint32_t V, uint32_t v, con
 #pragma unroll
     for (int i = 0; i < K; ++i) {
         uint32_t si = s[i];
-        if (HASQ) si += (si - q0) < R ? qcur : 0u;
         x[i] = sl[(size_t)si * V + v];
     }
     uint4 y;
@@ -178,9 +177,12 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
             sw[u] = 0u;
             sw[TW + u] = 0xFFFFFFFFu;
         }
+        // register slots: bank 0 always holds the CURRENT Q (state bank c0 & 1), bank 1 the
+        // next one; inputs never resolve banks — bank 1 is copied into bank 0 after each cycle
         for (uint32_t u = tid; u < 2 * R * TW; u += bd) {
             const uint32_t r = u / TW, w = u % TW;
-            sw[(size_t)(q0 + r) * TW + w] = st32[(uint64_t)(a.row_q0 + r) * w32_row + t0 + w];
+            const uint32_t sb = (r < R ? (uint32_t)(c0 & 1) : (uint32_t)((c0 + 1) & 1)) * R + (r < R ? r : r - R);
+            sw[(size_t)(q0 + r) * TW + w] = st32[(uint64_t)(a.row_q0 + sb) * w32_row + t0 + w];
         }
         for (uint32_t u = tid; u < 64 * TW; u += bd) {
             const uint32_t j = u / TW, w = u % TW;
@@ -189,7 +191,8 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
         group_sync(bar, GT);
         for (uint32_t c = 0; c < a.ncycles; ++c) {
             const unsigned long long cyc = c0 + c;
-            const uint32_t qcur = (cyc & 1) ? R : 0u, qnext = R - qcur;
+            constexpr uint32_t qcur = 0u;
+            const uint32_t qnext = R;
             // ---- primary inputs of this cycle (R2): one 64-bit hash per pair of words
             for (uint32_t u = tid; u < a.n_pi * (TW / 2); u += bd) {
                 const uint32_t p = u / (TW / 2), w2 = u % (TW / 2);
@@ -239,8 +242,7 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
             // ---- leftover latches into the next bank; MISR / popcount / trace of the POs
             for (uint32_t u = tid; u < a.n_latch * V; u += bd) {
                 const uint32_t e = u / V, v = u % V;
-                uint32_t s = __ldg(a.latch_src + e);
-                s += (s - q0) < R ? qcur : 0u;
+                const uint32_t s = __ldg(a.latch_src + e);
                 sl[(size_t)(q0 + __ldg(a.latch_dst + e) + qnext) * V + v] = sl[(size_t)s * V + v];
             }
             constexpr uint32_t NP = (64 * TW + GT - 1) / GT;    // MISR plane words per thread
@@ -259,9 +261,7 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
                            (cyc - a.ctl->sink_base) * a.n_po * (uint64_t)w32_row;
                 uint32_t vv = 0;
                 for (uint32_t o = j; o < a.n_po; o += 64) {
-                    uint32_t s = __ldg(a.po_slot + o);
-                    s += (s - q0) < R ? qcur : 0u;
-                    const uint32_t x = sw[(size_t)s * TW + w];
+                    const uint32_t x = sw[(size_t)__ldg(a.po_slot + o) * TW + w];
                     vv ^= x;
                     pop += __popc(x);
                     if (tslot >= 0)
@@ -277,12 +277,17 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
 #pragma unroll
             for (uint32_t i = 0; i < NP; ++i)
                 if (tid + i * bd < 64 * TW) mp[tid + i * bd] = newp[i];
+            if (HASQ && c + 1 < a.ncycles)                    // the clock edge: Q := next Q
+                for (uint32_t u = tid; u < R * V; u += bd) sl[(size_t)q0 * V + u] = sl[(size_t)(q0 + R) * V + u];
             group_sync(bar, GT);
         }
-        // ---- write back: both register banks, PO rows (read_outputs), MISR planes
+        // ---- write back: Q of the last cycle (bank 0) to state bank (last & 1), the latched
+        // next Q (bank 1) to the other bank; PO rows (read_outputs); MISR planes
+        const uint32_t lastp = (uint32_t)((c0 + a.ncycles - 1) & 1);
         for (uint32_t u = tid; u < 2 * R * TW; u += bd) {
             const uint32_t r = u / TW, w = u % TW;
-            st32w[(uint64_t)(a.row_q0 + r) * w32_row + t0 + w] = sw[(size_t)(q0 + r) * TW + w];
+            const uint32_t sb = (r < R ? lastp : lastp ^ 1u) * R + (r < R ? r : r - R);
+            st32w[(uint64_t)(a.row_q0 + sb) * w32_row + t0 + w] = sw[(size_t)(q0 + r) * TW + w];
         }
         for (uint32_t u = tid; u < a.n_wb * TW; u += bd) {
             const uint32_t e = u / TW, w = u % TW;
