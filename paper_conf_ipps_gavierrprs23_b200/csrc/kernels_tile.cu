@@ -27,6 +27,7 @@ cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_ev
         case 8: e = tile_setup_tw<8>(ng, smem, desc_smem, has_q, &per); break;
         case 16: e = tile_setup_tw<16>(ng, smem, desc_smem, has_q, &per); break;
         case 32: e = tile_setup_tw<32>(ng, smem, desc_smem, has_q, &per); break;
+        case 64: e = tile_setup_tw<64>(ng, smem, desc_smem, has_q, &per); break;
         default: return cudaErrorInvalidValue;
     }
     *per_sm = (uint32_t)per;
@@ -41,6 +42,7 @@ cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t gr
         case 8: return launch_tile_tw<8>(a, ng, grid, smem, s);
         case 16: return launch_tile_tw<16>(a, ng, grid, smem, s);
         case 32: return launch_tile_tw<32>(a, ng, grid, smem, s);
+        case 64: return launch_tile_tw<64>(a, ng, grid, smem, s);
         default: return cudaErrorInvalidValue;
     }
 }

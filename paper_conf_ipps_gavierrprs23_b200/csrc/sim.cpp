@@ -92,8 +92,9 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
     };
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, o.device);
-    if (o.tile_words && (o.tile_words != 4 && o.tile_words != 8 && o.tile_words != 16 && o.tile_words != 32))
-        return fail(GS_ERR_ARG, "TILE: tile_words must be 4, 8, 16 or 32");
+    if (o.tile_words && (o.tile_words != 4 && o.tile_words != 8 && o.tile_words != 16 && o.tile_words != 32 &&
+                         o.tile_words != 64))
+        return fail(GS_ERR_ARG, "TILE: tile_words must be 4, 8, 16, 32 or 64");
     if (o.tile_groups && (o.tile_groups != 1 && o.tile_groups != 2 && o.tile_groups != 4))
         return fail(GS_ERR_ARG, "TILE: tile_groups must be 1, 2 or 4");
     if (o.tile_words && o.lanes % (32ull * o.tile_words))
@@ -110,7 +111,7 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
         if (forced >= 0 && ds != forced) continue;
         for (uint32_t ng : {4u, 2u, 1u}) {
             if (o.tile_groups && ng != o.tile_groups) continue;
-            for (uint32_t tw : {4u, 8u, 16u, 32u}) {
+            for (uint32_t tw : {4u, 8u, 16u, 32u, 64u}) {
                 if (o.tile_words && tw != o.tile_words) continue;
                 if (o.lanes % (32ull * tw) || smem(tw, ng, ds) > TILE_SMEM_MAX) continue;
                 const uint64_t inflight = std::min<uint64_t>((uint64_t)ng * tw * 32 * sms, o.lanes);
