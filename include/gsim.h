@@ -245,7 +245,7 @@ typedef struct {
     uint32_t df_gates_per_warp;   /* DATAFLOW: gates per warp per work item, 1..32 (0 = 8) */
     uint32_t flags;               /* GS_SIM_* bits below                                   */
     uint32_t tile_words;          /* TILE: 32-bit words per slot, lanes per tile = 32 * this
-                                     (4, 8, 16 or 32; 0 = auto); lanes % (32 * it) == 0   */
+                                     (4, 8, 16, 32 or 64; 0 = auto); lanes % (32 * it) == 0 */
     uint32_t tile_groups;         /* TILE: independent thread groups (tiles) per 512-thread
                                      CTA, each with its own barrier (1, 2 or 4; 0 = auto)  */
 } gs_sim_opts;
