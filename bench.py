@@ -54,6 +54,8 @@ def parse():
     ap.add_argument("--no-pdl", action="store_true", help="disable programmatic dependent launch")
     ap.add_argument("--no-grid-stride", action="store_true", help="kernel A: one CTA per work chunk")
     ap.add_argument("--l2-hints", type=int, default=0, help="kernel A L2 hints: 0 off, 1 stores, 2 +loads")
+    ap.add_argument("--lut-bulk", default="auto", choices=["auto", "on", "off"],
+                    help="kernel A bulk-copy staged gathers (auto = library default: off)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend (gloo + --same-device: multi-rank test on one GPU)")
@@ -246,7 +248,8 @@ def main():
                  df_interleave=args.df_interleave, df_gates_per_warp=args.df_gpw, pdl=not args.no_pdl,
                  tile_words=args.tile_words, tile_groups=args.tile_groups,
                  flags=(2 if args.l2_hints >= 1 else 0) | (4 if args.l2_hints >= 2 else 0) |
-                 (8 if args.no_grid_stride else 0))
+                 (8 if args.no_grid_stride else 0) |
+                 {"auto": 0, "on": 64, "off": 128}[args.lut_bulk])
     sim.bind_generated(cfg.stim_seed)
     C = args.cycles_per_step
     launches_per_cycle = sim.launches_per_cycle()

@@ -265,6 +265,12 @@ typedef struct {
  * shared memory if the whole table fits, else the TMA stream, else global. */
 #define GS_SIM_TILE_DESC_GLOBAL 16u
 #define GS_SIM_TILE_DESC_TMA 32u
+/* flags (kernel A): gather a level's input rows with bulk copies (cp.async.bulk, whole-row
+ * chunks of 2-8 KB staged in a shared-memory ring by a producer warp) on every
+ * level whose gates all have 1 <= k <= 4 and whose rows are 2, 4 or 8 KB x a power of two;
+ * or never.  Default: never (measured slower than the register gathers on C3-C5). */
+#define GS_SIM_LUT_BULK 64u
+#define GS_SIM_LUT_NO_BULK 128u
 
 /* Device workspace bytes required for (prog, opts). */
 gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts, size_t* bytes);

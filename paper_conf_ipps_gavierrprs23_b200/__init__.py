@@ -26,6 +26,8 @@ GS_ERR_BUFFER_TOO_SMALL, GS_ERR_CUDA, GS_ERR_STATE, GS_ERR_NOMEM = -5, -6, -7, -
 GS_MAX_K = 6
 GS_MAX_K_POLY = 8
 GS_SIM_NO_PDL = 1
+GS_SIM_LUT_BULK = 64          # kernel A: bulk-copy staged gathers on (where eligible)
+GS_SIM_LUT_NO_BULK = 128      # ... off
 GS_KERNEL_AUTO, GS_KERNEL_LUT, GS_KERNEL_POLY, GS_KERNEL_AB, GS_KERNEL_DATAFLOW = 0, 1, 2, 3, 4
 GS_KERNEL_TILE = 5
 KERNELS = {"auto": 0, "lut": 1, "A": 1, "poly": 2, "B": 2, "ab": 3, "AB": 3, "df": 4, "dataflow": 4,

@@ -46,6 +46,8 @@ struct LevelArgs {
     uint32_t hint;                    // L2 eviction-priority stores (aux.k bit 8 = read next level)
     uint32_t hint_ld;                 // ... and evict_first input loads
     uint32_t grid_blocks;             // wide path: cap the grid at the resident capacity (0 = off)
+    uint32_t bulk;                    // gather input rows with bulk copies (k_level_bulk)
+    uint32_t sms;                     // multiprocessors of the device
 };
 
 struct EndArgs {
@@ -128,6 +130,10 @@ cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_ev
 cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s);
 
 cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s);
+// kernel A with bulk-copy staged gathers: chunk bytes used for rows of `words` 64-bit words
+// (slab of vslab 16-byte vectors when nonzero), 0 = rows not eligible
+uint32_t level_bulk_chunk(uint32_t words, uint32_t vslab);
+cudaError_t launch_level_bulk(const LevelArgs& a, cudaStream_t s);
 uint32_t level_lut_resident_blocks(int device);   // CTAs of k_level_lut_wide resident on the GPU
 cudaError_t launch_dataflow(const DfArgs& a, uint32_t grid, cudaStream_t s);
 cudaError_t dataflow_grid(uint32_t slab_vec, int device, uint32_t* grid);

@@ -228,6 +228,9 @@ struct gs_sim {
     uint32_t min_warps = 0;           // kernel A auto-U threshold (2 waves of resident warps)
     uint32_t resident_blocks = 0;     // kernel A wide path: CTAs resident on the GPU
     uint32_t grid_waves = 1;          // grid-stride grid = resident_blocks x this
+    uint32_t sms = 148;
+    bool bulk = false;                // kernel A: bulk-copy staged gathers (k_level_bulk)
+    std::vector<uint8_t> lv_bulk;     // [n_levels] every gate of the level has 1 <= k <= 4
 
     Ctl* ctl() const { return reinterpret_cast<Ctl*>(ws + L.ctl); }
     uint8_t* state() const { return ws + L.state; }
@@ -264,6 +267,8 @@ static LevelArgs level_args(const gs_sim* s, uint32_t l, uint32_t parity) {
     a.hint = (s->opts.flags & GS_SIM_L2_HINTS) ? 1u : 0u;
     a.hint_ld = (s->opts.flags & GS_SIM_L2_HINT_LOADS) ? 1u : 0u;
     a.grid_blocks = (s->opts.flags & GS_SIM_NO_GRID_STRIDE) ? 0u : s->resident_blocks * s->grid_waves;
+    a.bulk = (s->bulk && s->lv_bulk[l]) ? 1u : 0u;
+    a.sms = s->sms;
     return a;
 }
 
@@ -496,6 +501,17 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, opts->device);
         s->min_warps = (uint32_t)sms * 32u * 2u;   // 4 CTAs x 8 warps per SM, two waves
         s->resident_blocks = level_lut_resident_blocks(opts->device);
+        s->sms = (uint32_t)sms;
+    }
+    {
+        // bulk-copy gathers: opt-in (measured slower than the register gathers)
+        s->bulk = (opts->flags & GS_SIM_LUT_BULK) && !(opts->flags & GS_SIM_LUT_NO_BULK);
+        s->lv_bulk.assign(p.n_levels, 1);
+        for (uint32_t l = 0; l < p.n_levels; ++l)
+            for (uint32_t g = p.level_off[l]; g < p.level_off[l + 1]; ++g) {
+                const uint32_t k = p.aux[g].k & 0xFFu;
+                if (k < 1 || k > 4) s->lv_bulk[l] = 0;
+            }
     }
     s->slabs = (opts->lane_slabs && s->opts.kernel != GS_KERNEL_DATAFLOW) ? opts->lane_slabs : 1;
     if (s->slabs > 1) {

@@ -322,6 +322,46 @@ def test_launch_and_cache_options_do_not_change_results(flags):
         assert np.array_equal(a[key], b[key]), key
 
 
+# ------------------------------------------------------------------ kernel A, bulk-copy gathers
+@pytest.mark.parametrize("lanes", [16384, 32768, 65536])      # 2 / 4 / 8 KB rows: every chunk size
+@pytest.mark.parametrize("kernel", ["lut", "ab"])
+def test_lut_bulk_gathers_every_lane_vs_oracle(lanes, kernel):
+    """Kernel A with the bulk-copy staged gathers forced on (producer warp, mbarrier ring):
+    a sequential synthetic netlist (fused latches, Q-bank inputs), every lane vs the oracle,
+    and bit-identical to the register-gather path."""
+    nl = workloads.synthetic(3000, 120, 20, 32, 16, seed=21, name="bulk")
+    prog = compile_nl(nl)
+    cycles = 7
+    r = run_gpu(nl, lanes, cycles, kernel, seed=9, prog=prog, flags=gs.GS_SIM_LUT_BULK)
+    o = oracle.simulate(nl, np.arange(lanes), cycles, seed=9, want=("last", "regs", "sig"))
+    assert np.array_equal(gs.unpack_lanes(r["outputs"]).T, o["last"])
+    assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"])
+    assert np.array_equal(r["sigs"], o["sig"])
+    assert r["signature"]["ab_mismatch"] == 0 and r["signature"]["invariant_violations"] == 0
+    b = run_gpu(nl, lanes, cycles, kernel, seed=9, prog=prog, flags=gs.GS_SIM_LUT_NO_BULK)
+    for key in ("outputs", "regs", "sigs"):
+        assert np.array_equal(r[key], b[key]), key
+
+
+@pytest.mark.parametrize("case", range(4))
+def test_lut_bulk_mixed_fanin_slabs_and_offsets(case):
+    """Bulk gathers on programs whose levels mix k = 0..6 (levels with k > 4 fall back to the
+    register path inside the same cycle), with lane slabs and a nonzero lane offset."""
+    rng = np.random.default_rng(500 + case)
+    nl = _fuzz_netlist(rng, case)
+    lanes = [16384, 32768, 65536, 16384][case]
+    slabs = [0, 2, 4, 0][case]
+    offset = 64 * int(rng.integers(0, 1000))
+    cycles = int(rng.integers(2, 9))
+    prog = gs.Netlist.from_arrays(nl).compile(lut_k=[0, 4, 0, 3][case])
+    o = oracle.simulate(nl, np.arange(lanes) + offset, cycles, seed=case, want=("last", "regs", "sig"))
+    r = run_gpu(nl, lanes, cycles, "lut", seed=case, prog=prog, lane_offset=offset, lane_slabs=slabs,
+                flags=gs.GS_SIM_LUT_BULK)
+    assert np.array_equal(gs.unpack_lanes(r["outputs"]).T, o["last"])
+    assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"])
+    assert np.array_equal(r["sigs"], o["sig"])
+
+
 # ------------------------------------------------------------------ cone collapsing (lut_k)
 @pytest.mark.parametrize("L", [3, 6])
 @pytest.mark.parametrize("kernel", ["lut", "poly", "ab", "tile"])
