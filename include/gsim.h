@@ -248,6 +248,12 @@ typedef struct {
                                      (4, 8, 16, 32 or 64; 0 = auto); lanes % (32 * it) == 0 */
     uint32_t tile_groups;         /* TILE: independent thread groups (tiles) per 512-thread
                                      CTA, each with its own barrier (1, 2 or 4; 0 = auto)  */
+    uint32_t lane_groups;         /* LUT: cut the lanes into this many groups whose level
+                                     chains run CONCURRENTLY every cycle (parallel branches of
+                                     the cycle's CUDA graph / streams), so one group's level
+                                     ramp and drain overlap another's levels.  Needs
+                                     (lanes/128) % groups == 0 and >= 4096 lanes per group.
+                                     0 = auto, 1 = off.                      */
 } gs_sim_opts;
 /* flags: launch the per-cycle kernels WITHOUT programmatic dependent launch (by default a
  * level kernel may become resident while its predecessor drains; A/B measurement only). */
@@ -315,6 +321,9 @@ gs_status gs_sim_sync(gs_sim* sim);
 gs_status gs_sim_run_streamed(gs_sim* sim, const uint64_t* host_stim, uint64_t* host_out, uint32_t ncycles,
                               uint32_t chunk);
 gs_status gs_sim_get_cycle(const gs_sim* sim, uint64_t* cycle);
+/* The resolved launch configuration: kernel (GS_KERNEL_*, AUTO resolved) and the number of
+ * concurrent lane groups (1 = a single level chain per cycle). */
+gs_status gs_sim_get_config(const gs_sim* sim, int* kernel, uint32_t* lane_groups);
 
 /* Readback (synchronous).  Layouts, with W = lanes/64 local words:
  *   outputs   [po][W]  outputs of the last stepped cycle (before its latch, R4)

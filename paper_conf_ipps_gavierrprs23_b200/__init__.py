@@ -77,7 +77,8 @@ class gs_sim_opts(C.Structure):
                 ("trace_words", C.c_void_p), ("trace_cycles", C.c_uint32), ("use_graphs", C.c_int),
                 ("lane_slabs", C.c_uint32), ("lut_unroll", C.c_uint32),
                 ("df_interleave", C.c_uint32), ("df_gates_per_warp", C.c_uint32),
-                ("flags", C.c_uint32), ("tile_words", C.c_uint32), ("tile_groups", C.c_uint32)]
+                ("flags", C.c_uint32), ("tile_words", C.c_uint32), ("tile_groups", C.c_uint32),
+                ("lane_groups", C.c_uint32)]
 
 
 class gs_signature(C.Structure):
@@ -131,6 +132,7 @@ _SIGS = {
     "gs_sim_sync": (C.c_int32, [_P]),
     "gs_sim_run_streamed": (C.c_int32, [_P, _P, _P, C.c_uint32, C.c_uint32]),
     "gs_sim_get_cycle": (C.c_int32, [_P, _P]),
+    "gs_sim_get_config": (C.c_int32, [_P, _P, _P]),
     "gs_sim_read_outputs": (C.c_int32, [_P, _P, C.c_size_t]),
     "gs_sim_read_registers": (C.c_int32, [_P, _P, C.c_size_t]),
     "gs_sim_write_registers": (C.c_int32, [_P, _P, C.c_size_t]),
@@ -314,7 +316,7 @@ class Sim:
                  device: int = 0, stream=None, trace_words=(), trace_cycles: int = 0,
                  use_graphs: bool = True, lane_slabs: int = 0, lut_unroll: int = 0,
                  df_interleave: int = 0, df_gates_per_warp: int = 0, pdl: bool = True,
-                 tile_words: int = 0, tile_groups: int = 0, flags: int = 0):
+                 tile_words: int = 0, tile_groups: int = 0, flags: int = 0, lane_groups: int = 0):
         import torch
         self.program = program
         self.lanes, self.words = int(lanes), int(lanes) // 64
@@ -326,7 +328,8 @@ class Sim:
                         _p(self._tw) if len(self._tw) else None, int(trace_cycles),
                         1 if use_graphs else 0, int(lane_slabs), int(lut_unroll),
                         int(df_interleave), int(df_gates_per_warp),
-                        (0 if pdl else GS_SIM_NO_PDL) | int(flags), int(tile_words), int(tile_groups))
+                        (0 if pdl else GS_SIM_NO_PDL) | int(flags), int(tile_words), int(tile_groups),
+                        int(lane_groups))
         nbytes = C.c_size_t()
         _call("gs_sim_workspace_bytes", program.h, C.byref(o), C.byref(nbytes))
         self.workspace = torch.empty(int(nbytes.value) + 256, dtype=torch.uint8, device=self.device)
@@ -380,6 +383,13 @@ class Sim:
             assert out.dtype == np.uint64 and out.flags.c_contiguous and out.shape == (stim.shape[0], self.n_po, self.words)
         self._stim_keep = (stim, out)
         _call("gs_sim_run_streamed", self.h, _p(stim), _p(out), int(stim.shape[0]), int(chunk))
+
+    @property
+    def config(self) -> dict:
+        """Resolved launch configuration: {'kernel': GS_KERNEL_*, 'lane_groups': G}."""
+        k, g = C.c_int32(), C.c_uint32()
+        _call("gs_sim_get_config", self.h, C.byref(k), C.byref(g))
+        return {"kernel": k.value, "lane_groups": g.value}
 
     @property
     def cycle(self) -> int:

@@ -230,6 +230,9 @@ struct gs_sim {
     uint32_t grid_waves = 1;          // grid-stride grid = resident_blocks x this
     uint32_t sms = 148;
     bool bulk = false;                // kernel A: bulk-copy staged gathers (k_level_bulk)
+    bool concurrent = false;          // lane groups: the slabs' level chains run concurrently
+    std::vector<cudaStream_t> gstream;  // [slabs - 1] branch streams (group 0: the caller's)
+    std::vector<cudaEvent_t> gev;       // [0] fork, [1 .. slabs - 1] joins
     std::vector<uint8_t> lv_bulk;     // [n_levels] every gate of the level has 1 <= k <= 4
 
     Ctl* ctl() const { return reinterpret_cast<Ctl*>(ws + L.ctl); }
@@ -384,8 +387,10 @@ static cudaError_t tile_launch(const gs_sim* s, uint32_t ncycles, cudaStream_t s
     return launch_tile(a, s->tw, s->tile_groups, s->tile_grid, st);
 }
 
+// evs (profiling): timing events around every level launch (or around the concurrent level
+// region); ext = the launches are being captured, record the events as graph nodes
 static cudaError_t cycle_launches(const gs_sim* s, uint32_t parity, cudaStream_t st,
-                                  std::vector<cudaEvent_t>* evs = nullptr) {
+                                  std::vector<cudaEvent_t>* evs = nullptr, bool ext = false) {
     const Program& p = *s->prog;
     cudaError_t e = launch_stim(s->ctl(), s->state(), s->stride, s->words, p.row_pi0, p.n_pi,
                                 s->opts.lane_offset / 64, s->pdl, st);
@@ -395,6 +400,23 @@ static cudaError_t cycle_launches(const gs_sim* s, uint32_t parity, cudaStream_t
         e = dataflow_launch(s, parity, st);
         if (evs) cudaEventRecord((*evs)[1], st);
         if (e != cudaSuccess) return e;
+        return launch_end_cycle(end_args(s, parity), st);
+    }
+    if (s->concurrent) {
+        // lane groups: one branch per group, forked after the stimulus kernel and joined
+        // before the end-of-cycle kernel; the branches share nothing but the stimulus rows
+        if (evs) cudaEventRecordWithFlags((*evs)[0], st, ext ? cudaEventRecordExternal : 0u);
+        if ((e = cudaEventRecord(s->gev[0], st)) != cudaSuccess) return e;
+        for (uint32_t sl = 0; sl < s->slabs; ++sl) {
+            cudaStream_t b = sl ? s->gstream[sl - 1] : st;
+            if (sl && (e = cudaStreamWaitEvent(b, s->gev[0], 0)) != cudaSuccess) return e;
+            for (uint32_t l = 0; l < p.n_levels; ++l)
+                if ((e = level_launch(s, l, parity, b, sl)) != cudaSuccess) return e;
+            if (sl && (e = cudaEventRecord(s->gev[sl], b)) != cudaSuccess) return e;
+        }
+        for (uint32_t sl = 1; sl < s->slabs; ++sl)
+            if ((e = cudaStreamWaitEvent(st, s->gev[sl], 0)) != cudaSuccess) return e;
+        if (evs) cudaEventRecordWithFlags((*evs)[1], st, ext ? cudaEventRecordExternal : 0u);
         return launch_end_cycle(end_args(s, parity), st);
     }
     // slab-major order: every level on lanes [slab], then the next slab (lanes are
@@ -424,6 +446,32 @@ static gs_status ensure_graph(gs_sim* s, uint32_t parity) {
     cudaGraphDestroy(g);
     CU(e3);
     return GS_OK;
+}
+
+// lane_groups = 0: concurrent lane groups for kernel A (measured on C2-C5):
+// four groups of >= 4,096 lanes, but only two when a level launch averages > 1 GB of
+// algorithmic traffic (C5 shard: the level already fills the GPU for ~0.3 ms, and four
+// groups' 1 KB row segments lose more to short rows than the overlap gains).
+static uint32_t auto_lane_groups(const Program& p, const gs_sim_opts& o) {
+    if (o.kernel != GS_KERNEL_LUT || o.lane_slabs > 1 || o.lanes % 128) return 1;
+    const uint32_t vrow = (uint32_t)(o.lanes / 128);
+    double bytes = 0;
+    uint32_t nl = 0;
+    for (uint32_t l = 0; l < p.n_levels; ++l) nl += p.level_off[l + 1] > p.level_off[l] ? 1 : 0;
+    for (uint32_t g = 0; g < p.n_eval; ++g) bytes += (double)((p.aux[g].k & 0xFFu) + 1) * (double)(o.lanes / 8);
+    const uint32_t gmax = (nl && bytes / nl > 1e9) ? 2 : 4;
+    for (uint32_t G = gmax; G > 1; G /= 2)
+        if (vrow % G == 0 && (vrow / G) % 32 == 0) return G;
+    return 1;
+}
+
+static void destroy_groups(gs_sim* s) {
+    for (auto& b : s->gstream)
+        if (b) cudaStreamSynchronize(b), cudaStreamDestroy(b);
+    for (auto& v : s->gev)
+        if (v) cudaEventDestroy(v);
+    s->gstream.clear();
+    s->gev.clear();
 }
 
 static gs_status check_sim(const gs_sim* s, const char* fn) {
@@ -514,6 +562,18 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
             }
     }
     s->slabs = (opts->lane_slabs && s->opts.kernel != GS_KERNEL_DATAFLOW) ? opts->lane_slabs : 1;
+    uint32_t groups = opts->lane_groups;
+    if (groups == 0) groups = auto_lane_groups(p, *opts);
+    if (groups > 1) {
+        const uint32_t vrow = words / 2, G = groups;
+        if (opts->lane_slabs > 1 || s->opts.kernel != GS_KERNEL_LUT || words % 2 || vrow % G || (vrow / G) % 32) {
+            delete s;
+            return fail(GS_ERR_ARG, "gs_sim_create: lane_groups needs kernel A, no lane_slabs, (lanes/128) % groups "
+                                    "== 0 and a multiple of 4096 lanes per group");
+        }
+        s->slabs = G;
+        s->concurrent = true;
+    }
     if (s->slabs > 1) {
         const uint32_t vrow = words / 2;
         if (s->opts.kernel != GS_KERNEL_LUT || words % 2 || vrow % s->slabs || (vrow / s->slabs) % 32) {
@@ -553,6 +613,18 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
     }
     e = cudaStreamCreateWithFlags(&s->cap, cudaStreamNonBlocking);
     if (e != cudaSuccess) return cleanup(fail(GS_ERR_CUDA, std::string("cudaStreamCreate: ") + cudaGetErrorString(e)));
+    if (s->concurrent) {
+        s->gstream.assign(s->slabs - 1, nullptr);
+        s->gev.assign(s->slabs, nullptr);
+        for (auto& b : s->gstream)
+            if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&b, cudaStreamNonBlocking);
+        for (auto& v : s->gev)
+            if (e == cudaSuccess) e = cudaEventCreateWithFlags(&v, cudaEventDisableTiming);
+        if (e != cudaSuccess) {
+            destroy_groups(s);
+            return cleanup(fail(GS_ERR_CUDA, std::string("lane groups: ") + cudaGetErrorString(e)));
+        }
+    }
     // upload the program (descriptors are device-resident for the sim's lifetime)
     struct Up { size_t off; const void* src; size_t n; };
     std::vector<int32_t> slot(words, -1);
@@ -602,6 +674,7 @@ gs_status gs_sim_destroy(gs_sim* s) {
     if (!s) return GS_OK;
     cudaSetDevice(s->opts.device);
     cudaStreamSynchronize(s->stream);
+    destroy_groups(s);
     for (auto& x : s->exec)
         if (x) cudaGraphExecDestroy(x);
     if (s->cap) cudaStreamDestroy(s->cap);
@@ -806,6 +879,13 @@ gs_status gs_sim_get_cycle(const gs_sim* s, uint64_t* cycle) {
     return GS_OK;
 }
 
+gs_status gs_sim_get_config(const gs_sim* s, int* kernel, uint32_t* lane_groups) {
+    if (!s || !kernel || !lane_groups) return fail(GS_ERR_ARG, "gs_sim_get_config: NULL argument");
+    *kernel = s->opts.kernel;
+    *lane_groups = s->concurrent ? s->slabs : 1u;
+    return GS_OK;
+}
+
 gs_status gs_sim_read_outputs(gs_sim* s, uint64_t* host, size_t nwords) {
     if (gs_status st = check_sim(s, "gs_sim_read_outputs")) return st;
     const Program& p = *s->prog;
@@ -968,10 +1048,35 @@ gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
         for (uint32_t g = p.level_off[l]; g < p.level_off[l + 1]; ++g)
             lb[l] += (double)(p.aux[g].k + 1 + (p.aux[g].qdst != NONE32 ? 1 : 0)) * (double)s->stride;
     gs_status rc = GS_OK;
+    // concurrent lane groups: the branches only overlap as they do in gs_sim_step when the
+    // cycle is replayed as its graph, so profile a graph of the cycle with timing-event
+    // nodes at the fork and the join (eager launches of G x levels kernels would measure
+    // the host's launch rate instead)
+    cudaGraphExec_t px[2] = {nullptr, nullptr};
+    auto prof_graph = [&](uint32_t parity) -> cudaError_t {
+        if (px[parity]) return cudaSuccess;
+        cudaGraph_t g = nullptr;
+        cudaError_t e = cudaStreamBeginCapture(s->cap, cudaStreamCaptureModeThreadLocal);
+        if (e != cudaSuccess) return e;
+        e = cycle_launches(s, parity, s->cap, &evs, true);
+        cudaError_t e2 = cudaStreamEndCapture(s->cap, &g);
+        if (e == cudaSuccess) e = e2;
+        if (e == cudaSuccess) e = cudaGraphInstantiate(&px[parity], g, 0);
+        if (g) cudaGraphDestroy(g);
+        return e;
+    };
     for (uint32_t i = 0; i < n && rc == GS_OK; ++i) {
         const uint32_t parity = (uint32_t)(s->cycle & 1);
-        cudaEventRecord(e0, s->stream);
-        cudaError_t e = cycle_launches(s, parity, s->stream, &evs);
+        cudaError_t e = cudaSuccess;
+        if (s->concurrent) {
+            e = prof_graph(parity);
+            if (e != cudaSuccess) { rc = fail(GS_ERR_CUDA, cudaGetErrorString(e)); break; }
+            cudaEventRecord(e0, s->stream);
+            e = cudaGraphLaunch(px[parity], s->stream);
+        } else {
+            cudaEventRecord(e0, s->stream);
+            e = cycle_launches(s, parity, s->stream, &evs);
+        }
         cudaEventRecord(e1, s->stream);
         if (e != cudaSuccess) { rc = fail(GS_ERR_CUDA, cudaGetErrorString(e)); break; }
         s->cycle++;
@@ -980,11 +1085,13 @@ gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
         float ms = 0;
         cudaEventElapsedTime(&ms, e0, e1);
         total_ms += ms;
-        if (df) {                      // one persistent launch covers every level
+        if (df || s->concurrent) {     // one persistent launch / concurrent branches cover every level
             cudaEventElapsedTime(&ms, evs[0], evs[1]);
             level_ms += ms;
             for (uint32_t l = 0; l < p.n_levels; ++l) level_bytes += lb[l];
-            lvl_launches += s->df.nl ? 1 : 0;
+            if (df) lvl_launches += s->df.nl ? 1 : 0;
+            else
+                for (uint32_t l = 0; l < p.n_levels; ++l) lvl_launches += p.level_off[l + 1] > p.level_off[l] ? s->slabs : 0;
         } else
         for (uint32_t sl = 0; sl < s->slabs; ++sl)
             for (uint32_t l = 0; l < p.n_levels; ++l) {
@@ -997,6 +1104,8 @@ gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
             }
         launches += per;
     }
+    for (auto& x : px)
+        if (x) cudaGraphExecDestroy(x);
     for (auto& e : evs) cudaEventDestroy(e);
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);

@@ -322,6 +322,43 @@ def test_launch_and_cache_options_do_not_change_results(flags):
         assert np.array_equal(a[key], b[key]), key
 
 
+# ------------------------------------------------------------------ kernel A, concurrent lane groups
+@pytest.mark.parametrize("groups,lanes,graphs", [(2, 8192, True), (4, 16384, True), (3, 12288, True),
+                                                 (2, 8192, False), (8, 32768, True)])
+def test_lane_groups_every_lane_vs_oracle(groups, lanes, graphs):
+    """Lane groups (each group's level chain a concurrent graph branch / stream): a sequential
+    netlist with fused latches and Q-bank inputs, every lane, every cycle's trace of sampled
+    words, registers and signatures vs the oracle; identical to the single-chain run."""
+    nl = workloads.synthetic(3000, 120, 20, 32, 16, seed=22, name="groups")
+    prog = compile_nl(nl)
+    cycles = 9
+    W_ = lanes // 64
+    tw = [0, W_ // groups - 1, W_ // groups, W_ - 1]           # group boundaries
+    r = run_gpu(nl, lanes, cycles, "lut", seed=3, prog=prog, lane_groups=groups, use_graphs=graphs,
+                trace_words=tw, lane_offset=64 * 77)
+    o = oracle.simulate(nl, np.arange(lanes) + 64 * 77, cycles, seed=3)
+    assert np.array_equal(gs.unpack_lanes(r["outputs"]).T, o["last"])
+    assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"])
+    assert np.array_equal(r["sigs"], o["sig"])
+    tb = gpu_trace_bits(r["trace"], None)
+    sel = np.concatenate([np.arange(64) + 64 * w for w in tw])
+    assert np.array_equal(tb, o["trace"][sel])
+    b = run_gpu(nl, lanes, cycles, "lut", seed=3, prog=prog, lane_groups=1, lane_offset=64 * 77)
+    for key in ("outputs", "regs", "sigs"):
+        assert np.array_equal(r[key], b[key]), key
+
+
+def test_lane_groups_reject_bad_shapes():
+    nl = workloads.synthetic(2000, 60, 8, 32, 8, seed=2, name="g")
+    prog = compile_nl(nl)
+    for kw in (dict(lanes=8192, lane_groups=3), dict(lanes=4096, lane_groups=2),
+               dict(lanes=8192, lane_groups=2, lane_slabs=2), dict(lanes=8192, lane_groups=2, kernel="poly")):
+        kernel = kw.pop("kernel", "lut")
+        with pytest.raises(gs.GsError) as e:
+            gs.Sim(prog, kernel=kernel, **kw)
+        assert e.value.code == gs.GS_ERR_ARG
+
+
 # ------------------------------------------------------------------ kernel A, bulk-copy gathers
 @pytest.mark.parametrize("lanes", [16384, 32768, 65536])      # 2 / 4 / 8 KB rows: every chunk size
 @pytest.mark.parametrize("kernel", ["lut", "ab"])
