@@ -143,6 +143,18 @@ def ncu_traffic(config: str, kernel: str):
         return None
 
 
+def insitu_dram(config: str, groups: int, ms_per_cycle: float, peak: float):
+    """Actual DRAM rate of the whole cycle: the committed in-situ DRAM bytes of one cycle graph
+    (ncu --graph-profiling graph, profiles/traffic.json 'cycles') / this run's time per cycle."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            e = json.load(f)["cycles"][f"{config}:G{groups}"]
+    except Exception:
+        return None
+    gbs = e["dram_bytes_per_cycle"] / (ms_per_cycle / 1e3) / 1e9
+    return {"bytes_per_cycle": e["dram_bytes_per_cycle"], "gbs": gbs, "frac": gbs / peak, "source": e["source"]}
+
+
 # ------------------------------------------------------------------ CPU oracle
 def oracle_rate(nl, cfg, lane_offset, seconds: float, cycles_cap: int | None = None):
     """Time the oracle (as it stands) on a bounded sample: n_threads lanes x c cycles."""
@@ -305,6 +317,7 @@ def main():
                 "algorithmic_bytes_per_launch": per_launch_bytes,
                 "level_share_of_step": pr["level_ms"] / pr["total_ms"],
                 "lane_groups": G_groups,
+                "dram_insitu": insitu_dram(args.config, G_groups, ms_max / (args.steps * C), pk["hbm_gbs"]),
                 "avg_level_launch_us": pr["level_ms"] * 1e3 / max(pr["level_launches"], 1),
                 "measured": (f"CUDA events around every level launch on the sim stream, "
                              f"{min(C, 10)} un-graphed cycles after the timed region") if G_groups == 1 else
