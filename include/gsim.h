@@ -251,9 +251,10 @@ typedef struct {
     uint32_t lane_groups;         /* LUT: cut the lanes into this many groups whose level
                                      chains run CONCURRENTLY every cycle (parallel branches of
                                      the cycle's CUDA graph / streams), so one group's level
-                                     ramp and drain overlap another's levels.  Needs
-                                     (lanes/128) % groups == 0 and >= 4096 lanes per group.
-                                     0 = auto, 1 = off.                      */
+                                     ramp and drain overlap another's levels.  With
+                                     lane_slabs = S > 1 each group runs its lanes as S slabs,
+                                     slab-major.  Needs (lanes/128) % (groups x S) == 0 and
+                                     >= 4096 lanes per slab.  0 = auto, 1 = off. */
 } gs_sim_opts;
 /* flags: launch the per-cycle kernels WITHOUT programmatic dependent launch (by default a
  * level kernel may become resident while its predecessor drains; A/B measurement only). */

@@ -231,6 +231,7 @@ struct gs_sim {
     uint32_t sms = 148;
     bool bulk = false;                // kernel A: bulk-copy staged gathers (k_level_bulk)
     bool concurrent = false;          // lane groups: the slabs' level chains run concurrently
+    uint32_t branches = 1;            // concurrent lane groups; each runs slabs / branches slabs
     std::vector<cudaStream_t> gstream;  // [slabs - 1] branch streams (group 0: the caller's)
     std::vector<cudaEvent_t> gev;       // [0] fork, [1 .. slabs - 1] joins
     std::vector<uint8_t> lv_bulk;     // [n_levels] every gate of the level has 1 <= k <= 4
@@ -407,15 +408,17 @@ static cudaError_t cycle_launches(const gs_sim* s, uint32_t parity, cudaStream_t
         // before the end-of-cycle kernel; the branches share nothing but the stimulus rows
         if (evs) cudaEventRecordWithFlags((*evs)[0], st, ext ? cudaEventRecordExternal : 0u);
         if ((e = cudaEventRecord(s->gev[0], st)) != cudaSuccess) return e;
-        for (uint32_t sl = 0; sl < s->slabs; ++sl) {
-            cudaStream_t b = sl ? s->gstream[sl - 1] : st;
-            if (sl && (e = cudaStreamWaitEvent(b, s->gev[0], 0)) != cudaSuccess) return e;
-            for (uint32_t l = 0; l < p.n_levels; ++l)
-                if ((e = level_launch(s, l, parity, b, sl)) != cudaSuccess) return e;
-            if (sl && (e = cudaEventRecord(s->gev[sl], b)) != cudaSuccess) return e;
+        const uint32_t per = s->slabs / s->branches;      // slabs of one group, run slab-major
+        for (uint32_t br = 0; br < s->branches; ++br) {
+            cudaStream_t b = br ? s->gstream[br - 1] : st;
+            if (br && (e = cudaStreamWaitEvent(b, s->gev[0], 0)) != cudaSuccess) return e;
+            for (uint32_t j = 0; j < per; ++j)
+                for (uint32_t l = 0; l < p.n_levels; ++l)
+                    if ((e = level_launch(s, l, parity, b, br * per + j)) != cudaSuccess) return e;
+            if (br && (e = cudaEventRecord(s->gev[br], b)) != cudaSuccess) return e;
         }
-        for (uint32_t sl = 1; sl < s->slabs; ++sl)
-            if ((e = cudaStreamWaitEvent(st, s->gev[sl], 0)) != cudaSuccess) return e;
+        for (uint32_t br = 1; br < s->branches; ++br)
+            if ((e = cudaStreamWaitEvent(st, s->gev[br], 0)) != cudaSuccess) return e;
         if (evs) cudaEventRecordWithFlags((*evs)[1], st, ext ? cudaEventRecordExternal : 0u);
         return launch_end_cycle(end_args(s, parity), st);
     }
@@ -566,12 +569,14 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
     if (groups == 0) groups = auto_lane_groups(p, *opts);
     if (groups > 1) {
         const uint32_t vrow = words / 2, G = groups;
-        if (opts->lane_slabs > 1 || s->opts.kernel != GS_KERNEL_LUT || words % 2 || vrow % G || (vrow / G) % 32) {
+        const uint32_t S = std::max<uint32_t>(1, opts->lane_slabs);     // slabs per group
+        if (s->opts.kernel != GS_KERNEL_LUT || words % 2 || vrow % (G * S) || (vrow / (G * S)) % 32) {
             delete s;
-            return fail(GS_ERR_ARG, "gs_sim_create: lane_groups needs kernel A, no lane_slabs, (lanes/128) % groups "
-                                    "== 0 and a multiple of 4096 lanes per group");
+            return fail(GS_ERR_ARG, "gs_sim_create: lane_groups needs kernel A, (lanes/128) % (groups x lane_slabs) "
+                                    "== 0 and a multiple of 4096 lanes per slab");
         }
-        s->slabs = G;
+        s->slabs = G * S;
+        s->branches = G;
         s->concurrent = true;
     }
     if (s->slabs > 1) {
@@ -614,8 +619,8 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
     e = cudaStreamCreateWithFlags(&s->cap, cudaStreamNonBlocking);
     if (e != cudaSuccess) return cleanup(fail(GS_ERR_CUDA, std::string("cudaStreamCreate: ") + cudaGetErrorString(e)));
     if (s->concurrent) {
-        s->gstream.assign(s->slabs - 1, nullptr);
-        s->gev.assign(s->slabs, nullptr);
+        s->gstream.assign(s->branches - 1, nullptr);
+        s->gev.assign(s->branches, nullptr);
         for (auto& b : s->gstream)
             if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&b, cudaStreamNonBlocking);
         for (auto& v : s->gev)
@@ -882,7 +887,7 @@ gs_status gs_sim_get_cycle(const gs_sim* s, uint64_t* cycle) {
 gs_status gs_sim_get_config(const gs_sim* s, int* kernel, uint32_t* lane_groups) {
     if (!s || !kernel || !lane_groups) return fail(GS_ERR_ARG, "gs_sim_get_config: NULL argument");
     *kernel = s->opts.kernel;
-    *lane_groups = s->concurrent ? s->slabs : 1u;
+    *lane_groups = s->concurrent ? s->branches : 1u;
     return GS_OK;
 }
 

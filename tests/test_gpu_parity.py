@@ -323,9 +323,10 @@ def test_launch_and_cache_options_do_not_change_results(flags):
 
 
 # ------------------------------------------------------------------ kernel A, concurrent lane groups
-@pytest.mark.parametrize("groups,lanes,graphs", [(2, 8192, True), (4, 16384, True), (3, 12288, True),
-                                                 (2, 8192, False), (8, 32768, True)])
-def test_lane_groups_every_lane_vs_oracle(groups, lanes, graphs):
+@pytest.mark.parametrize("groups,lanes,graphs,slabs", [(2, 8192, True, 0), (4, 16384, True, 0), (3, 12288, True, 0),
+                                                       (2, 8192, False, 0), (8, 32768, True, 0), (2, 16384, True, 2),
+                                                       (2, 24576, False, 3)])
+def test_lane_groups_every_lane_vs_oracle(groups, lanes, graphs, slabs):
     """Lane groups (each group's level chain a concurrent graph branch / stream): a sequential
     netlist with fused latches and Q-bank inputs, every lane, every cycle's trace of sampled
     words, registers and signatures vs the oracle; identical to the single-chain run."""
@@ -335,7 +336,7 @@ def test_lane_groups_every_lane_vs_oracle(groups, lanes, graphs):
     W_ = lanes // 64
     tw = [0, W_ // groups - 1, W_ // groups, W_ - 1]           # group boundaries
     r = run_gpu(nl, lanes, cycles, "lut", seed=3, prog=prog, lane_groups=groups, use_graphs=graphs,
-                trace_words=tw, lane_offset=64 * 77)
+                trace_words=tw, lane_offset=64 * 77, lane_slabs=slabs)
     o = oracle.simulate(nl, np.arange(lanes) + 64 * 77, cycles, seed=3)
     assert np.array_equal(gs.unpack_lanes(r["outputs"]).T, o["last"])
     assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"])
@@ -353,6 +354,7 @@ def test_lane_groups_reject_bad_shapes():
     prog = compile_nl(nl)
     for kw in (dict(lanes=8192, lane_groups=3), dict(lanes=4096, lane_groups=2),
                dict(lanes=8192, lane_groups=2, lane_slabs=2), dict(lanes=8192, lane_groups=2, kernel="poly")):
+        # (8192 lanes as 2 groups x 2 slabs = 2048 lanes per slab: below the 4096 minimum)
         kernel = kw.pop("kernel", "lut")
         with pytest.raises(gs.GsError) as e:
             gs.Sim(prog, kernel=kernel, **kw)
