@@ -18,6 +18,7 @@
 // then ballot-packed back to 32 stimuli per word.  Outputs outside {0,1} are counted
 // (P:224 says they cannot happen).  Used standalone or as a cross-check of A.
 #include <algorithm>
+#include <atomic>
 
 #include <cuda_runtime.h>
 
@@ -377,12 +378,15 @@ __global__ void __launch_bounds__(BULK_THREADS, MINB) k_level_bulk(LevelArgs a, 
 template <int C, int S, int MINB>
 static cudaError_t launch_bulk(const LevelArgs& a, cudaStream_t st, int sms) {
     constexpr size_t smem = 1024 + (size_t)S * 4 * C;
-    static bool attr = false;                  // set once per process (same for every device)
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_level_bulk<C, S, MINB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)smem);
+    static std::atomic<uint64_t> attr{0};     // devices whose function attribute is set
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    const uint64_t bit = 1ull << (dev & 63);
+    if (!(attr.load() & bit)) {
+        e = cudaFuncSetAttribute(k_level_bulk<C, S, MINB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
-        attr = true;
+        attr.fetch_or(bit);
     }
     const uint32_t vrow = a.vslab ? a.vslab : a.words / 2;
     const uint32_t cpg = vrow * 16 / C;
