@@ -206,9 +206,10 @@ gs_status gs_program_tile_slots(const gs_program* prog, uint32_t* slots);
 
 /* ======================================================================= simulate */
 enum {
-    GS_KERNEL_AUTO = 0,   /* GS_KERNEL_TILE when every LUT has k <= 5 and one tile's live
+    GS_KERNEL_AUTO = 0,   /* GS_KERNEL_TILE when every LUT has k <= 5, one tile's live
                              state fits shared memory next to the gate descriptors
-                             (resident or TMA-streamed); else GS_KERNEL_LUT              */
+                             (resident or TMA-streamed) and the levels average <= 400
+                             gates (or lanes < 32,768); else GS_KERNEL_LUT               */
     GS_KERNEL_LUT = 1,    /* kernel A: bit-sliced LUT evaluation, 64 stimuli per word      */
     GS_KERNEL_POLY = 2,   /* kernel B: the paper's network, sum_S w_S Theta(sum x - |S| + 1)
                              per stimulus in int32, ballot-packed (Eq. 1-3)                */

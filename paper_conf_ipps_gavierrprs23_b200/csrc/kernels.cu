@@ -262,9 +262,9 @@ __device__ __forceinline__ void mbar_wait_d(uint64_t* bar, uint32_t parity) {
     uint32_t done = 0;
     while (!done) {
         asm volatile(
-            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n selp.u32 %0, 1, 0, p;\n}\n"
             : "=r"(done)
-            : "r"((uint32_t)__cvta_generic_to_shared(bar)), "r"(parity)
+            : "r"((uint32_t)__cvta_generic_to_shared(bar)), "r"(parity), "r"(1000000u)   // suspend, not spin
             : "memory");
     }
 }

@@ -127,9 +127,11 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
 }
 
 // GS_KERNEL_AUTO: kernel T when one tile's live state fits shared memory next to either the
-// whole descriptor table or the TMA descriptor double buffer (small and mid-size circuits:
-// measured 1.8x kernel A on C2, 5.8x on C1, 2.6x / 1.4x / 1.1x on 5k / 10k / 20k-gate
-// synthetic circuits), else kernel A (large circuits are HBM-bound; T cannot hold them).
+// whole descriptor table or the TMA descriptor double buffer and the levels are narrow
+// (small and mid-size circuits: measured 1.8x kernel A on C2, 5.8x on C1, 2.7x / 1.8x on
+// 5k / 10k-gate synthetic circuits), else kernel A (large circuits are HBM-bound and T
+// cannot hold them; from ~500 gates per level kernel A with concurrent lane groups wins:
+// 20k gates / 38 levels at 65,536 lanes A 9.4e12 vs T 8.6e12, profiles/r01_mid_size_*).
 // Programs with 6-8-input LUTs use kernel A.
 gs_sim_opts resolve_auto(const Program& p, const gs_sim_opts& o) {
     gs_sim_opts r = o;
@@ -138,6 +140,9 @@ gs_sim_opts resolve_auto(const Program& p, const gs_sim_opts& o) {
     // wide LUTs make every level ALU-heavy (2^k - 1 LOP3 per 32 lanes): kernel A's higher
     // occupancy wins from k = 6 on (measured on C2 collapsed to L = 6, 7, 8)
     if (p.max_k > 5) return r;
+    uint32_t nl = 0;
+    for (uint32_t l = 0; l < p.n_levels; ++l) nl += p.level_off[l + 1] > p.level_off[l] ? 1 : 0;
+    if (nl && p.n_eval / nl > 400 && o.lanes >= 32768) return r;
     r.kernel = GS_KERNEL_TILE;
     Plans pl;
     const std::string saved = gs_last_error();

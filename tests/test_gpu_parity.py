@@ -481,14 +481,15 @@ def test_collapsed_to_8_input_luts_closed_forms(L):
 
 
 # ------------------------------------------------------------------ streamed host I/O (f3)
-@pytest.mark.parametrize("kernel,chunk", [("lut", 4), ("lut", 0), ("tile", 7), ("poly", 5)])
-def test_run_streamed_every_output_every_cycle_vs_oracle(kernel, chunk):
+@pytest.mark.parametrize("kernel,chunk,lanes", [("lut", 4, 2048), ("lut", 0, 2048), ("tile", 7, 2048),
+                                               ("poly", 5, 2048), ("lut", 6, 16384)])   # 16,384: 4 lane groups
+def test_run_streamed_every_output_every_cycle_vs_oracle(kernel, chunk, lanes):
     """gs_sim_run_streamed: host stimuli in, EVERY output of EVERY cycle out (paper P:271),
     chunks pipelined on a copy stream; compared with the oracle on every lane and cycle."""
     import torch
     nl = workloads.random_tiny(8, n_pi=7, n_reg=6, n_gates=400, n_po=20, max_k=4)
     prog = compile_nl(nl)
-    lanes, cycles = 2048, 30
+    cycles = 30
     W_ = lanes // 64
     stim = workloads.random_host_stimulus(5, cycles, nl.n_pi, W_)
     pin_in = torch.from_numpy(stim.view(np.int64)).pin_memory()
