@@ -322,6 +322,64 @@ def test_launch_and_cache_options_do_not_change_results(flags):
         assert np.array_equal(a[key], b[key]), key
 
 
+# ------------------------------------------------------------------ degenerate netlists
+def _degenerate_netlists():
+    B = W.Builder
+    out = {}
+    b = B()                                  # no gates at all: PIs and registers straight to POs
+    p0, p1 = b.pi(), b.pi()
+    r = b.reg(1)
+    b.set_d(r, p1)
+    b.out(p0), b.out(r), b.out(p0)           # an output listed twice
+    out["no_gates"] = b.build("no_gates")
+    b = B()                                  # no PIs: a free-running 3-bit counter
+    q = [b.reg(0) for _ in range(3)]
+    t0 = b.gate(0b01, q[0])                                  # NOT
+    c1 = b.gate(0b0110, q[0], q[1])                          # XOR
+    a01 = b.gate(0b1000, q[0], q[1])
+    c2 = b.gate(0b0110, a01, q[2])
+    for r_, d in zip(q, (t0, c1, c2)):
+        b.set_d(r_, d)
+    for r_ in q:
+        b.out(r_)
+    out["no_pis"] = b.build("no_pis")
+    b = B()                                  # only constant (k = 0) gates and a 1-input buffer
+    p0 = b.pi()
+    c0, c1 = b.gate(0), b.gate(1)
+    buf = b.gate(0b10, p0)
+    b.out(c0), b.out(c1), b.out(buf)
+    out["consts"] = b.build("consts")
+    b = B()                                  # registers only, no outputs observed except one
+    r1, r2 = b.reg(1), b.reg(0)
+    b.set_d(r1, r2), b.set_d(r2, r1)
+    b.out(r1)
+    out["swap_only"] = b.build("swap_only")
+    return out
+
+
+@pytest.mark.parametrize("name", ["no_gates", "no_pis", "consts", "swap_only"])
+@pytest.mark.parametrize("kernel", ["auto", "lut", "poly", "ab", "tile"])
+def test_degenerate_netlists_every_kernel(name, kernel):
+    """Degenerate circuits (no gates, no primary inputs, only constant LUTs, registers only)
+    on every kernel, every lane and register vs the oracle; step(0) is a no-op."""
+    nl = _degenerate_netlists()[name]
+    prog = compile_nl(nl)
+    lanes, cycles = 256, 5
+    sim = gs.Sim(prog, lanes, kernel=kernel)
+    sim.bind_generated(17)
+    sim.step(0)
+    assert sim.cycle == 0
+    sim.step(cycles)
+    sim.sync()
+    o = oracle.simulate(nl, np.arange(lanes), cycles, seed=17, want=("last", "regs", "sig"))
+    assert np.array_equal(gs.unpack_lanes(sim.read_outputs()).T, o["last"])
+    if nl.n_reg:
+        assert np.array_equal(gs.unpack_lanes(sim.read_registers()).T, o["regs"])
+    assert np.array_equal(sim.read_lane_signatures(), o["sig"])
+    assert sim.signature()["cycles"] == cycles
+    sim.close()
+
+
 # ------------------------------------------------------------------ kernel A, concurrent lane groups
 @pytest.mark.parametrize("groups,lanes,graphs,slabs", [(2, 8192, True, 0), (4, 16384, True, 0), (3, 12288, True, 0),
                                                        (2, 8192, False, 0), (8, 32768, True, 0), (2, 16384, True, 2),
