@@ -1,4 +1,9 @@
-# A/B of two builds of libgsim.so in one box: $O/sweep.txt lines tagged new/head
+#!/bin/bash
+# A/B of two builds of libgsim.so on ONE box (boxes differ by up to ~6 %): bench lines tagged
+# new / head in gpurun_out/$TAG/sweep.txt, two repetitions each.  Prepare here:
+#   git worktree add /tmp/headrepo <ref> && (cd /tmp/headrepo && python -m paper_conf_ipps_gavierrprs23_b200._build)
+#   cp /tmp/headrepo/paper_conf_ipps_gavierrprs23_b200/libgsim.so paper_conf_ipps_gavierrprs23_b200/libgsim_head.so
+# then: gpurun -- 'TAG=ab CONFIGS="C3 C4" bash scripts/ab_libs.sh'
 O=gpurun_out/${TAG:-ab}; mkdir -p $O
 P=paper_conf_ipps_gavierrprs23_b200
 cp $P/libgsim.so $P/libgsim_new.so
