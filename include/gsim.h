@@ -150,6 +150,10 @@ typedef struct {
                          has <= L nets (logic is duplicated where a cone is shared); gates
                          nobody reads any more report k = 0.  Same simulation results,
                          fewer levels and LUTs.                                        */
+    uint64_t level_seed;  /* 0: levels from `balance`.  Otherwise every gate gets a seeded
+                         RANDOM level in [1 + max level of its gate inputs, ALAP] (a valid
+                         assignment of the same depth; results must not depend on it, a
+                         property test of DESIGN.md reading R11).                      */
 } gs_compile_opts;
 
 /* Validate (GS_ERR_UNDRIVEN, GS_ERR_COMB_LOOP, GS_ERR_ARITY), optionally collapse cones

@@ -131,8 +131,9 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
         asap[g] = l + 1;
         D = std::max(D, asap[g]);
     }
-    if (opts.balance && n_eval > 0) {
-        std::vector<uint32_t> alap(G, D);
+    std::vector<uint32_t> alap;
+    if ((opts.balance || opts.level_seed) && n_eval > 0) {
+        alap.assign(G, D);
         for (size_t i = topo.size(); i-- > 0;) {
             uint32_t g = topo[i];
             if (nl.gate_k[g] == 0) continue;
@@ -140,6 +141,25 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
             for (uint32_t e = cons_off[g]; e < cons_off[g + 1]; ++e) a = std::min(a, alap[cons[e]] - 1);
             alap[g] = a;
         }
+    }
+    if (opts.level_seed && n_eval > 0) {
+        // seeded random valid levels: in topological order, uniform in [1 + max input level,
+        // ALAP]; the upper end stays >= the lower one because every input's level is <= its
+        // own ALAP <= ALAP(g) - 1
+        for (uint32_t g : topo) {
+            if (nl.gate_k[g] == 0) continue;
+            uint32_t lo = 1;
+            for (uint32_t e = nl.gate_in_off[g]; e < nl.gate_in_off[g + 1]; ++e) {
+                uint32_t n = nl.gate_in[e];
+                if (is_eval_gate_net(n)) lo = std::max(lo, level[nl.net_index[n]] + 1);
+            }
+            uint64_t z = opts.level_seed ^ (0x9E3779B97F4A7C15ull * (g + 1));
+            z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+            z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+            z ^= z >> 31;
+            level[g] = lo + (uint32_t)(z % (uint64_t)(alap[g] - lo + 1));
+        }
+    } else if (opts.balance && n_eval > 0) {
         // list scheduling, level by level: least slack (smallest ALAP) first, must place
         // every gate whose ALAP is this level, otherwise fill up to the mean width.
         const uint64_t target = (n_eval + D - 1) / D;

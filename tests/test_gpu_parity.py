@@ -322,6 +322,24 @@ def test_launch_and_cache_options_do_not_change_results(flags):
         assert np.array_equal(a[key], b[key]), key
 
 
+# ------------------------------------------------------------------ random valid level assignments
+@pytest.mark.parametrize("seed", [1, 2, 3])
+@pytest.mark.parametrize("kernel", ["lut", "tile", "poly", "ab"])
+def test_random_level_assignments_do_not_change_results(seed, kernel):
+    """Any valid level assignment gives the same simulation (R11): seeded random
+    levels in [1 + max input level, ALAP] (uneven, sometimes empty levels), every lane and
+    register vs the oracle."""
+    nl = workloads.synthetic(3000, 120, 20, 32, 16, seed=30 + seed, name="lv")
+    prog = gs.Netlist.from_arrays(nl).compile(level_seed=seed)
+    lanes, cycles = 8192, 6
+    r = run_gpu(nl, lanes, cycles, kernel, seed=seed, prog=prog)
+    o = oracle.simulate(nl, np.arange(lanes), cycles, seed=seed, want=("last", "regs", "sig"))
+    assert np.array_equal(gs.unpack_lanes(r["outputs"]).T, o["last"])
+    assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"])
+    assert np.array_equal(r["sigs"], o["sig"])
+    assert r["signature"]["ab_mismatch"] == 0
+
+
 # ------------------------------------------------------------------ degenerate netlists
 def _degenerate_netlists():
     B = W.Builder

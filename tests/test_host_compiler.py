@@ -114,6 +114,32 @@ def test_levelizer_asap_and_balanced(name):
     assert np.array_equal(np.bincount(lv[ev], minlength=depth + 1)[1:], w1)
 
 
+@pytest.mark.parametrize("seed", [1, 2, 0xDEADBEEF])
+@pytest.mark.parametrize("name", ["C1", "C2", "C3"])
+def test_random_valid_levels(name, seed):
+    """level_seed: seeded random levels, each in [1 + max input level, ALAP] — valid (every
+    gate after its gate inputs), same depth, different from ASAP and from another seed."""
+    nl = workloads.build_netlist(name)
+    asap = oracle.asap_levels(nl).astype(np.int64)
+    depth = int(asap.max())
+    p = gs.Netlist.from_arrays(nl).compile(level_seed=seed)
+    lv = p.gate_levels().astype(np.int64)
+    assert p.info["n_levels"] == depth
+    alap = _alap(nl, asap, depth)
+    ev = nl.gate_k > 0
+    assert (lv[ev] >= asap[ev]).all() and (lv[ev] <= alap[ev]).all()
+    base = nl.n_pi + nl.n_reg
+    for g in np.nonzero(ev)[0][:: max(1, nl.n_gates // 20000)]:
+        for x in nl.inputs_of(int(g)):
+            if x >= base and nl.gate_k[x - base] > 0:
+                assert lv[g] > lv[x - base]
+    assert np.array_equal(np.bincount(lv[ev], minlength=depth + 1)[1:], p.level_widths())
+    if (alap[ev] > asap[ev]).any():
+        assert not np.array_equal(lv, asap)
+        lv2 = gs.Netlist.from_arrays(nl).compile(level_seed=seed + 7).gate_levels().astype(np.int64)
+        assert not np.array_equal(lv, lv2)
+
+
 def test_balancing_flattens_synthetic_widths():
     nl = workloads.build_netlist("C3")
     w0 = _compile(nl, False).level_widths()
