@@ -12,7 +12,10 @@ BASELINE.json configs[3] (C4: RISC-V-core-scale synthetic, 1M gates + 50k regist
 65,536 stimuli per GPU), the largest configuration that fits one GPU; its 1,000-cycle
 run is 10 steps.  Multi-GPU is weak scaling: every rank simulates its own 65,536 global
 lanes (lane_offset = rank * lanes) of the same netlist; the only collective is the
-all-reduce of the per-rank signatures.
+all-reduce of the per-rank signatures.  C5 (BASELINE configs[4], 8 shards of 32,768 lanes)
+runs its whole 262,144-lane batch at any N dividing 8: each rank simulates 8/N shards as
+sequential sub-batches in one workspace (gs_sim_set_lane_offset); a step is then C cycles of
+every sub-batch, each from reset.
 
 value = G_eval * lanes_total * cycles / max-over-ranks device time of the K timed steps.
 """
@@ -247,8 +250,12 @@ def main():
 
     cfg = workloads.CONFIGS[args.config]
     nl = cfg.netlist()
+    # lanes = one sim's lanes; a sharded config (C5: 8 shards of 32,768 lanes) gives every rank
+    # shards/world of them, run as sequential sub-batches in one workspace
     lanes = args.lanes or (cfg.lanes // cfg.shards if cfg.shards > 1 else cfg.lanes)
-    lane_offset = rank * lanes
+    subs = cfg.shards // world if (not args.lanes and cfg.shards > world and cfg.shards % world == 0) else 1
+    lanes_rank = lanes * subs
+    lane_offset = rank * lanes_rank
     t0 = time.perf_counter()
     prog = gs.Netlist.from_arrays(nl).compile(balance=True, lut_k=args.lut_k)
     compile_s = time.perf_counter() - t0
@@ -272,8 +279,22 @@ def main():
         if world > 1:
             dist.barrier()
 
+    sig_keys = ("lane_sig_sum", "out_popcount", "ab_mismatch", "invariant_violations")
+    sub_sigs = []
+
+    def one_step():
+        """C cycles over this rank's whole batch: one sim, or every sub-batch from reset."""
+        if subs == 1:
+            sim.step(C)
+            return
+        sub_sigs.clear()
+        for j in range(subs):
+            sim.set_lane_offset(lane_offset + j * lanes)      # syncs, re-targets, resets
+            sim.step(C)
+            sub_sigs.append(sim.signature())
+
     for _ in range(args.warmup):
-        sim.step(C)
+        one_step()
     sim.sync()
     torch.cuda.synchronize()
     barrier()
@@ -283,7 +304,7 @@ def main():
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ev0.record(stream)
     for _ in range(args.steps):
-        sim.step(C)
+        one_step()
     ev1.record(stream)
     torch.cuda.synchronize()
     clk = clocks.stop() if not args.quick else None
@@ -291,9 +312,11 @@ def main():
     barrier()
     ms_max = gdist.max_over_ranks(ms) if world > 1 else ms
     sig = sim.signature()
+    if subs > 1:                       # the last timed step's sub-batches, summed mod 2^64
+        sig = {k: (sum(d[k] for d in sub_sigs) % (1 << 64) if k in sig_keys else sig[k]) for k in sig}
     red = gdist.reduce_signature(sig) if world > 1 else sig
 
-    total_sgc = float(G) * lanes * world * C * args.steps
+    total_sgc = float(G) * lanes_rank * world * C * args.steps
     value = total_sgc / (ms_max / 1e3)
 
     # ---------------------------------------------------------------- roofline
@@ -348,13 +371,16 @@ def main():
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         for _ in range(K2):
-            sim.run_streamed(h_np, o_np)
+            for j in range(subs):
+                if subs > 1:
+                    sim.set_lane_offset(lane_offset + j * lanes)
+                sim.run_streamed(h_np, o_np)
         e1.record(stream)
         torch.cuda.synchronize()
         ems = e0.elapsed_time(e1)
         ems = gdist.max_over_ranks(ems) if world > 1 else ems
-        e2e = {"value": float(G) * lanes * world * C * K2 / (ems / 1e3), "unit": UNIT,
-               "h2d_bytes_per_step": int(host.numel() * 8), "d2h_bytes_per_step": int(out_buf.numel() * 8),
+        e2e = {"value": float(G) * lanes_rank * world * C * K2 / (ems / 1e3), "unit": UNIT,
+               "h2d_bytes_per_step": int(host.numel() * 8) * subs, "d2h_bytes_per_step": int(out_buf.numel() * 8) * subs,
                "steps": K2, "path": "gs_sim_run_streamed: pinned host stimuli in, every output of every "
                                     "cycle out, 25-cycle chunks overlapped with compute"}
 
@@ -369,7 +395,8 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
             "config": {"workload": f"{cfg.name}: {cfg.label}", "gates": G, "registers": info["n_reg"],
-                       "levels": info["n_levels"], "lanes_per_gpu": lanes, "lanes_total": lanes * world,
+                       "levels": info["n_levels"], "lanes_per_gpu": lanes_rank, "lanes_total": lanes_rank * world,
+                       "sub_batches_per_gpu": subs, "lanes_per_sub_batch": lanes,
                        "cycles_per_step": C, "kernel": args.kernel, "balance": True,
                        "lane_slabs": args.lane_slabs, "lut_unroll": args.lut_unroll,
                        "lane_groups": sim.config["lane_groups"],
@@ -378,11 +405,13 @@ def main():
                        "tile_groups": args.tile_groups, "l2_hints": args.l2_hints, "lut_k": args.lut_k,
                        "grid_stride": not args.no_grid_stride,
                        "l2": "inputs larger than L2 (state %.1f GB per GPU)" % (info["n_rows"] * lanes / 8 / 1e9),
+                       "step": f"{C} cycles over every lane of the GPU" + (
+                           f" ({subs} sub-batches of {lanes} lanes, each from reset)" if subs > 1 else ""),
                        "parallelism": f"dp{world} (stimulus sharding)" + (" TEST: all ranks on cuda:0"
                                                                               if args.same_device else ""),
                        "compile_s": round(compile_s, 2),
                        "paper_style_gcps": value * (G + info["n_reg"]) / G},
-            "gpu_launches": int(launches_per_cycle * (1 if args.kernel == "tile" else C) * args.steps),
+            "gpu_launches": int(launches_per_cycle * (1 if args.kernel == "tile" else C) * args.steps * subs),
             "signature": {k: str(v) for k, v in red.items()},
             "clocks": clk,
             "roofline": roof,

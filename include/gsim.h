@@ -307,6 +307,13 @@ gs_status gs_sim_bind_stimulus_device(gs_sim* sim, const uint64_t* dev_words, ui
 /* Q := init, cycle := 0, MISR := 0, counters := 0, trace cleared. */
 gs_status gs_sim_reset(gs_sim* sim);
 
+/* Re-target the sim at another lane range of the same job: lane_offset := the new
+ * global index of local lane 0 (a multiple of 64, else GS_ERR_ARG), then gs_sim_reset.
+ * Stimuli are independent, so a batch larger than one GPU's memory runs as
+ * sequential sub-batches in one workspace (C5 at fewer than 8 GPUs).
+ * Synchronises the sim's stream; the cycle graphs are re-captured on the next step. */
+gs_status gs_sim_set_lane_offset(gs_sim* sim, uint64_t lane_offset);
+
 /* Advance ncycles clock cycles (asynchronous on the stream).  Per cycle: stimulus
  * rows, every level in order (gates + fused register latch into the other Q bank),
  * remaining latches, output MISR/trace.  GS_ERR_STATE if no stimulus is bound or a

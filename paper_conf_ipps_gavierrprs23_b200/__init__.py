@@ -128,6 +128,7 @@ _SIGS = {
     "gs_sim_bind_stimulus_host": (C.c_int32, [_P, _P, C.c_uint32]),
     "gs_sim_bind_stimulus_device": (C.c_int32, [_P, _P, C.c_uint32]),
     "gs_sim_reset": (C.c_int32, [_P]),
+    "gs_sim_set_lane_offset": (C.c_int32, [_P, C.c_uint64]),
     "gs_sim_step": (C.c_int32, [_P, C.c_uint32]),
     "gs_sim_sync": (C.c_int32, [_P]),
     "gs_sim_run_streamed": (C.c_int32, [_P, _P, _P, C.c_uint32, C.c_uint32]),
@@ -368,6 +369,10 @@ class Sim:
 
     def reset(self):
         _call("gs_sim_reset", self.h)
+
+    def set_lane_offset(self, lane_offset: int):
+        """Move to another lane range of the same job (sub-batching), then reset."""
+        _call("gs_sim_set_lane_offset", self.h, int(lane_offset))
 
     def step(self, n: int = 1):
         _call("gs_sim_step", self.h, int(n))

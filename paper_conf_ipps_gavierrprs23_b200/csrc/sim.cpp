@@ -719,6 +719,23 @@ gs_status gs_sim_reset(gs_sim* s) {
     return GS_OK;
 }
 
+gs_status gs_sim_set_lane_offset(gs_sim* s, uint64_t lane_offset) {
+    if (gs_status st = check_sim(s, "gs_sim_set_lane_offset")) return st;
+    if (lane_offset % 64) return fail(GS_ERR_ARG, "gs_sim_set_lane_offset: lane_offset must be a multiple of 64");
+    CU(cudaSetDevice(s->opts.device));
+    if (lane_offset != s->opts.lane_offset) {
+        // the offset is a launch argument baked into the captured cycle graphs
+        CU(cudaStreamSynchronize(s->stream));
+        for (auto& x : s->exec)
+            if (x) {
+                cudaGraphExecDestroy(x);
+                x = nullptr;
+            }
+        s->opts.lane_offset = lane_offset;
+    }
+    return gs_sim_reset(s);
+}
+
 gs_status gs_sim_bind_stimulus_generated(gs_sim* s, uint64_t seed) {
     if (gs_status st = check_sim(s, "gs_sim_bind_stimulus_generated")) return st;
     CU(cudaSetDevice(s->opts.device));
