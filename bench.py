@@ -340,7 +340,7 @@ def main():
                 "algorithmic_bytes_per_launch": per_launch_bytes,
                 "level_share_of_step": pr["level_ms"] / pr["total_ms"],
                 "lane_groups": G_groups,
-                "dram_insitu": insitu_dram(args.config, G_groups, ms_max / (args.steps * C), pk["hbm_gbs"]),
+                "dram_insitu": insitu_dram(args.config, G_groups, ms_max / (args.steps * C * subs), pk["hbm_gbs"]),
                 "avg_level_launch_us": pr["level_ms"] * 1e3 / max(pr["level_launches"], 1),
                 "measured": (f"CUDA events around every level launch on the sim stream, "
                              f"{min(C, 10)} un-graphed cycles after the timed region") if G_groups == 1 else

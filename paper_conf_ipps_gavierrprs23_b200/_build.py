@@ -19,6 +19,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O2,-Wall",
           "-I" + os.path.join(ROOT, "include")]
+# experiment variants only (e.g. GS_NVCC_EXTRA="-DGS_TILE_VPT=1" for an A/B build)
+EXTRA = os.environ.get("GS_NVCC_EXTRA", "").split()
 
 
 def _sources():
@@ -44,7 +46,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     jobs = []
     for src in _sources():
         obj = os.path.join(OBJ, os.path.basename(src) + ".o")
-        cmd = [NVCC, *ARCH, *COMMON, "-c", src, "-o", obj]
+        cmd = [NVCC, *ARCH, *COMMON, *EXTRA, "-c", src, "-o", obj]
         if src.endswith(".cu"):
             cmd += ["-Xptxas", "-v"] if verbose else []
         jobs.append((cmd, obj))

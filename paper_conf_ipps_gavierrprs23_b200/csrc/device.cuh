@@ -96,23 +96,52 @@ __device__ __forceinline__ uint32_t lut_eval_wide(uint64_t tt, const uint32_t* x
     return (x[5] & hi) | (~x[5] & lo);
 }
 
+// s ? a : b bitwise, as ONE LOP3 (0xCA = F0 & CC | ~F0 & AA); written as PTX so the
+// compiler cannot split it into SEL/NOT sequences
+__device__ __forceinline__ uint32_t mux32(uint32_t s, uint32_t a, uint32_t b) {
+    uint32_t d;
+    asm("lop3.b32 %0, %1, %2, %3, 0xCA;" : "=r"(d) : "r"(s), "r"(a), "r"(b));
+    return d;
+}
+
+// minterm masks of a K <= 4 table: m[i] = all-ones iff f(i) = 1 (bit i of tt, LSB-first);
+// computed once per gate and shared by every word the thread evaluates
+template <int K>
+struct LutMasks {
+    uint32_t m[1 << K];
+};
+template <int K>
+__device__ __forceinline__ LutMasks<K> lut_masks(uint64_t tt) {
+    LutMasks<K> r;
+    const uint32_t t = (uint32_t)tt;                   // K <= 4: 16 table bits
+#pragma unroll
+    for (int i = 0; i < (1 << K); ++i)                 // sign-extended bit field: SHF + SGXT
+        asm("bfe.s32 %0, %1, %2, 1;" : "=r"(r.m[i]) : "r"(t), "r"(i));
+    return r;
+}
+
+// Shannon mux tree over the masks: 2^K - 1 LOP3 per 32 lanes
+template <int K>
+__device__ __forceinline__ uint32_t lut_eval_m(const LutMasks<K>& mk, const uint32_t* x) {
+    if constexpr (K == 0) {
+        return mk.m[0];
+    } else {
+        uint32_t v[1 << (K - 1)];
+#pragma unroll
+        for (int j = 0; j < (1 << (K - 1)); ++j) v[j] = mux32(x[0], mk.m[2 * j + 1], mk.m[2 * j]);
+#pragma unroll
+        for (int i = 1; i < K; ++i) {
+#pragma unroll
+            for (int j = 0; j < (1 << (K - 1 - i)); ++j) v[j] = mux32(x[i], v[2 * j + 1], v[2 * j]);
+        }
+        return v[0];
+    }
+}
+
 template <int K>
 __device__ __forceinline__ uint32_t lut_eval(uint64_t tt, const uint32_t* x) {
     if constexpr (K > 4) return lut_eval_wide<K>(tt, x);
-    constexpr int KK = K > 4 ? 4 : K;
-    uint32_t v[1 << (KK - 1)];
-#pragma unroll
-    for (int j = 0; j < (1 << (KK - 1)); ++j) {
-        const uint32_t c0 = 0u - (uint32_t)((tt >> (2 * j)) & 1u);
-        const uint32_t c1 = 0u - (uint32_t)((tt >> (2 * j + 1)) & 1u);
-        v[j] = (x[0] & c1) | (~x[0] & c0);
-    }
-#pragma unroll
-    for (int i = 1; i < KK; ++i) {
-#pragma unroll
-        for (int j = 0; j < (1 << (KK - 1 - i)); ++j) v[j] = (x[i] & v[2 * j + 1]) | (~x[i] & v[2 * j]);
-    }
-    return v[0];
+    else return lut_eval_m<K>(lut_masks<K>(tt), x);
 }
 
 
@@ -128,24 +157,47 @@ __device__ __forceinline__ uint32_t lut_eval_big(const uint64_t* t4, const uint3
     return (x[7] & hi) | (~x[7] & lo);
 }
 
+// evaluate one 16-byte vector (4 x 32 lanes) of a K <= 4 gate from precomputed masks
+template <int K>
+__device__ __forceinline__ uint4 lut_eval4_m(const LutMasks<K>& mk, const uint4* xv) {
+    uint4 y;
+    uint32_t x[K > 0 ? K : 1];
+#pragma unroll
+    for (int i = 0; i < K; ++i) x[i] = xv[i].x;
+    y.x = lut_eval_m<K>(mk, x);
+#pragma unroll
+    for (int i = 0; i < K; ++i) x[i] = xv[i].y;
+    y.y = lut_eval_m<K>(mk, x);
+#pragma unroll
+    for (int i = 0; i < K; ++i) x[i] = xv[i].z;
+    y.z = lut_eval_m<K>(mk, x);
+#pragma unroll
+    for (int i = 0; i < K; ++i) x[i] = xv[i].w;
+    y.w = lut_eval_m<K>(mk, x);
+    return y;
+}
+
 // evaluate 4 x 32-bit lanes-words (one 16-byte vector) of a K-input gate
 template <int K>
 __device__ __forceinline__ uint4 lut_eval4(uint64_t tt, const uint4* xv) {
-    uint4 y;
-    uint32_t x[K];
+    if constexpr (K <= 4) return lut_eval4_m<K>(lut_masks<K>(tt), xv);
+    else {
+        uint4 y;
+        uint32_t x[K];
 #pragma unroll
-    for (int i = 0; i < K; ++i) x[i] = xv[i].x;
-    y.x = lut_eval<K>(tt, x);
+        for (int i = 0; i < K; ++i) x[i] = xv[i].x;
+        y.x = lut_eval<K>(tt, x);
 #pragma unroll
-    for (int i = 0; i < K; ++i) x[i] = xv[i].y;
-    y.y = lut_eval<K>(tt, x);
+        for (int i = 0; i < K; ++i) x[i] = xv[i].y;
+        y.y = lut_eval<K>(tt, x);
 #pragma unroll
-    for (int i = 0; i < K; ++i) x[i] = xv[i].z;
-    y.z = lut_eval<K>(tt, x);
+        for (int i = 0; i < K; ++i) x[i] = xv[i].z;
+        y.z = lut_eval<K>(tt, x);
 #pragma unroll
-    for (int i = 0; i < K; ++i) x[i] = xv[i].w;
-    y.w = lut_eval<K>(tt, x);
-    return y;
+        for (int i = 0; i < K; ++i) x[i] = xv[i].w;
+        y.w = lut_eval<K>(tt, x);
+        return y;
+    }
 }
 
 }  // namespace gs

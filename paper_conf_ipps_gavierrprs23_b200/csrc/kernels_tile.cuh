@@ -25,6 +25,10 @@
 namespace gs {
 
 constexpr uint32_t TILE_CTA = 512;                   // threads per CTA (one CTA per SM)
+#ifndef GS_TILE_VPT
+#define GS_TILE_VPT 2
+#endif
+constexpr uint32_t TILE_VPT = GS_TILE_VPT;          // 16-byte vectors per thread and gate (TW >= 16)
 constexpr unsigned long long TILE_MISR_POLY = 0x42F0E1EBA9EA3693ULL;   // CRC-64/ECMA-182
 
 // Shared memory by descriptor mode:
@@ -59,12 +63,13 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     }
 }
 
-// One gate on one 16-byte group (4 words = 128 lanes) of its slots.  HASQ: the circuit has
-// registers, so an input slot may name a bank-0 register slot that must be moved to the
-// current bank.
-template <int K, bool HASQ>
-__device__ __forceinline__ void tile_gate(uint4* sl, uint32_t V, uint32_t v, const uint4& d, const uint4* desc_hi,
-                                          uint32_t g, uint32_t q0, uint32_t R, uint32_t qcur, uint32_t qnext) {
+// One gate on P 16-byte groups (4 words = 128 lanes each, VS uint4 apart) of its slots:
+// the descriptor is decoded and the truth-table masks built once for the P vectors, and
+// all P*K shared-memory loads are issued before the first is used.  HASQ: the circuit has
+// registers (fused latch of the gate's value into the next register bank).
+template <int K, bool HASQ, int P>
+__device__ __forceinline__ void tile_gate(uint4* sl, uint32_t V, uint32_t v, uint32_t VS, const uint4& d,
+                                          const uint4* desc_hi, uint32_t g, uint32_t q0, uint32_t qnext) {
     constexpr int KS = K > 4 ? 8 : 4;
     uint32_t s[KS];
     s[0] = d.x & 0xFFFFu; s[1] = d.x >> 16; s[2] = d.y & 0xFFFFu; s[3] = d.y >> 16;
@@ -80,29 +85,47 @@ __device__ __forceinline__ void tile_gate(uint4* sl, uint32_t V, uint32_t v, con
             t4[3] = ((uint64_t)h2.w << 32) | h2.z;
         }
     }
-    uint4 x[K];
-#pragma unroll
-    for (int i = 0; i < K; ++i) {
-        uint32_t si = s[i];
-        x[i] = sl[(size_t)si * V + v];
-    }
-    uint4 y;
-    if (K <= 6) {
-        y = lut_eval4<K <= 6 ? K : 6>(t4[0], x);
-    } else {
-        uint32_t xs[8];
-        uint32_t* yp = reinterpret_cast<uint32_t*>(&y);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-#pragma unroll
-            for (int i = 0; i < K; ++i) xs[i] = reinterpret_cast<const uint32_t*>(&x[i])[j];
-            yp[j] = lut_eval_big<K <= 6 ? 7 : K>(t4, xs);
-        }
-    }
-    sl[(size_t)(d.z >> 16) * V + v] = y;
+    uint4* dst = sl + (size_t)(d.z >> 16) * V + v;
+    uint4* qd = nullptr;
     if (HASQ) {
         const uint32_t reg = d.w >> 4;
-        if (reg) sl[(size_t)(q0 + reg - 1 + qnext) * V + v] = y;      // fused latch
+        if (reg) qd = sl + (size_t)(q0 + reg - 1 + qnext) * V + v;     // fused latch
+    }
+    if constexpr (K <= 4) {
+        const LutMasks<K> mk = lut_masks<K>(t4[0]);
+        uint4 x[P][K];
+#pragma unroll
+        for (int p = 0; p < P; ++p)
+#pragma unroll
+            for (int i = 0; i < K; ++i) x[p][i] = sl[(size_t)s[i] * V + v + p * VS];
+#pragma unroll
+        for (int p = 0; p < P; ++p) {
+            const uint4 y = lut_eval4_m<K>(mk, x[p]);
+            dst[p * VS] = y;
+            if (HASQ && qd) qd[p * VS] = y;
+        }
+    } else {
+#pragma unroll 1
+        for (int p = 0; p < P; ++p) {
+            uint4 x[K];
+#pragma unroll
+            for (int i = 0; i < K; ++i) x[i] = sl[(size_t)s[i] * V + v + p * VS];
+            uint4 y;
+            if (K <= 6) {
+                y = lut_eval4<K <= 6 ? K : 6>(t4[0], x);
+            } else {
+                uint32_t xs[8];
+                uint32_t* yp = reinterpret_cast<uint32_t*>(&y);
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+#pragma unroll
+                    for (int i = 0; i < K; ++i) xs[i] = reinterpret_cast<const uint32_t*>(&x[i])[j];
+                    yp[j] = lut_eval_big<K <= 6 ? 7 : K>(t4, xs);
+                }
+            }
+            dst[p * VS] = y;
+            if (HASQ && qd) qd[p * VS] = y;
+        }
     }
 }
 
@@ -110,15 +133,17 @@ __device__ __forceinline__ void group_sync(uint32_t id, uint32_t nthreads) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-// TW = 32-bit words per slot (tile = 32 * TW lanes).  A thread evaluates one gate on one
-// 16-byte group of 4 words (128 lanes): k 16-byte shared-memory loads, 4 x (2^k - 1) LOP3,
-// one 16-byte store.  The CTA (TILE_CTA threads) is split into NG independent groups; each
+// TW = 32-bit words per slot (tile = 32 * TW lanes).  A thread evaluates one gate on P
+// 16-byte groups of 4 words (128 lanes each; P = TILE_VPT when TW >= 16): P*k 16-byte
+// shared-memory loads, P*4*(2^k - 1) LOP3, P 16-byte stores.  The CTA (TILE_CTA threads) is split into NG independent groups; each
 // group simulates its own tile and synchronises only with itself (named barrier 1 + gid),
 // so one group's level barrier overlaps the other groups' work.  All groups share the
 // descriptor table in shared memory.
 template <int TW, bool HASQ, int NG, int DM>
 __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     constexpr uint32_t V = TW / 4;                       // uint4 per slot
+    constexpr uint32_t P = V >= 4 ? TILE_VPT : 1;        // 16-byte vectors per thread and gate
+    constexpr uint32_t VS = V / P;                       // threads per gate (vector stride)
     constexpr uint32_t GT = TILE_CTA / NG;               // threads per group
     extern __shared__ uint4 smem[];
     const uint4* dsm = DM == 1 ? smem : reinterpret_cast<const uint4*>(a.desc);
@@ -191,7 +216,6 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
         group_sync(bar, GT);
         for (uint32_t c = 0; c < a.ncycles; ++c) {
             const unsigned long long cyc = c0 + c;
-            constexpr uint32_t qcur = 0u;
             const uint32_t qnext = R;
             // ---- primary inputs of this cycle (R2): one 64-bit hash per pair of words
             for (uint32_t u = tid; u < a.n_pi * (TW / 2); u += bd) {
@@ -209,7 +233,7 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
             group_sync(bar, GT);
             // ---- levels: every (gate, 16-byte group) unit of the level, then a barrier
             for (uint32_t l = 0; l < a.n_levels; ++l) {
-                const uint32_t g0 = lvl[l], n = (lvl[l + 1] - g0) * V;
+                const uint32_t g0 = lvl[l], n = (lvl[l + 1] - g0) * VS;
                 const uint4* dl = dsm + g0;
                 if (DM == 2) {
                     const uint32_t b = step & 1;
@@ -223,18 +247,21 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
                     ++step;
                 }
                 for (uint32_t u = tid; u < n; u += bd) {
-                    const uint32_t gi = u / V, v = u % V;
+                    const uint32_t gi = u / VS, v = u % VS;
                     const uint32_t g = g0 + gi;
                     const uint4 d = dl[gi];
-                    switch (d.w & 15u) {                       // k: warp-uniform except at k-group edges
-                        case 1: tile_gate<1, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        case 2: tile_gate<2, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        case 3: tile_gate<3, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        case 4: tile_gate<4, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        case 5: tile_gate<5, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        case 6: tile_gate<6, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        case 7: tile_gate<7, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
-                        default: tile_gate<8, HASQ>(sl, V, v, d, a.desc_hi, g, q0, R, qcur, qnext); break;
+                    // k: warp-uniform except at k-group edges; the common 2-4-input gates are
+                    // tested first (a compare and branch each instead of the jump table)
+                    const uint32_t k = d.w & 15u;
+                    if (k == 2) tile_gate<2, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext);
+                    else if (k == 3) tile_gate<3, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext);
+                    else if (k == 4) tile_gate<4, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext);
+                    else switch (k) {
+                        case 1: tile_gate<1, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext); break;
+                        case 5: tile_gate<5, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext); break;
+                        case 6: tile_gate<6, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext); break;
+                        case 7: tile_gate<7, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext); break;
+                        default: tile_gate<8, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext); break;
                     }
                 }
                 group_sync(bar, GT);
