@@ -345,14 +345,16 @@ def test_lane_slabs_do_not_change_results(slabs):
         assert np.array_equal(a[key], b[key]), key
 
 
+@pytest.mark.parametrize("lanes", [8192, 65536])
 @pytest.mark.parametrize("flags", [gs.GS_SIM_NO_PDL, 2, 6, 8])
-def test_launch_and_cache_options_do_not_change_results(flags):
-    """PDL off, L2 eviction hints on stores, hints on stores and loads: bit-identical."""
+def test_launch_and_cache_options_do_not_change_results(flags, lanes):
+    """PDL off, L2 eviction hints on stores, hints on stores and loads, no grid stride:
+    bit-identical (8,192 lanes: one 16-byte vector per thread; 65,536: four, as on C4)."""
     cfg = workloads.CONFIGS["C3"]
     nl = cfg.netlist()
     prog = compile_nl(nl)
-    a = run_gpu(nl, 8192, 20, "lut", seed=4, prog=prog)
-    b = run_gpu(nl, 8192, 20, "lut", seed=4, prog=prog, flags=flags)
+    a = run_gpu(nl, lanes, 20, "lut", seed=4, prog=prog)
+    b = run_gpu(nl, lanes, 20, "lut", seed=4, prog=prog, flags=flags)
     for key in ("outputs", "regs", "sigs"):
         assert np.array_equal(a[key], b[key]), key
 
