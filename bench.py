@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab", "df", "tile"])
     ap.add_argument("--tile-words", type=int, default=0, help="kernel T: 32-bit words per slot")
     ap.add_argument("--tile-groups", type=int, default=0, help="kernel T: thread groups per CTA")
+    ap.add_argument("--tile-slots-global", action="store_true",
+                    help="kernel T: live slots in the workspace (L1/L2) instead of shared memory")
     ap.add_argument("--df-interleave", type=int, default=0, help="kernel D: slabs walked together")
     ap.add_argument("--df-gpw", type=int, default=0, help="kernel D: gates per warp per item")
     ap.add_argument("--lane-slabs", type=int, default=0, help="L2 lane slabs (0 = library default)")
@@ -269,7 +271,7 @@ def main():
                  df_interleave=args.df_interleave, df_gates_per_warp=args.df_gpw, pdl=not args.no_pdl,
                  tile_words=args.tile_words, tile_groups=args.tile_groups, lane_groups=args.lane_groups,
                  flags=(2 if args.l2_hints >= 1 else 0) | (4 if args.l2_hints >= 2 else 0) |
-                 (8 if args.no_grid_stride else 0) |
+                 (8 if args.no_grid_stride else 0) | (256 if args.tile_slots_global else 0) |
                  {"auto": 0, "on": 64, "off": 128}[args.lut_bulk])
     sim.bind_generated(cfg.stim_seed)
     C = args.cycles_per_step
@@ -402,7 +404,8 @@ def main():
                        "lane_groups": sim.config["lane_groups"],
                        "df_interleave": args.df_interleave, "df_gpw": args.df_gpw,
                        "pdl": not args.no_pdl, "tile_words": args.tile_words,
-                       "tile_groups": args.tile_groups, "l2_hints": args.l2_hints, "lut_k": args.lut_k,
+                       "tile_groups": args.tile_groups, "tile_slots_global": args.tile_slots_global,
+                       "l2_hints": args.l2_hints, "lut_k": args.lut_k,
                        "grid_stride": not args.no_grid_stride,
                        "l2": "inputs larger than L2 (state %.1f GB per GPU)" % (info["n_rows"] * lanes / 8 / 1e9),
                        "step": f"{C} cycles over every lane of the GPU" + (

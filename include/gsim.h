@@ -283,6 +283,11 @@ typedef struct {
  * or never.  Default: never (measured slower than the register gathers on C3-C5). */
 #define GS_SIM_LUT_BULK 64u
 #define GS_SIM_LUT_NO_BULK 128u
+/* flags (kernel T): keep each thread group's live slots in a private region of the device
+ * workspace (served by L1 and L2) instead of shared memory, so circuits whose live state
+ * does not fit shared memory (up to 65,535 live slots) still run tile by tile with no
+ * per-level launch; 128- or 256-lane tiles.  Default: off. */
+#define GS_SIM_TILE_SLOTS_GLOBAL 256u
 
 /* Device workspace bytes required for (prog, opts). */
 gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts, size_t* bytes);

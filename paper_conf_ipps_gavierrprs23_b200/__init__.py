@@ -28,6 +28,9 @@ GS_MAX_K_POLY = 8
 GS_SIM_NO_PDL = 1
 GS_SIM_LUT_BULK = 64          # kernel A: bulk-copy staged gathers on (where eligible)
 GS_SIM_LUT_NO_BULK = 128      # ... off
+GS_SIM_TILE_DESC_GLOBAL = 16  # kernel T: descriptors read from global memory
+GS_SIM_TILE_DESC_TMA = 32     # kernel T: descriptors TMA-streamed level by level
+GS_SIM_TILE_SLOTS_GLOBAL = 256  # kernel T: live slots in the workspace (L1/L2), not shared memory
 GS_KERNEL_AUTO, GS_KERNEL_LUT, GS_KERNEL_POLY, GS_KERNEL_AB, GS_KERNEL_DATAFLOW = 0, 1, 2, 3, 4
 GS_KERNEL_TILE = 5
 KERNELS = {"auto": 0, "lut": 1, "A": 1, "poly": 2, "B": 2, "ab": 3, "AB": 3, "df": 4, "dataflow": 4,

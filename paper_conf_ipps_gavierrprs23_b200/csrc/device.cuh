@@ -41,6 +41,17 @@ __device__ __forceinline__ void st_hint(uint4* ptr, const uint4& v, uint64_t pol
                  "r"(v.z), "r"(v.w), "l"(pol)
                  : "memory");
 }
+// the same store under an explicit predicate operand (no fused latch: store nothing).  A
+// C-level `if (qd) st_hint(qd + u * 32, ...)` was compiled into an unconditional store: the
+// pointer arithmetic let the compiler assume qd != nullptr (compute-sanitizer: 16-byte writes
+// to addresses 0x0 / 0x200 in k_level_lut_wide<4, true> on C4).
+__device__ __forceinline__ void st_hint_if(uint4* ptr, const uint4& v, uint64_t pol, uint32_t pred) {
+    asm volatile(
+        "{\n .reg .pred p;\n setp.ne.u32 p, %6, 0;\n"
+        " @p st.global.L2::cache_hint.v4.u32 [%0], {%1, %2, %3, %4}, %5;\n}\n" ::"l"(ptr),
+        "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "l"(pol), "r"(pred)
+        : "memory");
+}
 __device__ __forceinline__ uint4 ld_hint(const uint4* ptr, uint64_t pol) {
     uint4 v;
     asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0, %1, %2, %3}, [%4], %5;"

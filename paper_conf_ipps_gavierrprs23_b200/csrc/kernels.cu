@@ -172,8 +172,10 @@ __device__ __forceinline__ void lut_gate_u(const LevelArgs& a, uint32_t gate, ui
 #pragma unroll
         for (int i = 0; i < K; ++i) x[u][i] = (HINT && a.hint_ld) ? ld_hint(src[i] + u * 32, pf) : __ldg(src[i] + u * 32);
     uint4* dst = reinterpret_cast<uint4*>(a.state + (uint64_t)(a.row_gate0 + gate) * a.stride) + v0;
-    uint4* qd = qdst != 0xFFFFFFFFu ? reinterpret_cast<uint4*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride) + v0
-                                    : nullptr;
+    // fused latch target: a boolean, never a null pointer plus an offset (the compiler may
+    // assume such a pointer non-null and drop the test; seen with the L2-hint stores)
+    const bool latch = qdst != 0xFFFFFFFFu;
+    uint4* qd = reinterpret_cast<uint4*>(a.state + (uint64_t)((latch ? qdst : 0u) + a.qnext) * a.stride) + v0;
     uint64_t po = 0;
     if (HINT) po = hot ? l2_policy_last() : pf;
 #pragma unroll
@@ -181,10 +183,10 @@ __device__ __forceinline__ void lut_gate_u(const LevelArgs& a, uint32_t gate, ui
         const uint4 y = lut_eval4<K>(tt, x[u]);
         if (HINT) {
             st_hint(dst + u * 32, y, po);
-            if (qd) st_hint(qd + u * 32, y, pf);
+            st_hint_if(qd + u * 32, y, pf, latch);
         } else {
             dst[u * 32] = y;
-            if (qd) qd[u * 32] = y;
+            if (latch) qd[u * 32] = y;
         }
     }
 }
@@ -270,7 +272,8 @@ __device__ __forceinline__ void mbar_wait_d(uint64_t* bar, uint32_t parity) {
 }
 
 template <int K, int C>
-__device__ __forceinline__ void bulk_eval(const uint4* stage, uint8_t* dst, uint8_t* qd, uint64_t tt, uint32_t t) {
+__device__ __forceinline__ void bulk_eval(const uint4* stage, uint8_t* dst, uint8_t* qd, bool latch, uint64_t tt,
+                                          uint32_t t) {
 #pragma unroll
     for (uint32_t v = t; v < C / 16; v += 256) {
         uint4 x[K];
@@ -278,7 +281,7 @@ __device__ __forceinline__ void bulk_eval(const uint4* stage, uint8_t* dst, uint
         for (int i = 0; i < K; ++i) x[i] = stage[i * (C / 16) + v];
         const uint4 y = lut_eval4<K>(tt, x);
         reinterpret_cast<uint4*>(dst)[v] = y;
-        if (qd) reinterpret_cast<uint4*>(qd)[v] = y;
+        if (latch) reinterpret_cast<uint4*>(qd)[v] = y;
     }
 }
 
@@ -360,13 +363,14 @@ __global__ void __launch_bounds__(BULK_THREADS, MINB) k_level_bulk(LevelArgs a, 
         const uint32_t gate = a.g0 + (it >> cpg_shift);
         const uint64_t off = byte0 + (uint64_t)(it & cmask) * C;
         uint8_t* dst = a.state + (uint64_t)(a.row_gate0 + gate) * a.stride + off;
-        uint8_t* qd = h.z != 0xFFFFFFFFu ? a.state + (uint64_t)(h.z + a.qnext) * a.stride + off : nullptr;
+        const bool latch = h.z != 0xFFFFFFFFu;             // (never a null pointer + offset)
+        uint8_t* qd = a.state + (uint64_t)((latch ? h.z : 0u) + a.qnext) * a.stride + off;
         const uint4* st = buf + s * 4 * (C / 16);
         switch (h.w) {
-            case 1: bulk_eval<1, C>(st, dst, qd, tt, t); break;
-            case 2: bulk_eval<2, C>(st, dst, qd, tt, t); break;
-            case 3: bulk_eval<3, C>(st, dst, qd, tt, t); break;
-            default: bulk_eval<4, C>(st, dst, qd, tt, t); break;
+            case 1: bulk_eval<1, C>(st, dst, qd, latch, tt, t); break;
+            case 2: bulk_eval<2, C>(st, dst, qd, latch, tt, t); break;
+            case 3: bulk_eval<3, C>(st, dst, qd, latch, tt, t); break;
+            default: bulk_eval<4, C>(st, dst, qd, latch, tt, t); break;
         }
         __syncwarp();
         if (lane == 0)
@@ -532,13 +536,15 @@ __device__ __forceinline__ void df_gate(const DfArgs& a, uint32_t gate, uint4 in
 #pragma unroll
         for (int i = 0; i < K; ++i) x[u][i] = __ldcg(src[i] + u * LPG);
     uint4* dst = reinterpret_cast<uint4*>(a.state + (uint64_t)(a.row_gate0 + gate) * a.stride) + v0;
-    uint4* qd = qdst != 0xFFFFFFFFu ? reinterpret_cast<uint4*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride) + v0
-                                    : nullptr;
+    // fused latch target: a boolean, never a null pointer plus an offset (the compiler may
+    // assume such a pointer non-null and drop the test; seen with the L2-hint stores)
+    const bool latch = qdst != 0xFFFFFFFFu;
+    uint4* qd = reinterpret_cast<uint4*>(a.state + (uint64_t)((latch ? qdst : 0u) + a.qnext) * a.stride) + v0;
 #pragma unroll
     for (int u = 0; u < VPT; ++u) {
         const uint4 y = lut_eval4<K>(tt, x[u]);
         dst[u * LPG] = y;
-        if (qd) qd[u * LPG] = y;
+        if (latch) qd[u * LPG] = y;
     }
 }
 

@@ -101,7 +101,8 @@ struct TileArgs {
     const uint32_t* level_off;        // [n_levels + 1]
     uint32_t n_eval, n_levels;
     uint32_t desc_smem;               // 0: descriptors read from global; 1: resident in shared
-                                      // memory; 2: TMA-streamed level by level (double buffer)
+                                      // memory; 2: TMA-streamed level by level (double buffer);
+                                      // | 4: slots in global memory instead of shared memory
     uint32_t max_width;               // widest level (mode 2 buffer size, in descriptors)
     const uint32_t* po_slot;
     uint32_t n_po;
@@ -122,6 +123,7 @@ struct TileArgs {
     uint32_t ntw, trace_cap;
     uint64_t word_off;                // global 64-bit word of local lane 0
     uint32_t ncycles, n_tiles;
+    uint4* gslots;                    // desc_smem & 4: per-group slot regions [grid*NG][n_slots][TW/4]
 };
 size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
                        int desc_mode, uint32_t max_width);

@@ -8,7 +8,9 @@ static size_t lvl_bytes(uint32_t n_levels) { return (((size_t)n_levels + 1) * 4 
 
 size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
                        int desc_mode, uint32_t max_width) {
-    size_t b = 0, g = ((size_t)n_slots + 64) * 4 * tw;
+    const bool sg = (desc_mode & 4) != 0;                // slots in global memory: MISR only
+    desc_mode &= 3;
+    size_t b = 0, g = ((sg ? 0 : (size_t)n_slots) + 64) * 4 * tw;
     if (desc_mode == 1) b = (size_t)n_eval * 16 + lvl_bytes(n_levels);
     if (desc_mode == 2) {
         b = lvl_bytes(n_levels);

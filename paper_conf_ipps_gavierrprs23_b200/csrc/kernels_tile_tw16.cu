@@ -7,7 +7,8 @@ namespace gs {
     switch (dm) {                             \
         case 0: CALL(Q, G, 0); break;         \
         case 1: CALL(Q, G, 1); break;         \
-        default: CALL(Q, G, 2); break;        \
+        case 2: CALL(Q, G, 2); break;         \
+        default: return cudaErrorInvalidValue; \
     }
 #define TILE_QG(CALL)                                                                      \
     switch ((has_q ? 8 : 0) + (ng == 1 ? 0 : ng == 2 ? 1 : ng == 4 ? 2 : 7)) {             \

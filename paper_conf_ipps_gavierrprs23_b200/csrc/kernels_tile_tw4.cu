@@ -7,7 +7,10 @@ namespace gs {
     switch (dm) {                             \
         case 0: CALL(Q, G, 0); break;         \
         case 1: CALL(Q, G, 1); break;         \
-        default: CALL(Q, G, 2); break;        \
+        case 2: CALL(Q, G, 2); break;         \
+        case 4: CALL(Q, G, 4); break;         \
+        case 5: CALL(Q, G, 5); break;         \
+        default: CALL(Q, G, 6); break;        \
     }
 #define TILE_QG(CALL)                                                                      \
     switch ((has_q ? 8 : 0) + (ng == 1 ? 0 : ng == 2 ? 1 : ng == 4 ? 2 : 7)) {             \

@@ -24,7 +24,7 @@ size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 struct Layout {
     size_t ctl, state, din, aux, dhi, dtt, term_off, terms, po_rows, latch_src, latch_dst, reg_init,
         trace_slot, misr, trace, lane_sigs, scratch, lv_gate0, lv_item0, dfctl, dfctl_bytes,
-        t_desc, t_desc_hi, t_po, t_lsrc, t_ldst, t_wbrow, t_wbslot, t_lvl, total;
+        t_desc, t_desc_hi, t_po, t_lsrc, t_ldst, t_wbrow, t_wbslot, t_lvl, t_gslots, total;
 };
 
 // Work-item plan of the DATAFLOW schedule (kernels.cu k_dataflow): non-empty levels only
@@ -106,6 +106,7 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
     // circuit runs 1.33x faster with TMA and 4x wider tiles than resident with narrow
     // ones), then wider tiles, then resident > TMA stream > global, then fewer groups
     const int forced = (o.flags & GS_SIM_TILE_DESC_GLOBAL) ? 0 : (o.flags & GS_SIM_TILE_DESC_TMA) ? 2 : -1;
+    const int sg = (o.flags & GS_SIM_TILE_SLOTS_GLOBAL) ? 4 : 0;   // slots in global memory
     uint64_t best = 0;
     for (int ds : {1, 2, 0}) {
         if (forced >= 0 && ds != forced) continue;
@@ -113,12 +114,13 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
             if (o.tile_groups && ng != o.tile_groups) continue;
             for (uint32_t tw : {4u, 8u, 16u, 32u, 64u}) {
                 if (o.tile_words && tw != o.tile_words) continue;
-                if (o.lanes % (32ull * tw) || smem(tw, ng, ds) > TILE_SMEM_MAX) continue;
+                if (sg && tw > 8) continue;                  // global slots: 16/32-byte slot rows
+                if (o.lanes % (32ull * tw) || smem(tw, ng, ds | sg) > TILE_SMEM_MAX) continue;
                 const uint64_t inflight = std::min<uint64_t>((uint64_t)ng * tw * 32 * sms, o.lanes);
                 const uint64_t pref = ds == 1 ? 2 : ds == 2 ? 1 : 0;
                 const uint64_t score = ((inflight << (ds == 1 ? 1 : 0)) << 24) | ((uint64_t)tw << 16) | (pref << 12) |
                                        ((8 - ng) << 8);
-                if (score > best) { best = score; pl.tw = tw; pl.ng = ng; pl.desc_smem = ds; }
+                if (score > best) { best = score; pl.tw = tw; pl.ng = ng; pl.desc_smem = ds | sg; }
             }
         }
     }
@@ -193,6 +195,9 @@ Layout make_layout(const Program& p, const gs_sim_opts& o, const Plans& pl) {
     L.t_wbrow = take(t.wb_row.size() * 4);
     L.t_wbslot = take(t.wb_slot.size() * 4);
     L.t_lvl = take(pl.tw ? p.level_off.size() * 4 : 0);
+    // kernel T with global slots: one region of n_slots x tile bytes per tile (an upper bound
+    // on the resident groups) = n_slots x lanes / 8 bytes
+    L.t_gslots = take((pl.desc_smem & 4) ? (size_t)t.n_slots * (size_t)(o.lanes / 8) : 0);
     L.total = off;
     return L;
 }
@@ -366,6 +371,7 @@ static cudaError_t tile_launch(const gs_sim* s, uint32_t ncycles, cudaStream_t s
     a.n_levels = p.n_levels;
     a.desc_smem = (uint32_t)s->desc_smem;
     a.max_width = s->tile_max_width;
+    a.gslots = s->at<uint4>(s->L.t_gslots);
     a.po_slot = s->at<const uint32_t>(s->L.t_po);
     a.n_po = p.n_po;
     a.latch_src = s->at<const uint32_t>(s->L.t_lsrc);

@@ -782,6 +782,38 @@ def test_tile_descriptor_sources_global_and_tma_stream(flags):
     sim.close()
 
 
+@pytest.mark.parametrize("flags", [gs.GS_SIM_TILE_SLOTS_GLOBAL, gs.GS_SIM_TILE_SLOTS_GLOBAL | 16,
+                                   gs.GS_SIM_TILE_SLOTS_GLOBAL | 32])
+@pytest.mark.parametrize("tw", [4, 8])
+def test_tile_global_slots_vs_oracle(flags, tw):
+    """Kernel T with the live slots in global memory (L1/L2) instead of shared memory, each
+    descriptor source, 128- and 256-lane tiles: every lane vs the oracle on a sequential
+    circuit too large for shared-memory slots, steps split over several launches, and the
+    register / tiny wide-gate edge cases."""
+    nl = workloads.synthetic(60000, 2400, 64, 64, 36, seed=31, name="g60k")
+    prog = compile_nl(nl)
+    lanes = 4096
+    with pytest.raises(gs.GsError):                    # the shared-memory plan cannot hold it
+        gs.Sim(prog, lanes, kernel="tile", tile_words=tw).close()
+    sim = gs.Sim(prog, lanes, kernel="tile", flags=flags, tile_words=tw, trace_words=[0, 63], trace_cycles=12)
+    sim.bind_generated(7)
+    for n in (1, 4, 7):
+        sim.step(n)
+    o = oracle.simulate(nl, np.arange(lanes), 12, seed=7)
+    assert np.array_equal(sim.read_lane_signatures(), o["sig"])
+    assert np.array_equal(gs.unpack_lanes(sim.read_registers()).T, o["regs"])
+    assert np.array_equal(gs.unpack_lanes(sim.read_outputs()).T, o["last"])
+    rows = np.concatenate([np.arange(0, 64), np.arange(63 * 64, 64 * 64)])
+    assert np.array_equal(gpu_trace_bits(sim.read_trace(), None), o["trace"][rows])
+    sim.close()
+    for nl in (workloads.random_tiny(3, n_pi=6, n_reg=5, n_gates=300, n_po=12, max_k=6),
+               workloads.register_edge_cases(), workloads.probes_circuit()):
+        r = run_gpu(nl, 1024, 40, "tile", seed=3, tile_words=tw, flags=flags)
+        o = oracle.simulate(nl, np.arange(1024), 40, seed=3)
+        assert np.array_equal(r["sigs"], o["sig"])
+        assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"])
+
+
 def test_auto_kernel_selection():
     """AUTO = kernel T (one launch per step) when the circuit fits shared memory, else A."""
     for name, lanes, tile, L in (("C1", 1024, True, 0), ("C2", 1 << 14, True, 0), ("C3", 4096, False, 0),
