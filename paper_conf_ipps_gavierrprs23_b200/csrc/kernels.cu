@@ -693,7 +693,8 @@ cudaError_t launch_dataflow(const DfArgs& a, uint32_t grid, cudaStream_t s) {
 //                  |S|, so "> |S| - 1" is "== |S|");
 //   output neuron  acc += w_S h_S: a two's-complement accumulator of B bit-planes
 //                  (|acc| <= sum |w_S| <= 3^k: B = 8 for k <= 4, 16 for k <= 8), the
-//                  constant w_S added under the mask h_S by a ripple of full adders.
+//                  constant w_S added under the mask h_S one set bit of |w_S| at a time
+//                  (half-adder / half-subtractor ripples that stop once no lane carries).
 // The gate's output is [acc == 1]; lanes with acc outside {0, 1} are counted (P:224 says
 // there are none).  check_only: compare with the row kernel A wrote (GS_KERNEL_AB).
 template <int B, int KMAX>
@@ -713,28 +714,51 @@ __device__ __forceinline__ void poly_word(const LevelArgs& a, uint32_t gate, uin
         const uint32_t S = tm & 0xFFu;                          // monomial S (bit s <-> x_s)
         const uint32_t nS = (uint32_t)((int)(int8_t)((tm >> 8) & 0xFFu) + 1);   // |S| (bias + 1, Eq. 3)
         const int w = (int)(int16_t)(tm >> 16);                 // w_S (Eq. 1)
-        // hidden neuron: bit-sliced sum of the selected inputs, then the threshold
-        uint32_t c0 = 0u, c1 = 0u, c2 = 0u, c3 = 0u;
+        // hidden neuron: bit-sliced sum of the selected inputs (4-plane counter; a carry
+        // ripple stops as soon as no lane carries), then the threshold "sum > |S| - 1"
+        uint32_t c[4] = {0u, 0u, 0u, 0u};
 #pragma unroll
         for (int i = 0; i < KMAX; ++i) {
             if ((S >> i) & 1u) {
-                uint32_t cy = x[i], t;
-                t = c0 & cy; c0 ^= cy; cy = t;
-                t = c1 & cy; c1 ^= cy; cy = t;
-                t = c2 & cy; c2 ^= cy; cy = t;
-                c3 ^= cy;
+                uint32_t cy = x[i];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const uint32_t t = c[q] & cy;
+                    c[q] ^= cy;
+                    cy = t;
+                    if (!cy) break;
+                }
             }
         }
-        const uint32_t h = ((nS & 1u) ? c0 : ~c0) & ((nS & 2u) ? c1 : ~c1) & ((nS & 4u) ? c2 : ~c2) &
-                           ((nS & 8u) ? c3 : ~c3);
-        // output neuron: acc += w_S * h_S (two's complement, masked constant add)
-        uint32_t carry = 0u;
+        // the sum cannot exceed |S|, so "> |S| - 1" is "== |S|": compare the planes with |S|
+        const uint32_t h = ~((c[0] ^ (0u - (nS & 1u))) | (c[1] ^ (0u - ((nS >> 1) & 1u))) |
+                             (c[2] ^ (0u - ((nS >> 2) & 1u))) | (c[3] ^ (0u - ((nS >> 3) & 1u))));
+        // output neuron: acc += w_S * h_S in two's complement (mod 2^B): for every set bit p
+        // of |w_S|, add (w_S > 0) or subtract (w_S < 0) the mask h at plane p, rippling the
+        // carry / borrow upward only while some lane still carries
+        const uint32_t aw = (uint32_t)(w < 0 ? -w : w);
+        for (uint32_t m = aw; m; m &= m - 1) {
+            const int pb = __ffs(m) - 1;
+            uint32_t cy = h;
+            if (w > 0) {
 #pragma unroll
-        for (int b = 0; b < B; ++b) {
-            const uint32_t add = ((w >> b) & 1) ? h : 0u;
-            const uint32_t sum = acc[b] ^ add ^ carry;
-            carry = (acc[b] & add) | (carry & (acc[b] ^ add));
-            acc[b] = sum;
+                for (int b = 0; b < B; ++b) {
+                    if (b < pb) continue;
+                    const uint32_t t = acc[b] & cy;
+                    acc[b] ^= cy;
+                    cy = t;
+                    if (!cy) break;
+                }
+            } else {
+#pragma unroll
+                for (int b = 0; b < B; ++b) {
+                    if (b < pb) continue;
+                    const uint32_t t = ~acc[b] & cy;
+                    acc[b] ^= cy;
+                    cy = t;
+                    if (!cy) break;
+                }
+            }
         }
     }
     uint32_t hi = 0u;
