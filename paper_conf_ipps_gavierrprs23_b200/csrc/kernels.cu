@@ -882,10 +882,10 @@ __global__ void __launch_bounds__(256) k_end_cycle(EndArgs a, uint32_t latch_blo
         if (t < (uint64_t)64 * a.words) {
             const uint32_t j = (uint32_t)(t / a.words), w = (uint32_t)(t - (uint64_t)j * a.words);
             const int32_t slot = (a.trace && c < a.trace_cap) ? __ldg(a.trace_slot + w) : -1;
-            unsigned long long* sink = nullptr;                  // full per-cycle output stream
-            if (a.ctl->sink_ptr && c - a.ctl->sink_base < a.ctl->sink_cycles)
-                sink = reinterpret_cast<unsigned long long*>(a.ctl->sink_ptr) +
-                       (c - a.ctl->sink_base) * a.n_po * (uint64_t)a.words;
+            // full per-cycle output stream: a boolean, never a null pointer plus an offset
+            const bool to_sink = a.ctl->sink_ptr && c - a.ctl->sink_base < a.ctl->sink_cycles;
+            unsigned long long* sink = reinterpret_cast<unsigned long long*>(a.ctl->sink_ptr) +
+                                       (to_sink ? (c - a.ctl->sink_base) * a.n_po * (uint64_t)a.words : 0ull);
             unsigned long long v = 0;
             for (uint32_t o = j; o < a.n_po; o += 64) {
                 const uint32_t row = resolve(__ldg(a.po_rows + o), a.qcur);
@@ -893,7 +893,7 @@ __global__ void __launch_bounds__(256) k_end_cycle(EndArgs a, uint32_t latch_blo
                 v ^= x;
                 pop += __popcll(x);
                 if (slot >= 0) a.trace[((uint64_t)c * a.n_po + o) * a.ntw + slot] = x;
-                if (sink) sink[(uint64_t)o * a.words + w] = x;
+                if (to_sink) sink[(uint64_t)o * a.words + w] = x;
             }
             const unsigned long long prev = j ? a.misr_cur[(uint64_t)(j - 1) * a.words + w] : 0ULL;
             const unsigned long long fb = ((MISR_POLY >> j) & 1ULL) ? a.misr_cur[(uint64_t)63 * a.words + w] : 0ULL;

@@ -288,10 +288,10 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
                 const uint32_t j = u / TW, w = u % TW;
                 const uint32_t g32 = t0 + w;
                 const int32_t tslot = tr ? __ldg(a.trace_slot + (g32 >> 1)) : -1;
-                uint32_t* sink = nullptr;                          // full per-cycle output stream
-                if (a.ctl->sink_ptr && cyc - a.ctl->sink_base < a.ctl->sink_cycles)
-                    sink = reinterpret_cast<uint32_t*>(a.ctl->sink_ptr) +
-                           (cyc - a.ctl->sink_base) * a.n_po * (uint64_t)w32_row;
+                // full per-cycle output stream: a boolean, never a null pointer plus an offset
+                const bool to_sink = a.ctl->sink_ptr && cyc - a.ctl->sink_base < a.ctl->sink_cycles;
+                uint32_t* sink = reinterpret_cast<uint32_t*>(a.ctl->sink_ptr) +
+                                 (to_sink ? (cyc - a.ctl->sink_base) * a.n_po * (uint64_t)w32_row : 0ull);
                 uint32_t vv = 0;
                 for (uint32_t o = j; o < a.n_po; o += 64) {
                     const uint32_t x = sw[(size_t)__ldg(a.po_slot + o) * TW + w];
@@ -300,7 +300,7 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
                     if (tslot >= 0)
                         reinterpret_cast<uint32_t*>(a.trace)[(((uint64_t)cyc * a.n_po + o) * a.ntw + tslot) * 2 +
                                                              (g32 & 1)] = x;
-                    if (sink) sink[(uint64_t)o * w32_row + g32] = x;
+                    if (to_sink) sink[(uint64_t)o * w32_row + g32] = x;
                 }
                 const uint32_t prev = j ? mp[(j - 1) * TW + w] : 0u;
                 const uint32_t fb = ((TILE_MISR_POLY >> j) & 1ULL) ? mp[63 * TW + w] : 0u;
