@@ -4,6 +4,8 @@ Every comparison is element by element on the same seeded inputs; the oracle nev
 sees anything the GPU produced.  Closed forms (a+b, a*b, LFSR, counters) are checked
 on ALL lanes where the oracle would be too slow.
 """
+import os
+
 import numpy as np
 import pytest
 
@@ -895,7 +897,7 @@ def _fuzz_netlist(rng, case):
                                  n_po=n_po, max_k=max_k)
 
 
-@pytest.mark.parametrize("case", range(32))
+@pytest.mark.parametrize("case", range(int(os.environ.get("GS_FUZZ_CASES", "32"))))
 def test_fuzz_every_kernel_all_lanes_vs_oracle(case):
     """Seeded random netlists through every kernel / schedule / compile option, every lane and
     cycle against the oracle (outputs of the last cycle, registers, per-lane signatures)."""
@@ -911,11 +913,24 @@ def test_fuzz_every_kernel_all_lanes_vs_oracle(case):
     o = oracle.simulate(nl, np.arange(lanes) + offset, cycles, seed=seed, want=("last", "regs", "sig"))
     kernels = ["lut", "poly", "ab", "auto"] + (["tile"] if lanes % 128 == 0 else []) + \
         (["df"] if lanes % 4096 == 0 else [])
-    for kernel in kernels:
-        r = run_gpu(nl, lanes, cycles, kernel, seed=seed, prog=prog, lane_offset=offset)
-        assert np.array_equal(gs.unpack_lanes(r["outputs"]).T, o["last"]), kernel
-        assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"]), kernel
-        assert np.array_equal(r["sigs"], o["sig"]), kernel
+    runs = [(k, {}) for k in kernels]
+    # opt-in launch / cache / schedule options: one random pick per case for kernel A, and
+    # kernel T with global-memory slots where its 16-bit slot ids suffice
+    opt = [dict(flags=gs.GS_SIM_NO_PDL), dict(flags=2), dict(flags=6), dict(flags=8),
+           dict(flags=gs.GS_SIM_LUT_BULK), dict(lane_groups=1)][case % 6]
+    runs.append(("lut", opt))
+    if lanes % 128 == 0:
+        try:
+            prog.tile_slots()
+            runs.append(("tile", dict(flags=gs.GS_SIM_TILE_SLOTS_GLOBAL, tile_words=4)))
+        except gs.GsError:
+            pass
+    for kernel, kw in runs:
+        r = run_gpu(nl, lanes, cycles, kernel, seed=seed, prog=prog, lane_offset=offset, **kw)
+        tag = f"{kernel} {kw}"
+        assert np.array_equal(gs.unpack_lanes(r["outputs"]).T, o["last"]), tag
+        assert np.array_equal(gs.unpack_lanes(r["regs"]).T, o["regs"]), tag
+        assert np.array_equal(r["sigs"], o["sig"]), tag
         assert r["signature"]["ab_mismatch"] == 0 and r["signature"]["invariant_violations"] == 0
 
 
