@@ -884,6 +884,37 @@ def test_c5_shard_full_netlist_sampled_lanes():
     probe_closed_forms(nl, gs.unpack_lanes(r["outputs"]).T, cfg.cycles - 1, cfg.stim_seed, lanes, off)
 
 
+@pytest.mark.slow
+def test_c5_every_shard_sampled_lanes_sub_batches():
+    """C5's full netlist over ALL 8 shards of its 262,144-lane batch with one sim re-targeted by
+    gs_sim_set_lane_offset (the bench's sub-batch path): 32 sampled lanes per shard (256 in
+    all, shard-boundary lanes included) vs the oracle on every cycle, 20 cycles per shard."""
+    cfg = workloads.CONFIGS["C5"]
+    nl = cfg.netlist()
+    lanes = cfg.lanes // cfg.shards
+    W_ = lanes // 64
+    tw = [0, 1, W_ // 2, W_ - 1]
+    cycles = 20
+    prog = compile_nl(nl)
+    sim = gs.Sim(prog, lanes, kernel="lut", trace_words=tw, trace_cycles=cycles)
+    sim.bind_generated(cfg.stim_seed)
+    rng = np.random.default_rng(55)
+    tot = 0
+    for shard in range(cfg.shards):
+        off = shard * lanes
+        sim.set_lane_offset(off)
+        sim.step(cycles)
+        sim.sync()
+        r = dict(trace=sim.read_trace(), regs=sim.read_registers(), sigs=sim.read_lane_signatures())
+        words = rng.choice([1, W_ // 2], size=25)
+        sample = np.concatenate([[0, 63, 64, 127, lanes - 64, lanes - 2, lanes - 1],
+                                 words * 64 + rng.integers(0, 64, size=25)])
+        sampled_lane_check(nl, r, sample, off, cycles, cfg.stim_seed, tw)
+        tot = (tot + sim.signature()["lane_sig_sum"]) % (1 << 64)
+    sim.close()
+    assert tot != 0
+
+
 # ------------------------------------------------------------------ seeded fuzzing
 def _fuzz_netlist(rng, case):
     """Random sequential netlist: sizes, fan-in mix (k = 0..6, repeated inputs allowed),
