@@ -194,8 +194,12 @@ __device__ __forceinline__ void lut_gate_u(const LevelArgs& a, uint32_t gate, ui
 // Grid-stride over warp units (gate, chunk of U*32 vectors): the grid is sized to the
 // resident capacity (148 SMs x CTAs per SM, a.grid_blocks), so no level ends with a
 // partially filled wave of CTAs.
+#ifndef GS_U1_MINB
+#define GS_U1_MINB 4
+#endif
 template <int U, bool HINT>
-__global__ void __launch_bounds__(256, U > 4 ? 2 : 4) k_level_lut_wide(LevelArgs a, uint32_t cpg_shift, uint32_t vec0) {
+__global__ void __launch_bounds__(256, U > 4 ? 2 : U == 1 ? GS_U1_MINB : 4)
+    k_level_lut_wide(LevelArgs a, uint32_t cpg_shift, uint32_t vec0) {
     pdl_entry();
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t total = a.ng << cpg_shift;
@@ -464,7 +468,8 @@ cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s) {
             // grid-stride at the resident capacity when the level is only a few waves deep (a
             // partial last wave would idle SMs for a large share of the launch; measured: C3
             // +8.5 %); deep levels (C4: 12 waves, C5: 41) keep one CTA per chunk (-1 % otherwise)
-            if (a.grid_blocks && blocks > a.grid_blocks && blocks <= 4 * a.grid_blocks) blocks = a.grid_blocks;
+            const uint32_t cap = U == 1 ? a.grid_blocks / 4 * GS_U1_MINB : a.grid_blocks;   // resident CTAs
+            if (cap && blocks > cap && blocks <= 4 * cap) blocks = cap;
             if (U == 8) return launch_k(k_level_lut_wide<8, false>, blocks, s, a.pdl, a, sh, a.vec0);
             if (a.hint) {
                 if (U == 4) return launch_k(k_level_lut_wide<4, true>, blocks, s, a.pdl, a, sh, a.vec0);
