@@ -705,14 +705,21 @@ cudaError_t launch_dataflow(const DfArgs& a, uint32_t grid, cudaStream_t s) {
 template <int B, int KMAX>
 __device__ __forceinline__ void poly_word(const LevelArgs& a, uint32_t gate, uint32_t j, uint32_t k, uint32_t qdst,
                                           const uint32_t* r, int check_only, uint32_t& bad) {
-    uint32_t x[KMAX];
+    // j = 64-bit word: the thread holds 64 stimuli as two 32-lane words (NW = 2), so the
+    // term decode and its branches are shared by both
+    constexpr int NW = 2;
+    uint32_t x[KMAX][NW];
 #pragma unroll
-    for (int i = 0; i < KMAX; ++i)
-        x[i] = i < (int)k ? __ldg(reinterpret_cast<const uint32_t*>(a.state + (uint64_t)resolve(r[i], a.qcur) * a.stride) + j)
-                          : 0u;
-    uint32_t acc[B];
+    for (int i = 0; i < KMAX; ++i) {
+        uint2 v = make_uint2(0u, 0u);
+        if (i < (int)k)
+            v = __ldg(reinterpret_cast<const uint2*>(a.state + (uint64_t)resolve(r[i], a.qcur) * a.stride) + j);
+        x[i][0] = v.x;
+        x[i][1] = v.y;
+    }
+    uint32_t acc[B][NW];
 #pragma unroll
-    for (int b = 0; b < B; ++b) acc[b] = 0u;
+    for (int b = 0; b < B; ++b) acc[b][0] = acc[b][1] = 0u;
     const uint32_t t0 = __ldg(a.term_off + gate), t1 = __ldg(a.term_off + gate + 1);
     for (uint32_t ti = t0; ti < t1; ++ti) {
         const uint32_t tm = __ldg(a.terms + ti);
@@ -721,72 +728,89 @@ __device__ __forceinline__ void poly_word(const LevelArgs& a, uint32_t gate, uin
         const int w = (int)(int16_t)(tm >> 16);                 // w_S (Eq. 1)
         // hidden neuron: bit-sliced sum of the selected inputs (4-plane counter; a carry
         // ripple stops as soon as no lane carries), then the threshold "sum > |S| - 1"
-        uint32_t c[4] = {0u, 0u, 0u, 0u};
+        uint32_t c[4][NW] = {{0u, 0u}, {0u, 0u}, {0u, 0u}, {0u, 0u}};
 #pragma unroll
         for (int i = 0; i < KMAX; ++i) {
             if ((S >> i) & 1u) {
-                uint32_t cy = x[i];
+                uint32_t cy0 = x[i][0], cy1 = x[i][1];
 #pragma unroll
                 for (int q = 0; q < 4; ++q) {
-                    const uint32_t t = c[q] & cy;
-                    c[q] ^= cy;
-                    cy = t;
-                    if (!cy) break;
+                    const uint32_t u0 = c[q][0] & cy0, u1 = c[q][1] & cy1;
+                    c[q][0] ^= cy0;
+                    c[q][1] ^= cy1;
+                    cy0 = u0;
+                    cy1 = u1;
+                    if (!(cy0 | cy1)) break;
                 }
             }
         }
         // the sum cannot exceed |S|, so "> |S| - 1" is "== |S|": compare the planes with |S|
-        const uint32_t h = ~((c[0] ^ (0u - (nS & 1u))) | (c[1] ^ (0u - ((nS >> 1) & 1u))) |
-                             (c[2] ^ (0u - ((nS >> 2) & 1u))) | (c[3] ^ (0u - ((nS >> 3) & 1u))));
+        const uint32_t m0 = 0u - (nS & 1u), m1 = 0u - ((nS >> 1) & 1u), m2 = 0u - ((nS >> 2) & 1u),
+                       m3 = 0u - ((nS >> 3) & 1u);
+        uint32_t h[NW];
+#pragma unroll
+        for (int n = 0; n < NW; ++n)
+            h[n] = ~((c[0][n] ^ m0) | (c[1][n] ^ m1) | (c[2][n] ^ m2) | (c[3][n] ^ m3));
         // output neuron: acc += w_S * h_S in two's complement (mod 2^B): for every set bit p
         // of |w_S|, add (w_S > 0) or subtract (w_S < 0) the mask h at plane p, rippling the
         // carry / borrow upward only while some lane still carries
         const uint32_t aw = (uint32_t)(w < 0 ? -w : w);
         for (uint32_t m = aw; m; m &= m - 1) {
             const int pb = __ffs(m) - 1;
-            uint32_t cy = h;
+            uint32_t cy0 = h[0], cy1 = h[1];
             if (w > 0) {
 #pragma unroll
                 for (int b = 0; b < B; ++b) {
                     if (b < pb) continue;
-                    const uint32_t t = acc[b] & cy;
-                    acc[b] ^= cy;
-                    cy = t;
-                    if (!cy) break;
+                    const uint32_t u0 = acc[b][0] & cy0, u1 = acc[b][1] & cy1;
+                    acc[b][0] ^= cy0;
+                    acc[b][1] ^= cy1;
+                    cy0 = u0;
+                    cy1 = u1;
+                    if (!(cy0 | cy1)) break;
                 }
             } else {
 #pragma unroll
                 for (int b = 0; b < B; ++b) {
                     if (b < pb) continue;
-                    const uint32_t t = ~acc[b] & cy;
-                    acc[b] ^= cy;
-                    cy = t;
-                    if (!cy) break;
+                    const uint32_t u0 = ~acc[b][0] & cy0, u1 = ~acc[b][1] & cy1;
+                    acc[b][0] ^= cy0;
+                    acc[b][1] ^= cy1;
+                    cy0 = u0;
+                    cy1 = u1;
+                    if (!(cy0 | cy1)) break;
                 }
             }
         }
     }
-    uint32_t hi = 0u;
+    uint32_t one[NW];
 #pragma unroll
-    for (int b = 1; b < B; ++b) hi |= acc[b];
-    const uint32_t one = acc[0] & ~hi, zero = ~(acc[0] | hi);
-    bad += __popc(~(one | zero));
-    uint32_t* out = reinterpret_cast<uint32_t*>(a.state + (uint64_t)(a.row_gate0 + gate) * a.stride) + j;
+    for (int n = 0; n < NW; ++n) {
+        uint32_t hi = 0u;
+#pragma unroll
+        for (int b = 1; b < B; ++b) hi |= acc[b][n];
+        one[n] = acc[0][n] & ~hi;
+        const uint32_t zero = ~(acc[0][n] | hi);
+        bad += __popc(~(one[n] | zero));
+    }
+    const uint2 y = make_uint2(one[0], one[1]);
+    uint2* out = reinterpret_cast<uint2*>(a.state + (uint64_t)(a.row_gate0 + gate) * a.stride) + j;
     if (check_only) {
-        const uint32_t ref = *out;
-        if (ref != one) atomicAdd(&a.ctl->ab_mismatch, (unsigned long long)__popc(ref ^ one));
+        const uint2 ref = *out;
+        const uint32_t diff = __popc(ref.x ^ y.x) + __popc(ref.y ^ y.y);
+        if (diff) atomicAdd(&a.ctl->ab_mismatch, (unsigned long long)diff);
     } else {
-        *out = one;
-        if (qdst != 0xFFFFFFFFu) reinterpret_cast<uint32_t*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride)[j] = one;
+        *out = y;
+        if (qdst != 0xFFFFFFFFu) reinterpret_cast<uint2*>(a.state + (uint64_t)(qdst + a.qnext) * a.stride)[j] = y;
     }
 }
 
-// one thread = one gate x one 32-bit word (32 stimuli); consecutive threads = consecutive
+// one thread = one gate x one 64-bit word (64 stimuli); consecutive threads = consecutive
 // words of the same gate (coalesced loads, warp-uniform terms)
-__global__ void __launch_bounds__(256) k_level_poly(LevelArgs a, uint32_t words32, int check_only) {
+__global__ void __launch_bounds__(256) k_level_poly(LevelArgs a, uint32_t words64, int check_only) {
     pdl_entry();
     const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const uint32_t gi = (uint32_t)(t / words32), j = (uint32_t)(t - (uint64_t)gi * words32);
+    const uint32_t gi = (uint32_t)(t / words64), j = (uint32_t)(t - (uint64_t)gi * words64);
     uint32_t bad = 0u;
     if (gi < a.ng) {
         const uint32_t gate = a.g0 + gi;
@@ -809,11 +833,10 @@ __global__ void __launch_bounds__(256) k_level_poly(LevelArgs a, uint32_t words3
 
 cudaError_t launch_level_poly(const LevelArgs& a, int check_only, cudaStream_t s) {
     if (a.ng == 0) return cudaSuccess;
-    const uint32_t words32 = a.words * 2;
-    const uint64_t threads = (uint64_t)a.ng * words32;
+    const uint64_t threads = (uint64_t)a.ng * a.words;
     const uint64_t blocks = (threads + 255) / 256;
     if (blocks >= (1ull << 31)) return cudaErrorInvalidValue;
-    return launch_k(k_level_poly, (uint32_t)blocks, s, a.pdl, a, words32, check_only);
+    return launch_k(k_level_poly, (uint32_t)blocks, s, a.pdl, a, a.words, check_only);
 }
 
 // --------------------------------------------------------------------- stimulus
