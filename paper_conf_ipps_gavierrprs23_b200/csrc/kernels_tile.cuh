@@ -44,21 +44,24 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
 }
-__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+// dst_s / bar_s: shared-memory addresses (precomputed, see mbar_wait)
+__device__ __forceinline__ void tma_load_1d(uint32_t dst_s, const void* src, uint32_t bytes, uint32_t bar_s) {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // prior generic reads of dst
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar_s), "r"(bytes)
                  : "memory");
     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 ::"r"(dst_s), "l"(src), "r"(bytes), "r"(bar_s)
                  : "memory");
 }
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+// bar_s: the mbarrier's shared-memory address (computed once per kernel: the generic-to-
+// shared conversion costs an S2R of the CTA id, which sat on every level's critical path)
+__device__ __forceinline__ void mbar_wait(uint32_t bar_s, uint32_t parity) {
     uint32_t done = 0;
     while (!done) {
         asm volatile(
             "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n selp.u32 %0, 1, 0, p;\n}\n"
             : "=r"(done)
-            : "r"(smem_u32(bar)), "r"(parity), "r"(1000000u)   // suspend (<= 1 ms), not spin
+            : "r"(bar_s), "r"(parity), "r"(1000000u)   // suspend (<= 1 ms), not spin
             : "memory");
     }
 }
@@ -181,6 +184,8 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
+    const uint32_t mbar_s = smem_u32(mbar);                   // mode 2: the two mbarriers (8 B apart)
+    const uint32_t dbuf_s = smem_u32(dbuf);                   // mode 2: descriptor double buffer
     uint32_t* sw = reinterpret_cast<uint32_t*>(sl);          // slots as 32-bit words
     uint32_t* mp = SG ? reinterpret_cast<uint32_t*>(gsm) : sw + (size_t)a.n_slots * TW;   // MISR planes [64][TW]
     const unsigned long long c0 = a.ctl->cycle;
@@ -198,7 +203,7 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     // (the same sequence repeats every cycle and every tile)
     uint32_t step = 0;
     if (DM == 2 && tid == 0 && blockIdx.x * NG + gid < a.n_tiles)
-        tma_load_1d(dbuf, a.desc + lvl[0], (lvl[1] - lvl[0]) * 16, mbar);
+        tma_load_1d(dbuf_s, a.desc + lvl[0], (lvl[1] - lvl[0]) * 16, mbar_s);
 
     for (uint32_t tile = blockIdx.x * NG + gid; tile < a.n_tiles; tile += gridDim.x * NG) {
         const bool last_tile = tile + gridDim.x * NG >= a.n_tiles;
@@ -245,10 +250,10 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
                     const uint32_t b = step & 1;
                     if (tid == 0 && !(last_tile && c + 1 == a.ncycles && l + 1 == a.n_levels)) {
                         const uint32_t ln = l + 1 == a.n_levels ? 0 : l + 1;
-                        tma_load_1d(dbuf + (b ^ 1) * a.max_width, a.desc + lvl[ln], (lvl[ln + 1] - lvl[ln]) * 16,
-                                    mbar + (b ^ 1));
+                        tma_load_1d(dbuf_s + (b ^ 1) * a.max_width * 16, a.desc + lvl[ln],
+                                    (lvl[ln + 1] - lvl[ln]) * 16, mbar_s + 8 * (b ^ 1));
                     }
-                    mbar_wait(mbar + b, (step >> 1) & 1);
+                    mbar_wait(mbar_s + 8 * b, (step >> 1) & 1);
                     dl = dbuf + b * a.max_width;
                     ++step;
                 }
