@@ -57,15 +57,6 @@ __device__ __forceinline__ void tma_load_1d(uint32_t dst_s, const void* src, uin
 // shared conversion costs an S2R of the CTA id, which sat on every level's critical path)
 __device__ __forceinline__ void mbar_wait(uint32_t bar_s, uint32_t parity) {
     uint32_t done = 0;
-#ifdef GS_TILE_SPIN_WAIT
-    while (!done) {
-        asm volatile(
-            "{\n .reg .pred p;\n mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
-            : "=r"(done)
-            : "r"(bar_s), "r"(parity)
-            : "memory");
-    }
-#else
     while (!done) {
         asm volatile(
             "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n selp.u32 %0, 1, 0, p;\n}\n"
@@ -73,7 +64,6 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar_s, uint32_t parity) {
             : "r"(bar_s), "r"(parity), "r"(1000000u)   // suspend (<= 1 ms), not spin
             : "memory");
     }
-#endif
 }
 
 // One gate on P 16-byte groups (4 words = 128 lanes each, VS uint4 apart) of its slots:
