@@ -46,6 +46,7 @@ def parse():
     ap.add_argument("--config", default="C4")
     ap.add_argument("--cycles-per-step", type=int, default=100)
     ap.add_argument("--lut-k", type=int, default=0, help="cone-collapse into <= L-input LUTs first")
+    ap.add_argument("--order", type=int, default=0, help="gate order inside a level (0 by k/id, 1 recency)")
     ap.add_argument("--lanes", type=int, default=0, help="override lanes per GPU")
     ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab", "df", "tile"])
     ap.add_argument("--tile-words", type=int, default=0, help="kernel T: 32-bit words per slot")
@@ -259,7 +260,7 @@ def main():
     lanes_rank = lanes * subs
     lane_offset = rank * lanes_rank
     t0 = time.perf_counter()
-    prog = gs.Netlist.from_arrays(nl).compile(balance=True, lut_k=args.lut_k)
+    prog = gs.Netlist.from_arrays(nl).compile(balance=True, lut_k=args.lut_k, order=args.order)
     compile_s = time.perf_counter() - t0
     info = prog.info
     G = info["n_eval_gates"]
@@ -405,7 +406,7 @@ def main():
                        "df_interleave": args.df_interleave, "df_gpw": args.df_gpw,
                        "pdl": not args.no_pdl, "tile_words": args.tile_words,
                        "tile_groups": args.tile_groups, "tile_slots_global": args.tile_slots_global,
-                       "l2_hints": args.l2_hints, "lut_k": args.lut_k,
+                       "l2_hints": args.l2_hints, "lut_k": args.lut_k, "order": args.order,
                        "grid_stride": not args.no_grid_stride,
                        "l2": "inputs larger than L2 (state %.1f GB per GPU)" % (info["n_rows"] * lanes / 8 / 1e9),
                        "step": f"{C} cycles over every lane of the GPU" + (

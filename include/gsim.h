@@ -154,6 +154,10 @@ typedef struct {
                          RANDOM level in [1 + max level of its gate inputs, ALAP] (a valid
                          assignment of the same depth; results must not depend on it, a
                          property test of DESIGN.md reading R11).                      */
+    uint32_t order;       /* gate order inside a level (the level's execution order; results
+                         never depend on it).  0: by fan-in k, then gate id.  1: recency —
+                         gates whose newest input from the previous level was written last
+                         go first, so a level starts on the rows most likely still in L2.  */
 } gs_compile_opts;
 
 /* Validate (GS_ERR_UNDRIVEN, GS_ERR_COMB_LOOP, GS_ERR_ARITY), optionally collapse cones

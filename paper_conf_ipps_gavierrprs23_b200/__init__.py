@@ -57,7 +57,8 @@ class gs_netlist_counts(C.Structure):
 
 
 class gs_compile_opts(C.Structure):
-    _fields_ = [("balance", C.c_int), ("max_k", C.c_uint32), ("lut_k", C.c_uint32), ("level_seed", C.c_uint64)]
+    _fields_ = [("balance", C.c_int), ("max_k", C.c_uint32), ("lut_k", C.c_uint32), ("level_seed", C.c_uint64),
+                ("order", C.c_uint32)]
 
 
 class gs_program_info(C.Structure):
@@ -252,16 +253,17 @@ class Netlist:
         _call("gs_netlist_get_counts", self.h, C.byref(c))
         return {f: int(getattr(c, f)) for f, _ in c._fields_}
 
-    def compile(self, balance: bool = True, max_k: int = 0, lut_k: int = 0, level_seed: int = 0) -> "Program":
-        return Program(self, balance, max_k, lut_k, level_seed=level_seed)
+    def compile(self, balance: bool = True, max_k: int = 0, lut_k: int = 0, level_seed: int = 0,
+                order: int = 0) -> "Program":
+        return Program(self, balance, max_k, lut_k, level_seed=level_seed, order=order)
 
 
 class Program:
     def __init__(self, netlist: Netlist | None, balance: bool = True, max_k: int = 0, lut_k: int = 0,
-                 _handle=None, level_seed: int = 0):
+                 _handle=None, level_seed: int = 0, order: int = 0):
         if _handle is None:
             h = C.c_void_p()
-            o = gs_compile_opts(1 if balance else 0, max_k, lut_k, int(level_seed))
+            o = gs_compile_opts(1 if balance else 0, max_k, lut_k, int(level_seed), int(order))
             _call("gs_compile", netlist.h, C.byref(o), C.byref(h))
         else:
             h = _handle

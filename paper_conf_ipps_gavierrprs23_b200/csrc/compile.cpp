@@ -212,13 +212,43 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
     for (uint32_t l = 0; l <= D; ++l) pr.level_off[l] = (uint32_t)bucket[(uint64_t)l * (GS_MAX_K_POLY + 1)];
     std::vector<uint32_t> exec_pos(G, NONE32);
     pr.exec_gate.assign(n_eval, 0);
-    for (uint32_t g = 0; g < G; ++g)
-        if (nl.gate_k[g] > 0) {
-            uint64_t b = (uint64_t)(level[g] - 1) * (GS_MAX_K_POLY + 1) + nl.gate_k[g];
-            uint32_t pos = (uint32_t)bucket[b]++;
-            exec_pos[g] = pos;
-            pr.exec_gate[pos] = g;
+    if (opts.order == 0) {
+        for (uint32_t g = 0; g < G; ++g)
+            if (nl.gate_k[g] > 0) {
+                uint64_t b = (uint64_t)(level[g] - 1) * (GS_MAX_K_POLY + 1) + nl.gate_k[g];
+                uint32_t pos = (uint32_t)bucket[b]++;
+                exec_pos[g] = pos;
+                pr.exec_gate[pos] = g;
+            }
+    } else {
+        // recency order: level by level, a gate's key is the latest execution position among
+        // its inputs from the previous level; larger keys first (LIFO with respect to the
+        // previous level's stores), ties by gate id.  Level offsets are unchanged.
+        std::vector<std::vector<uint32_t>> by_level(D);
+        for (uint32_t g = 0; g < G; ++g)
+            if (nl.gate_k[g] > 0) by_level[level[g] - 1].push_back(g);
+        uint32_t pos = 0;
+        std::vector<std::pair<int64_t, uint32_t>> key;
+        for (uint32_t l = 0; l < D; ++l) {
+            key.clear();
+            for (uint32_t g : by_level[l]) {
+                int64_t m = -1;
+                for (uint32_t j = nl.gate_in_off[g]; j < nl.gate_in_off[g + 1]; ++j) {
+                    const uint32_t n = nl.gate_in[j];
+                    if (nl.net_kind[n] != NET_GATE) continue;
+                    const uint32_t h = nl.net_index[n];
+                    if (nl.gate_k[h] > 0 && level[h] + 1 == level[g]) m = std::max<int64_t>(m, exec_pos[h]);
+                }
+                key.push_back({-m, g});
+            }
+            std::sort(key.begin(), key.end());
+            for (auto& kg : key) {
+                exec_pos[kg.second] = pos;
+                pr.exec_gate[pos] = kg.second;
+                ++pos;
+            }
         }
+    }
 
     auto row_of = [&](uint32_t n) -> uint32_t {
         uint32_t i = nl.net_index[n];

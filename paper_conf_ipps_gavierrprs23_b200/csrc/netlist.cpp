@@ -239,11 +239,12 @@ gs_status gs_netlist_get_counts(const gs_netlist* h, gs_netlist_counts* out) {
 gs_status gs_compile(const gs_netlist* h, const gs_compile_opts* opts, gs_program** out) {
     NvtxRange nvtx("gs_compile");
     if (!h || !out) return fail(GS_ERR_ARG, "gs_compile: NULL argument");
-    gs_compile_opts o{1, 0, 0, 0};
+    gs_compile_opts o{1, 0, 0, 0, 0};
     if (opts) o = *opts;
     if (o.max_k == 0 || o.max_k > GS_MAX_K_POLY) o.max_k = GS_MAX_K_POLY;
     if (o.lut_k == 1 || o.lut_k > o.max_k)
         return fail(GS_ERR_ARG, "gs_compile: lut_k must be 0 or in [2, max_k]");
+    if (o.order > 1) return fail(GS_ERR_ARG, "gs_compile: order must be 0 or 1");
     Program* p = nullptr;
     gs_status st;
     try {

@@ -884,6 +884,17 @@ def test_c5_shard_full_netlist_sampled_lanes():
     probe_closed_forms(nl, gs.unpack_lanes(r["outputs"]).T, cfg.cycles - 1, cfg.stim_seed, lanes, off)
 
 
+@pytest.mark.parametrize("kernel", ["lut", "tile", "ab"])
+def test_recency_gate_order_same_results(kernel):
+    """gs_compile_opts.order = 1 (gates inside a level ordered by input recency) changes only
+    the execution order: every lane signature and register equals the default order's."""
+    nl = workloads.synthetic(20000, 800, 32, 48, 24, seed=12, name="s")
+    a = run_gpu(nl, 4096, 30, kernel, seed=4, prog=gs.Netlist.from_arrays(nl).compile())
+    b = run_gpu(nl, 4096, 30, kernel, seed=4, prog=gs.Netlist.from_arrays(nl).compile(order=1))
+    assert np.array_equal(a["sigs"], b["sigs"]) and np.array_equal(a["regs"], b["regs"])
+    assert np.array_equal(a["outputs"], b["outputs"])
+
+
 @pytest.mark.slow
 def test_c5_every_shard_sampled_lanes_sub_batches():
     """C5's full netlist over ALL 8 shards of its 262,144-lane batch with one sim re-targeted by

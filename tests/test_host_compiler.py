@@ -297,3 +297,16 @@ def test_program_save_load_round_trip(tmp_path):
         (tmp_path / "flip.gsp").write_bytes(bytes(flipped))
         with pytest.raises(gs.GsError):
             gs.Program.load(str(tmp_path / "flip.gsp"))
+
+
+def test_recency_order_is_a_permutation_within_levels():
+    """order = 1 keeps every gate's level and the level widths; only positions inside a level
+    move (gs_compile_opts.order)."""
+    nl = workloads.synthetic(20000, 800, 32, 48, 24, seed=12, name="s")
+    a = gs.Netlist.from_arrays(nl).compile()
+    b = gs.Netlist.from_arrays(nl).compile(order=1)
+    assert np.array_equal(a.level_widths(), b.level_widths())
+    assert np.array_equal(a.gate_levels(), b.gate_levels())
+    assert a.info["program_hash"] != b.info["program_hash"]
+    with pytest.raises(gs.GsError):
+        gs.Netlist.from_arrays(nl).compile(order=2)
