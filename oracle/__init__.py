@@ -31,7 +31,7 @@ def build(force: bool = False) -> str:
     """Compile oracle.c with gcc (-O2, OpenMP).  Building the checker is not using it."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fopenmp", "-fPIC", "-shared",
+        subprocess.check_call(["gcc", "-O3", "-std=c11", "-fopenmp", "-fPIC", "-shared",
                                "-Wall", "-Wextra", "-Wno-unused-parameter",
                                "-o", tmp, _SRC])
         os.replace(tmp, _LIB)

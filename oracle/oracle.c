@@ -141,8 +141,33 @@ static uint32_t tt_bit(const orc_netlist* nl, uint32_t g, uint32_t idx) {
     return (uint32_t)((nl->gate_tt_hi[(uint64_t)g * 3 + (idx >> 6) - 1] >> (idx & 63)) & 1u);
 }
 
+/* binary min-heap of gate ids (for the topological order below) */
+static void heap_push(uint32_t* h, uint32_t* n, uint32_t v) {
+    uint32_t i = (*n)++;
+    while (i > 0) {
+        uint32_t p = (i - 1) / 2;
+        if (h[p] <= v) break;
+        h[i] = h[p];
+        i = p;
+    }
+    h[i] = v;
+}
+static uint32_t heap_pop(uint32_t* h, uint32_t* n) {
+    uint32_t top = h[0], v = h[--(*n)], i = 0;
+    for (;;) {
+        uint32_t c = 2 * i + 1;
+        if (c >= *n) break;
+        if (c + 1 < *n && h[c + 1] < h[c]) c++;
+        if (v <= h[c]) break;
+        h[i] = h[c];
+        i = c;
+    }
+    if (*n) h[i] = v;
+    return top;
+}
+
 /* Kahn topological order of the gate DAG: a gate is ready when all of
- * its gate inputs are done; ties by gate id (FIFO seeded in id order).
+ * its gate inputs are done; among ready gates the smallest id goes first.
  * Returns 0, or -1 on a combinational loop (reading R8) or a bad net id. */
 int orc_topo_order(const orc_netlist* nl, uint32_t* order) {
     uint32_t G = nl->n_gates, base = nl->n_pi + nl->n_reg;
@@ -168,13 +193,20 @@ int orc_topo_order(const orc_netlist* nl, uint32_t* order) {
         free(fill);
     }
     {
-        uint32_t head = 0, tail = 0;
-        for (uint32_t g = 0; g < G; ++g) if (indeg[g] == 0) order[tail++] = g;
-        while (head < tail) {
-            uint32_t g = order[head++];
+        /* Kahn's algorithm taking the ready gate with the SMALLEST id first (a binary
+         * min-heap): the lexicographically first topological order, which is plain id
+         * order whenever every gate's inputs have smaller ids (SURVEY §8(c) "Kahn, by gate
+         * id").  Any topological order gives the same values (reading R11). */
+        uint32_t* heap = (uint32_t*)malloc((G ? G : 1) * sizeof(uint32_t));
+        uint32_t hn = 0, tail = 0;
+        for (uint32_t g = 0; g < G; ++g) if (indeg[g] == 0) heap_push(heap, &hn, g);
+        while (hn) {
+            uint32_t g = heap_pop(heap, &hn);
+            order[tail++] = g;
             for (uint32_t e = cnt[g]; e < cnt[g + 1]; ++e)
-                if (--indeg[adj[e]] == 0) order[tail++] = adj[e];
+                if (--indeg[adj[e]] == 0) heap_push(heap, &hn, adj[e]);
         }
+        free(heap);
         if (tail != G) rc = -1;
     }
 done:
@@ -204,6 +236,101 @@ int orc_asap_levels(const orc_netlist* nl, uint32_t* level) {
 
 /* ------------------------------------------------------------- simulation */
 
+#define ORC_BLOCK_MAX 64   /* most lanes a thread advances in lockstep (see orc_simulate) */
+
+/* Lanes [0, nlanes) in blocks of B lane slots; slots past the last lane repeat the block's
+ * first lane and are never reported (a fixed trip count keeps the lane loops simple).
+ * Inlined with a literal B by orc_simulate. */
+static inline __attribute__((always_inline)) int64_t sim_blocks(
+        const orc_netlist* nl, int mode, uint64_t seed, const uint64_t* host_stim, uint64_t stim_words,
+        uint32_t cycles, const uint64_t* lanes, uint32_t nlanes, const uint32_t* order,
+        const uint32_t* woff, const int64_t* wall, uint8_t* trace, uint8_t* last, uint8_t* regs,
+        uint64_t* sig, const uint32_t B) {
+    uint32_t G = nl->n_gates, P = nl->n_pi, R = nl->n_reg, O = nl->n_po;
+    uint32_t base = P + R, N = base + G;
+    int64_t violations = 0;
+    const int64_t nblocks = ((int64_t)nlanes + B - 1) / B;
+#ifdef _OPENMP
+#pragma omp parallel reduction(+ : violations)
+#endif
+    {
+        uint8_t* v = (uint8_t*)malloc((size_t)(N ? N : 1) * B);     /* v[net * B + b] */
+        uint8_t* q = (uint8_t*)malloc((size_t)(R ? R : 1) * B);     /* Q(c)   [r * B + b] */
+        uint8_t* qn = (uint8_t*)malloc((size_t)(R ? R : 1) * B);    /* Q(c+1) */
+        uint64_t misr[ORC_BLOCK_MAX];
+        uint64_t lane[ORC_BLOCK_MAX];
+#ifdef _OPENMP
+#pragma omp for schedule(dynamic, 1)
+#endif
+        for (int64_t bi = 0; bi < nblocks; ++bi) {
+            const uint64_t l0 = (uint64_t)bi * B;
+            const uint32_t nb = (uint32_t)((l0 + B <= nlanes) ? B : nlanes - l0);
+            for (uint32_t b = 0; b < B; ++b) {
+                lane[b] = lanes[l0 + (b < nb ? b : 0)];
+                misr[b] = 0;
+            }
+            for (uint32_t r = 0; r < R; ++r)
+                for (uint32_t b = 0; b < B; ++b) q[(size_t)r * B + b] = nl->reg_init[r] & 1u;
+            for (uint32_t c = 0; c < cycles; ++c) {
+                for (uint32_t p = 0; p < P; ++p)
+                    for (uint32_t b = 0; b < B; ++b) {
+                        const uint64_t s = lane[b];
+                        uint64_t word = host_stim ? host_stim[((uint64_t)c * P + p) * stim_words + (s >> 6)]
+                                                  : orc_stim_word(seed, p, c, s >> 6);
+                        v[(size_t)p * B + b] = (uint8_t)((word >> (s & 63)) & 1u);
+                    }
+                memcpy(v + (size_t)P * B, q, (size_t)R * B);
+                for (uint32_t i = 0; i < G; ++i) {
+                    const uint32_t g = order[i];
+                    const uint32_t k = nl->gate_k[g];
+                    const uint32_t* in = nl->gate_in + nl->gate_in_off[g];
+                    uint8_t idx[ORC_BLOCK_MAX];               /* truth-table index of every lane (R1), k <= 8 */
+                    for (uint32_t b = 0; b < B; ++b) idx[b] = 0;
+                    for (uint32_t j = 0; j < k; ++j) {
+                        const uint8_t* restrict x = v + (size_t)in[j] * B;
+                        for (uint32_t b = 0; b < B; ++b) idx[b] |= (uint8_t)(x[b] << j);
+                    }
+                    uint8_t* restrict y = v + (size_t)(base + g) * B;
+                    if (mode == 1) {
+                        for (uint32_t b = 0; b < B; ++b) {
+                            int64_t val = orc_poly_eval(wall + woff[g], (int)k, idx[b]);
+                            if (b < nb && val != 0 && val != 1) violations++;
+                            y[b] = (uint8_t)(val & 1);
+                        }
+                    } else if (k <= 6) {
+                        const uint64_t tt = nl->gate_tt[g];
+                        for (uint32_t b = 0; b < B; ++b) y[b] = (uint8_t)((tt >> idx[b]) & 1u);
+                    } else {
+                        for (uint32_t b = 0; b < B; ++b) y[b] = (uint8_t)tt_bit(nl, g, idx[b]);
+                    }
+                }
+                for (uint32_t b = 0; b < nb; ++b) {
+                    const uint64_t li = l0 + b;
+                    uint64_t word = 0;
+                    for (uint32_t o = 0; o < O; ++o) {
+                        uint8_t x = v[(size_t)nl->po[o] * B + b];
+                        if (trace) trace[((uint64_t)li * cycles + c) * O + o] = x;
+                        if (last && c + 1 == cycles) last[(uint64_t)li * O + o] = x;
+                        word ^= (uint64_t)x << (o & 63);
+                    }
+                    misr[b] = orc_misr_step(misr[b], word);
+                }
+                for (uint32_t r = 0; r < R; ++r)
+                    memcpy(qn + (size_t)r * B, v + (size_t)nl->reg_d[r] * B, B);
+                memcpy(q, qn, (size_t)R * B);
+            }
+            for (uint32_t b = 0; b < nb; ++b) {
+                const uint64_t li = l0 + b;
+                if (regs)
+                    for (uint32_t r = 0; r < R; ++r) regs[li * R + r] = q[(size_t)r * B + b];
+                if (sig) sig[li] = misr[b];
+            }
+        }
+        free(v); free(q); free(qn);
+    }
+    return violations;
+}
+
 /*
  * Simulate `nlanes` lanes (global stimulus indices lanes[i]) for `cycles`
  * clock cycles.  For lane s and cycle c:
@@ -215,6 +342,12 @@ int orc_asap_levels(const orc_netlist* nl, uint32_t* level) {
  *   out_o(c,s)= value of net po[o] after the evaluation, before the latch (R4)
  *   Q_r(c+1,s)= value of net reg_d[r] in cycle c, all registers at once (R3)
  *   sig_s     = orc_misr_step(sig_s, xor_o out_o(c,s) << (o mod 64))  (R5)
+ * Lanes never interact (stimulus independence), so a thread advances a block of up
+ * to ORC_BLOCK_MAX lanes in lockstep: per cycle it visits every gate once in the topological
+ * order and applies the same per-lane rule to each lane of the block (one byte per lane
+ * and net; no bit packing).  The netlist tables are then read once per block and cycle
+ * instead of once per lane and cycle; the value of every lane is computed exactly as in
+ * the one-lane formulation above.
  * Outputs (any may be NULL):
  *   trace  [nlanes][cycles][n_po] bytes  — every output of every cycle
  *   last   [nlanes][n_po] bytes          — outputs of the last cycle
@@ -251,58 +384,25 @@ int64_t orc_simulate(const orc_netlist* nl, int mode, uint64_t seed,
         }
     }
 
-    int64_t violations = 0;
 #ifdef _OPENMP
     if (threads > 0) omp_set_num_threads(threads);
-#pragma omp parallel reduction(+ : violations)
 #endif
-    {
-        uint8_t* v = (uint8_t*)malloc(N ? N : 1);
-        uint8_t* q = (uint8_t*)malloc(R ? R : 1);
-        uint8_t* qn = (uint8_t*)malloc(R ? R : 1);
+    /* lanes per block: 64 (one cache line per net and block) when there are enough lanes
+     * for every thread, else 32 or 16 */
+    uint32_t nth = 1;
 #ifdef _OPENMP
-#pragma omp for schedule(dynamic, 1)
+    nth = (uint32_t)omp_get_max_threads();
 #endif
-        for (int64_t li = 0; li < (int64_t)nlanes; ++li) {
-            uint64_t s = lanes[li];
-            uint64_t misr = 0;
-            for (uint32_t r = 0; r < R; ++r) q[r] = nl->reg_init[r] & 1u;
-            for (uint32_t c = 0; c < cycles; ++c) {
-                for (uint32_t p = 0; p < P; ++p) {
-                    uint64_t word = host_stim ? host_stim[((uint64_t)c * P + p) * stim_words + (s >> 6)]
-                                              : orc_stim_word(seed, p, c, s >> 6);
-                    v[p] = (uint8_t)((word >> (s & 63)) & 1u);
-                }
-                for (uint32_t r = 0; r < R; ++r) v[P + r] = q[r];
-                for (uint32_t i = 0; i < G; ++i) {
-                    uint32_t g = order[i];
-                    uint32_t k = nl->gate_k[g], idx = 0;
-                    for (uint32_t j = 0; j < k; ++j)
-                        idx |= (uint32_t)v[nl->gate_in[nl->gate_in_off[g] + j]] << j;
-                    if (mode == 1) {
-                        int64_t y = orc_poly_eval(wall + woff[g], (int)k, idx);
-                        if (y != 0 && y != 1) violations++;
-                        v[base + g] = (uint8_t)(y & 1);
-                    } else {
-                        v[base + g] = (uint8_t)tt_bit(nl, g, idx);
-                    }
-                }
-                uint64_t word = 0;
-                for (uint32_t o = 0; o < O; ++o) {
-                    uint8_t b = v[nl->po[o]];
-                    if (trace) trace[((uint64_t)li * cycles + c) * O + o] = b;
-                    if (last && c + 1 == cycles) last[(uint64_t)li * O + o] = b;
-                    word ^= (uint64_t)b << (o & 63);
-                }
-                misr = orc_misr_step(misr, word);
-                for (uint32_t r = 0; r < R; ++r) qn[r] = v[nl->reg_d[r]];
-                memcpy(q, qn, R);
-            }
-            if (regs) memcpy(regs + (uint64_t)li * R, q, R);
-            if (sig) sig[li] = misr;
-        }
-        free(v); free(q); free(qn);
-    }
+    int64_t violations;
+    if ((uint64_t)nlanes >= 64ull * nth)
+        violations = sim_blocks(nl, mode, seed, host_stim, stim_words, cycles, lanes, nlanes, order, woff, wall,
+                                trace, last, regs, sig, 64);
+    else if ((uint64_t)nlanes >= 32ull * nth)
+        violations = sim_blocks(nl, mode, seed, host_stim, stim_words, cycles, lanes, nlanes, order, woff, wall,
+                                trace, last, regs, sig, 32);
+    else
+        violations = sim_blocks(nl, mode, seed, host_stim, stim_words, cycles, lanes, nlanes, order, woff, wall,
+                                trace, last, regs, sig, 16);
     free(order); free(woff); free(wall);
     return violations;
 }

@@ -148,10 +148,16 @@ def test_wide_gates_algorithm1_definition_and_eq1(k):
 
 
 def test_algorithm1_operation_count():
-    # "our algorithm requires at most 2^L L operations"
-    for L in range(0, 12):
-        assert mobius.alg1_op_count(L) == L * 2 ** (L - 1) if L else True
-        assert mobius.alg1_op_count(L) <= (2 ** L) * L
+    """"our algorithm requires at most 2^L L operations".  The subtractions Algorithm 1
+    performs are COUNTED while it runs (oracle/mobius.py instruments its merge); the count is
+    L 2^(L-1) — each of the L recursion depths merges 2^(L-1) coefficient pairs in total — and
+    independent of the table."""
+    rng = np.random.default_rng(3)
+    for L in range(0, 11):
+        for tt in (0, (1 << (1 << L)) - 1, int(rng.integers(0, 2**63)) & ((1 << (1 << L)) - 1)):
+            n = mobius.alg1_op_count(L, tt)
+            assert n == (L * 2 ** (L - 1) if L else 0), (L, n)
+            assert n <= (2 ** L) * L
 
 
 def test_threshold_function_claims():
@@ -381,5 +387,31 @@ def test_asap_depth_of_structural_circuits():
     # ripple adder built from (XOR, XOR, AND, AND, OR) cells is at depth 2i+1 ... 2i+2
     lv = oracle.asap_levels(workloads.adder(8))
     assert lv.max() == 15
-    lv2 = oracle.asap_levels(workloads.array_multiplier(32))
-    assert lv2 is not None and lv2.max() > 60
+    # n x n array multiplier of ripple-carry rows: depth 6n - 8 (n >= 3), so 184 at n = 32
+    # (SURVEY §8(a) row a2); checked against an independent memoised-DFS longest path
+    def dfs_depth(nl):
+        base = nl.n_pi + nl.n_reg
+        memo = {}
+        for g0 in range(nl.n_gates):                     # iterative DFS, any order
+            stack = [g0]
+            while stack:
+                g = stack[-1]
+                if g in memo:
+                    stack.pop()
+                    continue
+                ins = [int(n) - base for n in nl.gate_in[nl.gate_in_off[g]:nl.gate_in_off[g + 1]] if n >= base]
+                todo = [h for h in ins if h not in memo]
+                if todo:
+                    stack.extend(todo)
+                    continue
+                memo[g] = 0 if nl.gate_k[g] == 0 else 1 + max((memo[h] for h in ins), default=0)
+                stack.pop()
+        return memo
+    for n in (3, 4, 5, 8, 13, 16, 32):
+        nl = workloads.array_multiplier(n)
+        lv = oracle.asap_levels(nl)
+        assert lv.max() == 6 * n - 8, (n, lv.max())
+        if n <= 16:
+            d = dfs_depth(nl)
+            assert all(int(lv[g]) == d[g] for g in range(nl.n_gates))
+    assert oracle.asap_levels(workloads.array_multiplier(32)).max() == 184
