@@ -1,29 +1,32 @@
 #!/usr/bin/env python
 """bench.py — stimulus·gate·cycle evaluations per second of the gsim hot path on B200.
 
-Contract:
+Contract (see DESIGN.md §7 "Measurement"):
   python bench.py --gpus N --steps K --warmup W           (N > 1: under torch.distributed.run)
   python bench.py --impl reference ...                     (the CPU oracle arm, rank 0 only)
 
-A *step* is ``--cycles-per-step`` clock cycles (default 100) of the whole hot path —
-stimulus generation, every level of gates with the fused register latch, the remaining
-latches and the output MISR — over one batch of stimuli.  The default workload is
-BASELINE.json configs[3] (C4: RISC-V-core-scale synthetic, 1M gates + 50k registers,
-65,536 stimuli per GPU), the largest configuration that fits one GPU; its 1,000-cycle
-run is 10 steps.  Multi-GPU is weak scaling: every rank simulates its own 65,536 global
-lanes (lane_offset = rank * lanes) of the same netlist; the only collective is the
-all-reduce of the per-rank signatures.  C5 (BASELINE configs[4], 8 shards of 32,768 lanes)
-runs its whole 262,144-lane batch at any N dividing 8: each rank simulates 8/N shards as
-sequential sub-batches in one workspace (gs_sim_set_lane_offset); a step is then C cycles of
-every sub-batch, each from reset.
+Default workload: BASELINE.json configs[4] (C5, the north_star's "largest config"): the
+NVDLA-scale synthetic netlist (10M gates + 500k registers) over its whole batch of 262,144
+stimuli for 100 cycles.  A *step* is that whole job: every lane of the batch simulated from
+reset for 100 clock cycles through the whole hot path (stimulus generation, every level with
+the fused register latch, the leftover latches and the output MISR).  The batch is STRONG-
+scaled over the N ranks: rank r owns a contiguous 262,144/N-lane range (dist.shard) and runs
+it as sequential sub-batches of at most --sub-lanes lanes in one workspace (the whole state
+of C5 does not fit one GPU); every sub-batch starts from reset, so the all-reduced
+lane_sig_sum is identical at every N (a self-check of the sharding).
+`--config C4` (BASELINE configs[3], 1M gates, 65,536 lanes per GPU, weak-scaled) keeps the
+round-1 shape: a step is --cycles-per-step cycles continuing from the previous step.
 
 value = G_eval * lanes_total * cycles / max-over-ranks device time of the K timed steps.
 """
 from __future__ import annotations
 
 import argparse
+import glob
 import json
 import os
+import platform
+import re
 import statistics
 import subprocess
 import sys
@@ -40,38 +43,34 @@ UNIT = "sgc/s"
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="C4")
-    ap.add_argument("--cycles-per-step", type=int, default=100)
+    ap.add_argument("--config", default="C5")
+    ap.add_argument("--cycles-per-step", type=int, default=0,
+                    help="cycles per step (0 = the config's cycle count for sharded configs, else 100)")
+    ap.add_argument("--sub-lanes", type=int, default=32768,
+                    help="sharded configs: lanes per sub-batch (a multiple of the shard size / 2^k)")
     ap.add_argument("--lut-k", type=int, default=0, help="cone-collapse into <= L-input LUTs first")
-    ap.add_argument("--order", type=int, default=0, help="gate order inside a level (0 by k/id, 1 recency)")
-    ap.add_argument("--lanes", type=int, default=0, help="override lanes per GPU")
-    ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab", "df", "tile"])
+    ap.add_argument("--lanes", type=int, default=0, help="override lanes per GPU (unsharded configs)")
+    ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab", "tile", "auto"])
+    ap.add_argument("--no-balance", action="store_true", help="ASAP levels (balance-off A/B)")
     ap.add_argument("--tile-words", type=int, default=0, help="kernel T: 32-bit words per slot")
     ap.add_argument("--tile-groups", type=int, default=0, help="kernel T: thread groups per CTA")
-    ap.add_argument("--tile-slots-global", action="store_true",
-                    help="kernel T: live slots in the workspace (L1/L2) instead of shared memory")
-    ap.add_argument("--df-interleave", type=int, default=0, help="kernel D: slabs walked together")
-    ap.add_argument("--df-gpw", type=int, default=0, help="kernel D: gates per warp per item")
-    ap.add_argument("--lane-slabs", type=int, default=0, help="L2 lane slabs (0 = library default)")
     ap.add_argument("--lut-unroll", type=int, default=0, help="vectors per thread (0 = auto)")
     ap.add_argument("--lane-groups", type=int, default=0,
                     help="kernel A: concurrent lane groups per cycle (0 = library auto, 1 = off)")
     ap.add_argument("--no-pdl", action="store_true", help="disable programmatic dependent launch")
     ap.add_argument("--no-grid-stride", action="store_true", help="kernel A: one CTA per work chunk")
-    ap.add_argument("--l2-hints", type=int, default=0, help="kernel A L2 hints: 0 off, 1 stores, 2 +loads")
-    ap.add_argument("--lut-bulk", default="auto", choices=["auto", "on", "off"],
-                    help="kernel A bulk-copy staged gathers (auto = library default: off)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend (gloo + --same-device: multi-rank test on one GPU)")
     ap.add_argument("--same-device", action="store_true",
                     help="test only: every rank uses cuda:0 (timings are NOT a scaling measurement)")
-    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true", help="skip the oracle parity leg")
+    ap.add_argument("--parity-lanes", type=int, default=256, help="oracle-checked lanes (parity leg)")
     ap.add_argument("--no-roofline", action="store_true")
-    ap.add_argument("--cpu-seconds", type=float, default=25.0, help="target oracle wall time (calibrated)")
+    ap.add_argument("--core-seconds", type=float, default=12.0, help="target wall time of the 1-thread oracle leg")
     ap.add_argument("--quick", action="store_true", help="ncu mode: no e2e/cpu/roofline/clocks")
     return ap.parse_args()
 
@@ -113,6 +112,7 @@ class ClockSampler:
             self.proc.kill()
         sm = [float(r[1]) for r in self.rows if len(r) > 2 and r[1].replace(".", "").isdigit()]
         mx = [float(r[2]) for r in self.rows if len(r) > 2 and r[2].replace(".", "").isdigit()]
+        pw = [float(r[3]) for r in self.rows if len(r) > 3 and r[3].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = set()
         for r in self.rows:
@@ -121,69 +121,85 @@ class ClockSampler:
                     reasons.add(n)
         return {"sm_mhz": statistics.median(sm) if sm else None,
                 "sm_max_mhz": max(mx) if mx else None, "reasons": sorted(reasons),
-                "samples": len(self.rows)}
+                "power_w_median": statistics.median(pw) if pw else None, "samples": len(self.rows)}
 
 
 def peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
-            return json.load(f), "measured"
+            return json.load(f), "measured (MEASURED_PEAKS.json)"
     except Exception:
-        return {"hbm_gbs": 6650.0}, "fallback"
+        return {"hbm_gbs": 6650.0}, "fallback (B200_PROFILING.md)"
 
 
-KERNEL_NAMES = {"lut": "k_level_lut_wide<4, 0>", "df": "k_dataflow<1>", "poly": "k_level_poly",
-                "ab": "k_level_lut_wide<4, 0>", "tile": "k_tile"}
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    return ln.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return platform.processor() or "unknown"
 
 
-def ncu_traffic(config: str, kernel: str):
-    """dram read+write bytes per launch of `kernel` on `config` from the committed ncu --set
-    full summary (profiles/traffic.json, from scripts/ncu_summary.py on the same bench command)."""
+def insitu_traffic(key: str, build_id: str, program_hash: int):
+    """In-situ DRAM bytes of one simulated cycle (ncu --graph-profiling graph of the cycle's
+    CUDA graph, concurrency intact) from profiles/traffic.json — only if that entry was
+    captured on THIS build of libgsim.so and THIS program; a stale entry is refused."""
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-            d = json.load(f)
-        e = d["kernels"][f"{config}:{kernel}"]
-        return {"traffic_bytes_per_launch": e["traffic_bytes_per_launch"],
-                "source": e.get("source", d.get("source"))}
+            e = json.load(f)["insitu"][key]
     except Exception:
-        return None
+        return None, f"no in-situ capture for {key}"
+    if e.get("build_id") != build_id:
+        return None, f"stale: captured on build {e.get('build_id')}, this is {build_id}"
+    if int(e.get("program_hash", -1)) != int(program_hash):
+        return None, "stale: captured on another program"
+    return e, e.get("source")
 
 
-def insitu_dram(config: str, groups: int, ms_per_cycle: float, peak: float):
-    """Actual DRAM rate of the whole cycle: the committed in-situ DRAM bytes of one cycle graph
-    (ncu --graph-profiling graph, profiles/traffic.json 'cycles') / this run's time per cycle."""
-    try:
-        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-            e = json.load(f)["cycles"][f"{config}:G{groups}"]
-    except Exception:
-        return None
-    gbs = e["dram_bytes_per_cycle"] / (ms_per_cycle / 1e3) / 1e9
-    return {"bytes_per_cycle": e["dram_bytes_per_cycle"], "gbs": gbs, "frac": gbs / peak, "source": e["source"]}
-
-
-# ------------------------------------------------------------------ CPU oracle
-def oracle_rate(nl, cfg, lane_offset, seconds: float, cycles_cap: int | None = None):
-    """Time the oracle (as it stands) on a bounded sample: n_threads lanes x c cycles."""
+# ------------------------------------------------------------------ CPU oracle legs
+def oracle_parity_and_rate(nl, cfg, lanes_global, cycles, gpu_sigs, gpu_regs):
+    """The parity leg (rank 0, N = 1): the oracle, as it stands, simulates the sampled lanes
+    for exactly the GPU run's cycles (from reset, same seed); its per-lane MISR signatures and
+    final registers are compared bit for bit with the GPU's.  Its wall time is the
+    cpu_baseline rate (G x lanes x cycles / s) on all host threads."""
     import numpy as np
     import oracle
     threads = oracle.max_threads()
     G = int((nl.gate_k > 0).sum())
-    lanes_total = cfg.lanes
-    # calibration: one lane per thread, 8 cycles
-    sample = np.linspace(0, lanes_total - 1, threads).astype(np.int64) + lane_offset
     t = time.perf_counter()
-    oracle.simulate(nl, sample, 8, seed=cfg.stim_seed, threads=threads, want=("sig",))
-    dt = max(time.perf_counter() - t, 1e-3)
-    per_cycle = dt / 8
-    cycles = max(2, int(seconds / per_cycle))
-    if cycles_cap:
-        cycles = min(cycles, cycles_cap)
-    t = time.perf_counter()
-    oracle.simulate(nl, sample, cycles, seed=cfg.stim_seed, threads=threads, want=("sig",))
+    o = oracle.simulate(nl, lanes_global, cycles, seed=cfg.stim_seed, threads=threads, want=("regs", "sig"))
     dt = time.perf_counter() - t
-    return {"value": G * len(sample) * cycles / dt, "unit": UNIT, "cores": threads, "kind": "oracle",
-            "sample": f"{len(sample)} lanes (one per thread, spread over the batch) x {cycles} cycles "
-                      f"of {cfg.name}, generated stimuli seed {cfg.stim_seed}; {dt:.1f} s wall"}, dt
+    sig_mm = int((o["sig"] != gpu_sigs).sum())
+    reg_mm = int((o["regs"] != gpu_regs).sum()) if nl.n_reg else 0
+    parity = {"lanes_checked": int(len(lanes_global)), "cycles": int(cycles),
+              "registers_per_lane": int(nl.n_reg),
+              "lane_signature_mismatches": sig_mm, "register_bit_mismatches": reg_mm,
+              "mismatches": sig_mm + reg_mm,
+              "what": "per-lane 64-bit MISR over every output of every cycle (R5) and every register "
+                      "bit after the last cycle, oracle vs GPU, same netlist / seed / cycles from reset"}
+    cpu = {"value": G * len(lanes_global) * cycles / dt, "unit": UNIT, "cores": threads, "kind": "oracle",
+           "cpu_model": cpu_model(),
+           "sample": f"{len(lanes_global)} lanes spread over every shard x {cycles} cycles of {cfg.name} "
+                     f"(the parity leg), generated stimuli seed {cfg.stim_seed}; {dt:.1f} s wall on {threads} threads"}
+    return parity, cpu
+
+
+def oracle_per_core(nl, cfg, seconds: float):
+    """--threads 1 figure: one lane on one thread for as many cycles as fit `seconds`."""
+    import numpy as np
+    import oracle
+    G = int((nl.gate_k > 0).sum())
+    t = time.perf_counter()
+    oracle.simulate(nl, np.array([5]), 2, seed=cfg.stim_seed, threads=1, want=("sig",))
+    per_cycle = max((time.perf_counter() - t) / 2, 1e-5)
+    c = max(2, int(seconds / per_cycle))
+    t = time.perf_counter()
+    oracle.simulate(nl, np.array([5]), c, seed=cfg.stim_seed, threads=1, want=("sig",))
+    dt = time.perf_counter() - t
+    return {"value": G * c / dt, "unit": UNIT, "cores": 1, "sample": f"1 lane x {c} cycles, {dt:.1f} s"}
 
 
 def run_reference(args):
@@ -199,12 +215,14 @@ def run_reference(args):
     G = int((nl.gate_k > 0).sum())
     threads = oracle.max_threads()
     sample = np.linspace(0, cfg.lanes - 1, threads).astype(np.int64)
-    # per step: every thread simulates one lane for c cycles; size c so the run is minutes
+    cps = args.cycles_per_step or (cfg.cycles if cfg.shards > 1 else 100)
+    # per step: every thread simulates one lane for c cycles from reset; size c so the whole
+    # run is a few minutes
     t = time.perf_counter()
     oracle.simulate(nl, sample, 2, seed=cfg.stim_seed, threads=threads, want=("sig",))
     per_cycle = max((time.perf_counter() - t) / 2, 1e-4)
     budget = 150.0 / max(args.steps + args.warmup, 1)
-    c = max(1, min(args.cycles_per_step, int(budget / per_cycle)))
+    c = max(1, min(cps, int(budget / per_cycle)))
     for _ in range(args.warmup):
         oracle.simulate(nl, sample, c, seed=cfg.stim_seed, threads=threads, want=("sig",))
     t = time.perf_counter()
@@ -214,14 +232,29 @@ def run_reference(args):
     val = G * len(sample) * c * args.steps / dt
     line = {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": dt * 1e3 / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-            "impl": "reference",
+            "scaling": "strong" if cfg.shards > 1 else "weak", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic", "impl": "reference",
             "config": {"workload": f"{cfg.name}: {cfg.label}", "gates": G, "lanes_per_step": len(sample),
                        "cycles_per_step": c},
             "cpu_baseline": {"value": val, "unit": UNIT, "cores": threads, "kind": "oracle",
-                             "sample": f"{len(sample)} lanes x {c} cycles per step of {cfg.name}"},
+                             "cpu_model": cpu_model(),
+                             "sample": f"{len(sample)} lanes x {c} cycles from reset per step of {cfg.name}"},
             "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+def nccl_nranks(pattern: str):
+    """nRanks that NCCL's INIT log reported for this process's communicator (None if absent)."""
+    n = None
+    for f in glob.glob(pattern):
+        try:
+            for ln in open(f, errors="replace"):
+                m = re.search(r"nRanks\s+(\d+)", ln)
+                if m:
+                    n = int(m.group(1))
+        except Exception:
+            pass
+    return n
 
 
 # ------------------------------------------------------------------ GPU arm
@@ -230,6 +263,16 @@ def main():
     if args.impl == "reference":
         return run_reference(args)
 
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    nccl_log = f"/tmp/gsim_nccl_{os.getpid()}.log"
+    if world > 1 and args.dist_backend == "nccl":
+        # NCCL INIT log to a file (never stdout: the driver reads one JSON line there)
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        os.environ.setdefault("NCCL_DEBUG_FILE", nccl_log)
+
     import numpy as np
     import torch
     import torch.distributed as dist
@@ -237,9 +280,6 @@ def main():
     import paper_conf_ipps_gavierrprs23_b200 as gs
     from paper_conf_ipps_gavierrprs23_b200 import dist as gdist
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         print(f"warning: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
     if args.same_device:
@@ -253,29 +293,34 @@ def main():
 
     cfg = workloads.CONFIGS[args.config]
     nl = cfg.netlist()
-    # lanes = one sim's lanes; a sharded config (C5: 8 shards of 32,768 lanes) gives every rank
-    # shards/world of them, run as sequential sub-batches in one workspace
-    lanes = args.lanes or (cfg.lanes // cfg.shards if cfg.shards > 1 else cfg.lanes)
-    subs = cfg.shards // world if (not args.lanes and cfg.shards > world and cfg.shards % world == 0) else 1
-    lanes_rank = lanes * subs
-    lane_offset = rank * lanes_rank
+    sharded = cfg.shards > 1 and not args.lanes
+    C = args.cycles_per_step or (cfg.cycles if sharded else 100)
+    if sharded:
+        # strong scaling: the whole batch is split over the ranks, each rank runs its range as
+        # sub-batches (from reset every step) of at most --sub-lanes lanes
+        lane_offset, lanes_rank = gdist.shard(cfg.lanes, world, rank)
+        lanes = min(args.sub_lanes, lanes_rank)
+        if lanes_rank % lanes:
+            raise SystemExit(f"rank range {lanes_rank} is not a multiple of --sub-lanes {lanes}")
+        subs = lanes_rank // lanes
+    else:
+        lanes = args.lanes or cfg.lanes
+        lanes_rank, subs = lanes, 1
+        lane_offset = rank * lanes                      # weak scaling: own global range per rank
+    lanes_total = lanes_rank * world
     t0 = time.perf_counter()
-    prog = gs.Netlist.from_arrays(nl).compile(balance=True, lut_k=args.lut_k, order=args.order)
+    prog = gs.Netlist.from_arrays(nl).compile(balance=not args.no_balance, lut_k=args.lut_k)
     compile_s = time.perf_counter() - t0
     info = prog.info
     G = info["n_eval_gates"]
     if world > 1:
         gdist.check_same_program(info["program_hash"])
     stream = torch.cuda.Stream(device=local)
+    flags = (8 if args.no_grid_stride else 0)
     sim = gs.Sim(prog, lanes, lane_offset=lane_offset, kernel=args.kernel, device=local, stream=stream,
-                 lane_slabs=args.lane_slabs, lut_unroll=args.lut_unroll,
-                 df_interleave=args.df_interleave, df_gates_per_warp=args.df_gpw, pdl=not args.no_pdl,
-                 tile_words=args.tile_words, tile_groups=args.tile_groups, lane_groups=args.lane_groups,
-                 flags=(2 if args.l2_hints >= 1 else 0) | (4 if args.l2_hints >= 2 else 0) |
-                 (8 if args.no_grid_stride else 0) | (256 if args.tile_slots_global else 0) |
-                 {"auto": 0, "on": 64, "off": 128}[args.lut_bulk])
+                 lut_unroll=args.lut_unroll, pdl=not args.no_pdl, tile_words=args.tile_words,
+                 tile_groups=args.tile_groups, lane_groups=args.lane_groups, flags=flags)
     sim.bind_generated(cfg.stim_seed)
-    C = args.cycles_per_step
     launches_per_cycle = sim.launches_per_cycle()
 
     def barrier():
@@ -285,16 +330,19 @@ def main():
     sig_keys = ("lane_sig_sum", "out_popcount", "ab_mismatch", "invariant_violations")
     sub_sigs = []
 
-    def one_step():
-        """C cycles over this rank's whole batch: one sim, or every sub-batch from reset."""
-        if subs == 1:
+    def one_step(record=None):
+        """One step: sharded -> every sub-batch of this rank from reset for C cycles;
+        otherwise C more cycles of the one sim.  record(j) is called after sub-batch j."""
+        if not sharded:
             sim.step(C)
             return
         sub_sigs.clear()
         for j in range(subs):
-            sim.set_lane_offset(lane_offset + j * lanes)      # syncs, re-targets, resets
+            sim.set_lane_offset(lane_offset + j * lanes)      # re-targets and resets
             sim.step(C)
             sub_sigs.append(sim.signature())
+            if record:
+                record(j)
 
     for _ in range(args.warmup):
         one_step()
@@ -315,43 +363,54 @@ def main():
     barrier()
     ms_max = gdist.max_over_ranks(ms) if world > 1 else ms
     sig = sim.signature()
-    if subs > 1:                       # the last timed step's sub-batches, summed mod 2^64
+    if sharded:                        # the last timed step's sub-batches, summed mod 2^64
         sig = {k: (sum(d[k] for d in sub_sigs) % (1 << 64) if k in sig_keys else sig[k]) for k in sig}
     red = gdist.reduce_signature(sig) if world > 1 else sig
-
-    total_sgc = float(G) * lanes_rank * world * C * args.steps
+    cycles_per_rank_step = C * subs
+    total_sgc = float(G) * lanes_total * C * args.steps
     value = total_sgc / (ms_max / 1e3)
 
-    # ---------------------------------------------------------------- roofline
+    # ---------------------------------------------------------------- roofline (last sub-batch)
     roof = None
     pk, pk_src = peaks()
     if not args.no_roofline and not args.quick:
-        pr = sim.profile_step(min(C, 10))
+        ncyc = min(C, 10)
+        pr = sim.profile_step(ncyc)
         achieved = pr["level_bytes"] / (pr["level_ms"] / 1e3) / 1e9
         per_launch_bytes = pr["level_bytes"] / max(pr["level_launches"], 1)
-        kname = KERNEL_NAMES[args.kernel]
-        if args.kernel == "df":
-            kname = f"k_dataflow<{lanes // (args.lane_slabs or lanes // 4096) // 4096}>"
-        G_groups = sim.config["lane_groups"]
-        tr = ncu_traffic(args.config, f"{kname}:G{G_groups}")
-        roof = {"bound": "hbm", "kernel": kname,
-                "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
-                "frac": achieved / pk["hbm_gbs"],
-                "traffic": tr["traffic_bytes_per_launch"] if tr else None,
-                "traffic_source": tr["source"] if tr else None,
-                "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({pk_src})",
+        groups = sim.config["lane_groups"]
+        key = f"{cfg.name}:{lanes}:{args.kernel}:G{groups}"
+        tr, tr_src = insitu_traffic(key, gs.build_id(), info["program_hash"])
+        ms_cycle = ms_max / (args.steps * cycles_per_rank_step)
+        dram = None
+        if tr:
+            gbs = tr["dram_bytes_per_cycle"] / (ms_cycle / 1e3) / 1e9
+            dram = {"bytes_per_cycle": tr["dram_bytes_per_cycle"], "read_bytes_per_cycle": tr.get("read_bytes"),
+                    "write_bytes_per_cycle": tr.get("write_bytes"), "gbs": gbs, "frac": gbs / pk["hbm_gbs"],
+                    "l2_hit_pct": tr.get("l2_hit_pct"), "source": tr_src,
+                    "note": "actual DRAM bytes of one cycle (in-situ ncu graph capture of this build and "
+                            "program) / this run's device time per cycle"}
+        lvl_per_cycle = pr["level_launches"] / max(ncyc, 1)
+        roof = {"bound": "hbm", "kernel": "k_level_lut_wide<4>" if args.kernel in ("lut", "auto") else args.kernel,
+                "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s", "frac": achieved / pk["hbm_gbs"],
+                "frac_basis": "algorithmic gather-model bytes (k reads + 1 write + fused latch per gate-row) "
+                              "/ measured HBM copy peak; L2 hits let it exceed the DRAM fraction, which is "
+                              "dram_insitu.frac",
+                "traffic": (tr["dram_bytes_per_cycle"] / lvl_per_cycle) if tr and lvl_per_cycle else None,
+                "traffic_source": (f"in-situ DRAM bytes per cycle / {lvl_per_cycle:.0f} level launches per "
+                                   f"cycle ({tr_src})") if tr else tr_src,
+                "peak_source": f"hbm_gbs {pk_src}",
                 "algorithmic_bytes_per_launch": per_launch_bytes,
                 "level_share_of_step": pr["level_ms"] / pr["total_ms"],
-                "lane_groups": G_groups,
-                "dram_insitu": insitu_dram(args.config, G_groups, ms_max / (args.steps * C * subs), pk["hbm_gbs"]),
+                "lane_groups": groups, "lanes_per_launch": lanes // max(groups, 1),
+                "dram_insitu": dram,
                 "avg_level_launch_us": pr["level_ms"] * 1e3 / max(pr["level_launches"], 1),
-                "measured": (f"CUDA events around every level launch on the sim stream, "
-                             f"{min(C, 10)} un-graphed cycles after the timed region") if G_groups == 1 else
-                            (f"{G_groups} lane groups run their level chains concurrently: timing-event "
-                             f"graph nodes at the fork and join of the level region of each of {min(C, 10)} "
-                             f"graph-replayed cycles after the timed region; achieved = algorithmic bytes "
-                             f"of all level launches / region time, avg_level_launch_us = region time / "
-                             f"launches (launches overlap)")}
+                "measured": (f"CUDA events around every level launch on the sim stream, {ncyc} un-graphed "
+                             f"cycles of the last sub-batch after the timed region") if groups == 1 else
+                            (f"{groups} lane groups run their level chains concurrently: timing-event graph "
+                             f"nodes at the fork and join of the level region of each of {ncyc} graph-replayed "
+                             f"cycles after the timed region; achieved = algorithmic bytes of all level "
+                             f"launches / region time, avg_level_launch_us = region time / launches")}
 
     # ---------------------------------------------------------------- e2e
     # paper-style: every step streams its stimuli host->device and EVERY output of
@@ -361,7 +420,7 @@ def main():
     if not args.no_e2e and not args.quick:
         n_pi, n_po = info["n_pi"], info["n_po"]
         words = lanes // 64
-        K2 = max(1, min(args.steps, 3))
+        K2 = max(1, min(args.steps, 2))
         host = torch.empty((C, n_pi, words), dtype=torch.int64).pin_memory()
         host.random_()
         h_np = host.numpy().view(np.uint64)
@@ -375,50 +434,81 @@ def main():
         e0.record(stream)
         for _ in range(K2):
             for j in range(subs):
-                if subs > 1:
+                if sharded:
                     sim.set_lane_offset(lane_offset + j * lanes)
                 sim.run_streamed(h_np, o_np)
         e1.record(stream)
         torch.cuda.synchronize()
         ems = e0.elapsed_time(e1)
         ems = gdist.max_over_ranks(ems) if world > 1 else ems
-        e2e = {"value": float(G) * lanes_rank * world * C * K2 / (ems / 1e3), "unit": UNIT,
+        e2e = {"value": float(G) * lanes_total * C * K2 / (ems / 1e3), "unit": UNIT,
                "h2d_bytes_per_step": int(host.numel() * 8) * subs, "d2h_bytes_per_step": int(out_buf.numel() * 8) * subs,
                "steps": K2, "path": "gs_sim_run_streamed: pinned host stimuli in, every output of every "
-                                    "cycle out, 25-cycle chunks overlapped with compute"}
+                                    "cycle out, 25-cycle chunks overlapped with compute"
+                                    + ("; every sub-batch from reset" if sharded else "")}
+        sim.bind_generated(cfg.stim_seed)
 
-    # ---------------------------------------------------------------- cpu baseline
-    cpu = None
+    # ---------------------------------------------------------------- parity leg + cpu baseline
+    cpu, parity = None, None
     if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.quick:
-        cpu, _ = oracle_rate(nl, cfg, lane_offset, args.cpu_seconds, cycles_cap=None)
+        # a verification pass identical to a timed step's work (every sub-batch from reset
+        # for the config's cycles), reading back per-lane signatures and registers, then the
+        # oracle on the sampled lanes
+        vc = cfg.cycles
+        sample = workloads.sample_lanes(lanes_total, max(cfg.shards, 1) if sharded else 1,
+                                        args.parity_lanes // (cfg.shards if sharded else 1), seed=2,
+                                        groups=max(sim.config["lane_groups"], 1))
+        sample = sample[(sample >= lane_offset) & (sample < lane_offset + lanes_rank)]
+        gsig = np.zeros(len(sample), dtype=np.uint64)
+        greg = np.zeros((len(sample), info["n_reg"]), dtype=np.uint8)
+
+        def record(j):
+            lo = lane_offset + j * lanes
+            m = (sample >= lo) & (sample < lo + lanes)
+            if not m.any():
+                return
+            loc = sample[m] - lo
+            gsig[m] = sim.read_lane_signatures()[loc]
+            if info["n_reg"]:
+                greg[m] = gs.unpack_lanes(sim.read_registers())[:, loc].T
+        t = time.perf_counter()
+        for j in range(subs):
+            sim.set_lane_offset(lane_offset + j * lanes)
+            sim.step(vc)
+            record(j)
+        vdt = time.perf_counter() - t
+        parity, cpu = oracle_parity_and_rate(nl, cfg, sample, vc, gsig, greg)
+        parity["gpu_verification_pass_s"] = round(vdt, 2)
+        cpu["per_core"] = oracle_per_core(nl, cfg, args.core_seconds)
 
     if rank == 0:
+        nranks = nccl_nranks(nccl_log) if world > 1 and args.dist_backend == "nccl" else None
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+            "scaling": "strong" if sharded else "weak", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic",
             "config": {"workload": f"{cfg.name}: {cfg.label}", "gates": G, "registers": info["n_reg"],
-                       "levels": info["n_levels"], "lanes_per_gpu": lanes_rank, "lanes_total": lanes_rank * world,
+                       "levels": info["n_levels"], "lanes_total": lanes_total, "lanes_per_gpu": lanes_rank,
                        "sub_batches_per_gpu": subs, "lanes_per_sub_batch": lanes,
-                       "cycles_per_step": C, "kernel": args.kernel, "balance": True,
-                       "lane_slabs": args.lane_slabs, "lut_unroll": args.lut_unroll,
-                       "lane_groups": sim.config["lane_groups"],
-                       "df_interleave": args.df_interleave, "df_gpw": args.df_gpw,
-                       "pdl": not args.no_pdl, "tile_words": args.tile_words,
-                       "tile_groups": args.tile_groups, "tile_slots_global": args.tile_slots_global,
-                       "l2_hints": args.l2_hints, "lut_k": args.lut_k, "order": args.order,
-                       "grid_stride": not args.no_grid_stride,
-                       "l2": "inputs larger than L2 (state %.1f GB per GPU)" % (info["n_rows"] * lanes / 8 / 1e9),
-                       "step": f"{C} cycles over every lane of the GPU" + (
-                           f" ({subs} sub-batches of {lanes} lanes, each from reset)" if subs > 1 else ""),
+                       "cycles_per_step": C, "kernel": args.kernel, "balance": not args.no_balance,
+                       "lut_unroll": args.lut_unroll, "lane_groups": sim.config["lane_groups"],
+                       "pdl": not args.no_pdl, "tile_words": args.tile_words, "tile_groups": args.tile_groups,
+                       "lut_k": args.lut_k, "grid_stride": not args.no_grid_stride,
+                       "l2": "inputs larger than L2 (state %.1f GB per sub-batch)" % (info["n_rows"] * lanes / 8 / 1e9),
+                       "step": (f"the whole batch: {subs} sub-batch(es) of {lanes} lanes per GPU, each from reset "
+                                f"for {C} cycles" if sharded else f"{C} more cycles over every lane of the GPU"),
                        "parallelism": f"dp{world} (stimulus sharding)" + (" TEST: all ranks on cuda:0"
                                                                               if args.same_device else ""),
-                       "compile_s": round(compile_s, 2),
+                       "compile_s": round(compile_s, 2), "build_id": gs.build_id(),
+                       "program_hash": str(info["program_hash"]),
                        "paper_style_gcps": value * (G + info["n_reg"]) / G},
             "gpu_launches": int(launches_per_cycle * (1 if args.kernel == "tile" else C) * args.steps * subs),
             "signature": {k: str(v) for k, v in red.items()},
+            "nccl": ({"nranks": nranks, "ok": nranks == world} if nranks is not None else None),
             "clocks": clk,
             "roofline": roof,
+            "parity": parity,
             "cpu_baseline": cpu,
             "e2e": e2e,
         }

@@ -44,7 +44,7 @@
 extern "C" {
 #endif
 
-#define GSIM_VERSION "0.1.0"
+#define GSIM_VERSION "0.2.0"
 #define GS_MAX_K 6        /* largest fan-in of gs_add_gate (the table fits one uint64)        */
 #define GS_MAX_K_POLY 8   /* largest LUT fan-in L of the netlist, the compiler and every kernel
                              ("4, 6 or 8"); tables of up to 2^8 bits (gs_add_gate_wide) */
@@ -70,6 +70,10 @@ typedef struct gs_sim gs_sim;
 /* Thread-local text of the last error (never NULL; "" after success). */
 const char* gs_last_error(void);
 const char* gs_version(void);
+/* Build identity of the loaded library: a hash of every source file and compiler flag it was
+ * built from (set by the in-tree build).  Measurement files keyed by it (profiles/traffic.json)
+ * are refused by bench.py when the kernels changed since they were captured. */
+const char* gs_build_id(void);
 
 /* ======================================================================= netlist
  * Nets are numbered in creation order by the incremental calls.  Every add_*
@@ -154,10 +158,6 @@ typedef struct {
                          RANDOM level in [1 + max level of its gate inputs, ALAP] (a valid
                          assignment of the same depth; results must not depend on it, a
                          property test of DESIGN.md reading R11).                      */
-    uint32_t order;       /* gate order inside a level (the level's execution order; results
-                         never depend on it).  0: by fan-in k, then gate id.  1: recency —
-                         gates whose newest input from the previous level was written last
-                         go first, so a level starts on the rows most likely still in L2.  */
 } gs_compile_opts;
 
 /* Validate (GS_ERR_UNDRIVEN, GS_ERR_COMB_LOOP, GS_ERR_ARITY), optionally collapse cones
@@ -201,9 +201,12 @@ gs_status gs_program_coeffs(const gs_program* prog, uint32_t gate, int32_t* w, u
 gs_status gs_program_gate_lut(const gs_program* prog, uint32_t gate, uint32_t* k, gs_net* in, uint64_t* tt);
 
 /* Persist / restore a compiled program (the paper's saved network model, Fig. 1):
- * a binary file of every table the simulator uses plus the query tables; loading checks the
- * format and the program hash (GS_ERR_ARG on a foreign, truncated or edited file).  The
- * loaded program behaves exactly like the one saved (same program_hash). */
+ * a binary file of every table the simulator uses plus the query tables.  Loading checks the
+ * format, a checksum, every table size, every index (row references in range and from an
+ * earlier level, register / output / latch maps, term and coefficient offsets monotonic and
+ * inside their arrays) and the program hash, and returns GS_ERR_ARG on a foreign, truncated,
+ * edited or inconsistent file.  The loaded program behaves exactly like the one saved (same
+ * program_hash). */
 gs_status gs_program_save(const gs_program* prog, const char* path);
 gs_status gs_program_load(const char* path, gs_program** out);
 
@@ -219,15 +222,14 @@ enum {
                              (resident or TMA-streamed) and the levels average <= 400
                              gates (or lanes < 32,768); else GS_KERNEL_LUT               */
     GS_KERNEL_LUT = 1,    /* kernel A: bit-sliced LUT evaluation, 64 stimuli per word      */
-    GS_KERNEL_POLY = 2,   /* kernel B: the paper's network, sum_S w_S Theta(sum x - |S| + 1)
-                             per stimulus in int32, ballot-packed (Eq. 1-3)                */
+    GS_KERNEL_POLY = 2,   /* kernel B: the paper's network (Eq. 1-3, Fig. 2) in exact
+                             integer arithmetic, bit-sliced: per nonzero monomial S
+                             the hidden neuron Theta(sum_{s in S} x_s - |S| + 1) as a
+                             bit-plane counter, the output neuron sum_S w_S h_S as a
+                             two's-complement bit-plane accumulator; outputs outside {0,1}
+                             are counted                                            */
     GS_KERNEL_AB = 3,     /* A writes, B recomputes every level and counts mismatches      */
-    GS_KERNEL_DATAFLOW = 4, /* kernel A evaluation in ONE persistent launch per cycle: lanes cut
-                             into slabs, (slab, level, gate chunk) items from a work queue, an
-                             item waits only for the previous level of its slab, so a slab's
-                             recent levels are read from L2 (DESIGN.md §6 "kernel D").
-                             Needs lanes/lane_slabs in {4096, 8192, 16384}.  Experimental:
-                             measured slower than LUT on C2-C4.              */
+    /* 4: retired in 0.2.0 (an experimental persistent schedule, measured slower than A)   */
     GS_KERNEL_TILE = 5     /* kernel T: each CTA owns a tile of 32*tile_words lanes and runs
                              every level of every cycle of a gs_sim_step in shared memory
                              (gate values in slots reused by live range); one launch per
@@ -245,13 +247,7 @@ typedef struct {
     const uint32_t* trace_words;  /* [n_trace_words] local word indices (copied)           */
     uint32_t trace_cycles;        /* capacity of the trace, in cycles                      */
     int use_graphs;               /* 1: replay each cycle as a CUDA graph (default)        */
-    uint32_t lane_slabs;          /* LUT: run all levels on 1/lane_slabs of the lanes at a
-                                     time so recent levels stay L2-resident (0/1 = off); needs
-                                     (lanes/128) % lane_slabs == 0 and slabs >= 4096 lanes.
-                                     DATAFLOW: number of slabs (0 = lanes/4096)              */
     uint32_t lut_unroll;          /* kernel A: max 16-byte vectors per thread (0 = auto)   */
-    uint32_t df_interleave;       /* DATAFLOW: slabs walked level by level together (0 = 8) */
-    uint32_t df_gates_per_warp;   /* DATAFLOW: gates per warp per work item, 1..32 (0 = 8) */
     uint32_t flags;               /* GS_SIM_* bits below                                   */
     uint32_t tile_words;          /* TILE: 32-bit words per slot, lanes per tile = 32 * this
                                      (4, 8, 16, 32 or 64; 0 = auto); lanes % (32 * it) == 0 */
@@ -260,19 +256,13 @@ typedef struct {
     uint32_t lane_groups;         /* LUT: cut the lanes into this many groups whose level
                                      chains run CONCURRENTLY every cycle (parallel branches of
                                      the cycle's CUDA graph / streams), so one group's level
-                                     ramp and drain overlap another's levels.  With
-                                     lane_slabs = S > 1 each group runs its lanes as S slabs,
-                                     slab-major.  Needs (lanes/128) % (groups x S) == 0 and
-                                     >= 4096 lanes per slab.  0 = auto, 1 = off. */
+                                     ramp and drain overlap another's levels.  Needs
+                                     (lanes/128) % groups == 0 and a multiple of 4096 lanes
+                                     per group.  0 = auto, 1 = off.           */
 } gs_sim_opts;
 /* flags: launch the per-cycle kernels WITHOUT programmatic dependent launch (by default a
  * level kernel may become resident while its predecessor drains; A/B measurement only). */
 #define GS_SIM_NO_PDL 1u
-/* flags: kernel A stores a gate row that the next level reads with L2 evict_last and all
- * other rows with evict_first (the compiler marks the rows). */
-#define GS_SIM_L2_HINTS 2u
-/* flags: with GS_SIM_L2_HINTS, also load gate inputs with L2 evict_first. */
-#define GS_SIM_L2_HINT_LOADS 4u
 /* flags: kernel A launches one CTA per work chunk instead of a grid-stride grid sized to
  * the resident capacity (A/B measurement only). */
 #define GS_SIM_NO_GRID_STRIDE 8u
@@ -281,17 +271,9 @@ typedef struct {
  * shared memory if the whole table fits, else the TMA stream, else global. */
 #define GS_SIM_TILE_DESC_GLOBAL 16u
 #define GS_SIM_TILE_DESC_TMA 32u
-/* flags (kernel A): gather a level's input rows with bulk copies (cp.async.bulk, whole-row
- * chunks of 2-8 KB staged in a shared-memory ring by a producer warp) on every
- * level whose gates all have 1 <= k <= 4 and whose rows are 2, 4 or 8 KB x a power of two;
- * or never.  Default: never (measured slower than the register gathers on C3-C5). */
-#define GS_SIM_LUT_BULK 64u
-#define GS_SIM_LUT_NO_BULK 128u
-/* flags (kernel T): keep each thread group's live slots in a private region of the device
- * workspace (served by L1 and L2) instead of shared memory, so circuits whose live state
- * does not fit shared memory (up to 65,535 live slots) still run tile by tile with no
- * per-level launch; 128- or 256-lane tiles.  Default: off. */
-#define GS_SIM_TILE_SLOTS_GLOBAL 256u
+/* Retired in 0.2.0 (measured slower, DESIGN.md §6 "removed"): flag bits 2, 4 (L2 eviction
+ * hints), 64, 128 (bulk-copy gathers) and 256 (kernel T slots in global memory) are rejected
+ * with GS_ERR_ARG. */
 
 /* Device workspace bytes required for (prog, opts). */
 gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts, size_t* bytes);
@@ -338,8 +320,9 @@ gs_status gs_sim_sync(gs_sim* sim);
  * device->host copy of chunk i-1 run on a library-owned copy stream while chunk i is
  * computed (pinned host buffers required for overlap).  Uses a library-owned device
  * staging buffer (2 x chunk of inputs and outputs, freed by gs_sim_destroy).  Asynchronous
- * on the sim's stream: host_out is complete after gs_sim_sync.  Afterwards the stimulus
- * binding is the last chunk (bind again before gs_sim_step). */
+ * on the sim's stream: host_out is complete after gs_sim_sync.  Afterwards a generated
+ * binding that was in place before the call is restored; any other binding is cleared
+ * (gs_sim_step returns GS_ERR_STATE until the caller binds again). */
 gs_status gs_sim_run_streamed(gs_sim* sim, const uint64_t* host_stim, uint64_t* host_out, uint32_t ncycles,
                               uint32_t chunk);
 gs_status gs_sim_get_cycle(const gs_sim* sim, uint64_t* cycle);
@@ -376,6 +359,9 @@ typedef struct {
     double level_ms, total_ms;
     uint64_t level_launches, total_launches;
     double level_bytes;
+    uint64_t grid_stride_launches;  /* kernel A level launches (host launch decisions; with lane
+                                       groups one per captured graph) whose grid was capped at
+                                       the resident CTA capacity, grid-striding over the level */
 } gs_profile;
 gs_status gs_sim_profile_step(gs_sim* sim, uint32_t ncycles, gs_profile* out);
 

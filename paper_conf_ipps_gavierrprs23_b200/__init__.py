@@ -26,15 +26,11 @@ GS_ERR_BUFFER_TOO_SMALL, GS_ERR_CUDA, GS_ERR_STATE, GS_ERR_NOMEM = -5, -6, -7, -
 GS_MAX_K = 6
 GS_MAX_K_POLY = 8
 GS_SIM_NO_PDL = 1
-GS_SIM_LUT_BULK = 64          # kernel A: bulk-copy staged gathers on (where eligible)
-GS_SIM_LUT_NO_BULK = 128      # ... off
+GS_SIM_NO_GRID_STRIDE = 8     # kernel A: one CTA per work chunk (A/B measurement only)
 GS_SIM_TILE_DESC_GLOBAL = 16  # kernel T: descriptors read from global memory
 GS_SIM_TILE_DESC_TMA = 32     # kernel T: descriptors TMA-streamed level by level
-GS_SIM_TILE_SLOTS_GLOBAL = 256  # kernel T: live slots in the workspace (L1/L2), not shared memory
-GS_KERNEL_AUTO, GS_KERNEL_LUT, GS_KERNEL_POLY, GS_KERNEL_AB, GS_KERNEL_DATAFLOW = 0, 1, 2, 3, 4
-GS_KERNEL_TILE = 5
-KERNELS = {"auto": 0, "lut": 1, "A": 1, "poly": 2, "B": 2, "ab": 3, "AB": 3, "df": 4, "dataflow": 4,
-           "tile": 5, "T": 5}
+GS_KERNEL_AUTO, GS_KERNEL_LUT, GS_KERNEL_POLY, GS_KERNEL_AB, GS_KERNEL_TILE = 0, 1, 2, 3, 5
+KERNELS = {"auto": 0, "lut": 1, "A": 1, "poly": 2, "B": 2, "ab": 3, "AB": 3, "tile": 5, "T": 5}
 
 
 class GsError(RuntimeError):
@@ -57,8 +53,7 @@ class gs_netlist_counts(C.Structure):
 
 
 class gs_compile_opts(C.Structure):
-    _fields_ = [("balance", C.c_int), ("max_k", C.c_uint32), ("lut_k", C.c_uint32), ("level_seed", C.c_uint64),
-                ("order", C.c_uint32)]
+    _fields_ = [("balance", C.c_int), ("max_k", C.c_uint32), ("lut_k", C.c_uint32), ("level_seed", C.c_uint64)]
 
 
 class gs_program_info(C.Structure):
@@ -79,10 +74,8 @@ class gs_sim_opts(C.Structure):
     _fields_ = [("device", C.c_int), ("stream", C.c_void_p), ("lanes", C.c_uint64),
                 ("lane_offset", C.c_uint64), ("kernel", C.c_int), ("n_trace_words", C.c_uint32),
                 ("trace_words", C.c_void_p), ("trace_cycles", C.c_uint32), ("use_graphs", C.c_int),
-                ("lane_slabs", C.c_uint32), ("lut_unroll", C.c_uint32),
-                ("df_interleave", C.c_uint32), ("df_gates_per_warp", C.c_uint32),
-                ("flags", C.c_uint32), ("tile_words", C.c_uint32), ("tile_groups", C.c_uint32),
-                ("lane_groups", C.c_uint32)]
+                ("lut_unroll", C.c_uint32), ("flags", C.c_uint32), ("tile_words", C.c_uint32),
+                ("tile_groups", C.c_uint32), ("lane_groups", C.c_uint32)]
 
 
 class gs_signature(C.Structure):
@@ -96,7 +89,8 @@ class gs_signature(C.Structure):
 
 class gs_profile(C.Structure):
     _fields_ = [("level_ms", C.c_double), ("total_ms", C.c_double), ("level_launches", C.c_uint64),
-                ("total_launches", C.c_uint64), ("level_bytes", C.c_double)]
+                ("total_launches", C.c_uint64), ("level_bytes", C.c_double),
+                ("grid_stride_launches", C.c_uint64)]
 
 
 # ------------------------------------------------------------------ loading
@@ -104,6 +98,7 @@ _P = C.c_void_p
 _SIGS = {
     "gs_last_error": (C.c_char_p, []),
     "gs_version": (C.c_char_p, []),
+    "gs_build_id": (C.c_char_p, []),
     "gs_netlist_create": (C.c_int32, [_P]),
     "gs_netlist_destroy": (C.c_int32, [_P]),
     "gs_add_input": (C.c_int32, [_P, _P]),
@@ -253,17 +248,16 @@ class Netlist:
         _call("gs_netlist_get_counts", self.h, C.byref(c))
         return {f: int(getattr(c, f)) for f, _ in c._fields_}
 
-    def compile(self, balance: bool = True, max_k: int = 0, lut_k: int = 0, level_seed: int = 0,
-                order: int = 0) -> "Program":
-        return Program(self, balance, max_k, lut_k, level_seed=level_seed, order=order)
+    def compile(self, balance: bool = True, max_k: int = 0, lut_k: int = 0, level_seed: int = 0) -> "Program":
+        return Program(self, balance, max_k, lut_k, level_seed=level_seed)
 
 
 class Program:
     def __init__(self, netlist: Netlist | None, balance: bool = True, max_k: int = 0, lut_k: int = 0,
-                 _handle=None, level_seed: int = 0, order: int = 0):
+                 _handle=None, level_seed: int = 0):
         if _handle is None:
             h = C.c_void_p()
-            o = gs_compile_opts(1 if balance else 0, max_k, lut_k, int(level_seed), int(order))
+            o = gs_compile_opts(1 if balance else 0, max_k, lut_k, int(level_seed))
             _call("gs_compile", netlist.h, C.byref(o), C.byref(h))
         else:
             h = _handle
@@ -320,8 +314,7 @@ class Sim:
 
     def __init__(self, program: Program, lanes: int, lane_offset: int = 0, kernel="lut",
                  device: int = 0, stream=None, trace_words=(), trace_cycles: int = 0,
-                 use_graphs: bool = True, lane_slabs: int = 0, lut_unroll: int = 0,
-                 df_interleave: int = 0, df_gates_per_warp: int = 0, pdl: bool = True,
+                 use_graphs: bool = True, lut_unroll: int = 0, pdl: bool = True,
                  tile_words: int = 0, tile_groups: int = 0, flags: int = 0, lane_groups: int = 0):
         import torch
         self.program = program
@@ -332,8 +325,7 @@ class Sim:
         o = gs_sim_opts(device, C.c_void_p(self.stream.cuda_stream), self.lanes, int(lane_offset),
                         KERNELS[kernel] if isinstance(kernel, str) else int(kernel), len(self._tw),
                         _p(self._tw) if len(self._tw) else None, int(trace_cycles),
-                        1 if use_graphs else 0, int(lane_slabs), int(lut_unroll),
-                        int(df_interleave), int(df_gates_per_warp),
+                        1 if use_graphs else 0, int(lut_unroll),
                         (0 if pdl else GS_SIM_NO_PDL) | int(flags), int(tile_words), int(tile_groups),
                         int(lane_groups))
         nbytes = C.c_size_t()
@@ -451,6 +443,11 @@ class Sim:
 
 def version() -> str:
     return lib().gs_version().decode()
+
+
+def build_id() -> str:
+    """Hash of the sources and flags libgsim.so was built from (gs_build_id)."""
+    return lib().gs_build_id().decode()
 
 
 def unpack_lanes(words: np.ndarray) -> np.ndarray:

@@ -6,6 +6,7 @@ from __future__ import annotations
 
 import concurrent.futures as cf
 import glob
+import hashlib
 import os
 import subprocess
 import sys
@@ -32,6 +33,18 @@ def _deps():
             + [os.path.join(ROOT, "include", "gsim.h")])
 
 
+def build_id() -> str:
+    """Hash of every source / header and every compiler flag: the identity of the kernels in
+    libgsim.so (gs_build_id()), used to refuse stale measurement files (bench.py)."""
+    h = hashlib.sha256()
+    for f in sorted(_deps()):
+        h.update(os.path.relpath(f, ROOT).encode())
+        with open(f, "rb") as fh:
+            h.update(fh.read())
+    h.update(" ".join(ARCH + COMMON + EXTRA).encode())
+    return h.hexdigest()[:16]
+
+
 def up_to_date() -> bool:
     if not os.path.exists(LIB):
         return False
@@ -44,9 +57,12 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     os.makedirs(OBJ, exist_ok=True)
     jobs = []
+    bid = build_id()
     for src in _sources():
         obj = os.path.join(OBJ, os.path.basename(src) + ".o")
         cmd = [NVCC, *ARCH, *COMMON, *EXTRA, "-c", src, "-o", obj]
+        if os.path.basename(src) == "netlist.cpp":
+            cmd.append(f'-DGS_BUILD_ID="{bid}"')
         if src.endswith(".cu"):
             cmd += ["-Xptxas", "-v"] if verbose else []
         jobs.append((cmd, obj))

@@ -11,6 +11,7 @@
 //  * row layout + per-level SoA descriptors for the device.
 #include <algorithm>
 #include <cstring>
+#include <memory>
 #include <queue>
 
 #include "internal.h"
@@ -191,17 +192,14 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
     }
 
     // ---------------------------------------------------------------- execution order
-    Program* p = new Program();
+    std::unique_ptr<Program> p(new Program());   // freed on every early return / exception
     Program& pr = *p;
     pr.n_pi = P; pr.n_reg = R; pr.n_po = O; pr.n_gates = G; pr.n_eval = n_eval; pr.n_levels = D;
     pr.row_pi0 = 2;
     pr.row_q0 = 2 + P;
     pr.row_gate0 = 2 + P + 2 * R;
     pr.n_rows = (uint64_t)pr.row_gate0 + n_eval;
-    if (pr.n_rows >= QFLAG) {
-        delete p;
-        return fail(GS_ERR_ARG, "gs_compile: too many state rows");
-    }
+    if (pr.n_rows >= QFLAG) return fail(GS_ERR_ARG, "gs_compile: too many state rows");
 
     // counting sort by (level, k), stable in gate id
     pr.level_off.assign(D + 1, 0);
@@ -212,43 +210,13 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
     for (uint32_t l = 0; l <= D; ++l) pr.level_off[l] = (uint32_t)bucket[(uint64_t)l * (GS_MAX_K_POLY + 1)];
     std::vector<uint32_t> exec_pos(G, NONE32);
     pr.exec_gate.assign(n_eval, 0);
-    if (opts.order == 0) {
-        for (uint32_t g = 0; g < G; ++g)
-            if (nl.gate_k[g] > 0) {
-                uint64_t b = (uint64_t)(level[g] - 1) * (GS_MAX_K_POLY + 1) + nl.gate_k[g];
-                uint32_t pos = (uint32_t)bucket[b]++;
-                exec_pos[g] = pos;
-                pr.exec_gate[pos] = g;
-            }
-    } else {
-        // recency order: level by level, a gate's key is the latest execution position among
-        // its inputs from the previous level; larger keys first (LIFO with respect to the
-        // previous level's stores), ties by gate id.  Level offsets are unchanged.
-        std::vector<std::vector<uint32_t>> by_level(D);
-        for (uint32_t g = 0; g < G; ++g)
-            if (nl.gate_k[g] > 0) by_level[level[g] - 1].push_back(g);
-        uint32_t pos = 0;
-        std::vector<std::pair<int64_t, uint32_t>> key;
-        for (uint32_t l = 0; l < D; ++l) {
-            key.clear();
-            for (uint32_t g : by_level[l]) {
-                int64_t m = -1;
-                for (uint32_t j = nl.gate_in_off[g]; j < nl.gate_in_off[g + 1]; ++j) {
-                    const uint32_t n = nl.gate_in[j];
-                    if (nl.net_kind[n] != NET_GATE) continue;
-                    const uint32_t h = nl.net_index[n];
-                    if (nl.gate_k[h] > 0 && level[h] + 1 == level[g]) m = std::max<int64_t>(m, exec_pos[h]);
-                }
-                key.push_back({-m, g});
-            }
-            std::sort(key.begin(), key.end());
-            for (auto& kg : key) {
-                exec_pos[kg.second] = pos;
-                pr.exec_gate[pos] = kg.second;
-                ++pos;
-            }
+    for (uint32_t g = 0; g < G; ++g)
+        if (nl.gate_k[g] > 0) {
+            uint64_t b = (uint64_t)(level[g] - 1) * (GS_MAX_K_POLY + 1) + nl.gate_k[g];
+            uint32_t pos = (uint32_t)bucket[b]++;
+            exec_pos[g] = pos;
+            pr.exec_gate[pos] = g;
         }
-    }
 
     auto row_of = [&](uint32_t n) -> uint32_t {
         uint32_t i = nl.net_index[n];
@@ -283,14 +251,6 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
         }
         pr.aux[pos].qdst = NONE32;
         pr.aux[pos].k = k;
-    }
-    // "hot" rows: read by a gate of the very next level (kernel A keeps them in L2 with
-    // an evict_last store)
-    pr.hot.assign(n_eval, 0);
-    for (uint32_t g = 0; g < G; ++g) {
-        if (nl.gate_k[g] == 0) continue;
-        for (uint32_t e = cons_off[g]; e < cons_off[g + 1]; ++e)
-            if (level[cons[e]] == level[g] + 1) { pr.hot[exec_pos[g]] = 1; break; }
     }
     // registers: fuse the latch into the D-driving gate's store when possible (the
     // recurrent connection of P:241 becomes a dual store into the other Q bank)
@@ -365,7 +325,7 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
     in.hidden_neurons = hidden;
     in.n_rows = pr.n_rows;
     in.program_hash = program_hash(pr);
-    out = p;
+    out = p.release();
     return GS_OK;
 }
 

@@ -22,44 +22,6 @@ __device__ __forceinline__ unsigned long long dmix64(unsigned long long z) {
     return z ^ (z >> 31);
 }
 
-// ------------------------------------------------------------- L2 eviction priority
-// createpolicy / st.global.L2::cache_hint: a row the next level reads is stored
-// evict_last (kept in L2 for its consumers), every other row evict_first (streamed to HBM
-// without displacing the kept rows).
-__device__ __forceinline__ uint64_t l2_policy_last() {
-    uint64_t p;
-    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
-    return p;
-}
-__device__ __forceinline__ uint64_t l2_policy_first() {
-    uint64_t p;
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-    return p;
-}
-__device__ __forceinline__ void st_hint(uint4* ptr, const uint4& v, uint64_t pol) {
-    asm volatile("st.global.L2::cache_hint.v4.u32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(ptr), "r"(v.x), "r"(v.y),
-                 "r"(v.z), "r"(v.w), "l"(pol)
-                 : "memory");
-}
-// the same store under an explicit predicate operand (no fused latch: store nothing).  A
-// C-level `if (qd) st_hint(qd + u * 32, ...)` was compiled into an unconditional store: the
-// pointer arithmetic let the compiler assume qd != nullptr (compute-sanitizer: 16-byte writes
-// to addresses 0x0 / 0x200 in k_level_lut_wide<4, true> on C4).
-__device__ __forceinline__ void st_hint_if(uint4* ptr, const uint4& v, uint64_t pol, uint32_t pred) {
-    asm volatile(
-        "{\n .reg .pred p;\n setp.ne.u32 p, %6, 0;\n"
-        " @p st.global.L2::cache_hint.v4.u32 [%0], {%1, %2, %3, %4}, %5;\n}\n" ::"l"(ptr),
-        "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "l"(pol), "r"(pred)
-        : "memory");
-}
-__device__ __forceinline__ uint4 ld_hint(const uint4* ptr, uint64_t pol) {
-    uint4 v;
-    asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
-                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
-                 : "l"(ptr), "l"(pol));
-    return v;
-}
-
 // ------------------------------------------------------- programmatic dependent launch
 // Every kernel of the per-cycle chain is launched with programmatic stream serialization
 // (when enabled): it may become resident while its predecessor drains, and waits at

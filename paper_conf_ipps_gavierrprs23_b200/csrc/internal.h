@@ -4,6 +4,8 @@
 #pragma once
 
 #include <cstdint>
+#include <exception>
+#include <new>
 #include <string>
 #include <vector>
 
@@ -25,6 +27,19 @@ struct NvtxRange {
 void set_error(const std::string& msg);
 void clear_error();
 gs_status fail(gs_status code, const std::string& msg);
+
+// Every extern "C" body runs inside GS_TRY: no C++ exception crosses the ABI (gsim.h).
+// Variadic, so a body with top-level commas (declarations, templates) passes through intact.
+#define GS_TRY(...)                                                   \
+    try {                                                             \
+        __VA_ARGS__                                                   \
+    } catch (const std::bad_alloc&) {                                 \
+        return ::gs::fail(GS_ERR_NOMEM, "out of host memory");        \
+    } catch (const std::exception& e) {                               \
+        return ::gs::fail(GS_ERR_ARG, e.what());                      \
+    } catch (...) {                                                   \
+        return ::gs::fail(GS_ERR_ARG, "unexpected exception");        \
+    }
 
 // ---------------------------------------------------------------- netlist
 enum NetKind : uint8_t { NET_PI = 0, NET_REG = 1, NET_GATE = 2 };
@@ -52,8 +67,8 @@ struct Netlist {
 };
 
 // ---------------------------------------------------------------- program
-constexpr uint32_t QFLAG = 0x80000000u;
-constexpr uint32_t GS_MAX_K_LUT64 = 6;    // widest LUT whose table fits GateAux::tt (64 bits)   // row ref is a Q row: add the current bank offset
+constexpr uint32_t QFLAG = 0x80000000u;   // row ref is a Q row: add the current bank offset
+constexpr uint32_t GS_MAX_K_LUT64 = 6;    // widest LUT whose table fits GateAux::tt (64 bits)
 constexpr uint32_t NONE32 = 0xFFFFFFFFu;
 
 // 16-byte per-gate auxiliary descriptor (device layout, see kernels.cu)
@@ -76,7 +91,6 @@ struct Program {
     std::vector<uint32_t> in_lo;              // [n_eval * 4] row refs (QFLAG for Q rows)
     std::vector<uint32_t> in_hi;              // [n_eval * 4] (inputs 4..7) if any_wide
     std::vector<GateAux> aux;                 // [n_eval]
-    std::vector<uint8_t> hot;                 // [n_eval] a gate of the next level reads it
     std::vector<uint64_t> tt_full;            // [n_eval * 4] 256-bit tables if max_k > 6
     std::vector<uint32_t> term_off;           // [n_eval + 1] kernel B nonzero terms
     std::vector<uint32_t> terms;              // S | (|S|-1)<<8 | (w & 0xffff)<<16

@@ -39,14 +39,11 @@ struct LevelArgs {
     uint32_t row_gate0;
     uint32_t qcur, qnext;             // bank offsets (0 or n_reg) for Q refs / latch stores
     Ctl* ctl;
-    uint32_t vec0, vslab;             // lane slab in 16-byte vectors (vslab 0 = whole row)
+    uint32_t vec0, vslab;             // lane group in 16-byte vectors (vslab 0 = whole row)
     uint32_t unroll;                  // max vectors per thread on the wide path (0 = auto)
     uint32_t pdl;                     // launch with programmatic stream serialization
     uint32_t min_warps;               // auto U: prefer smaller U below this many warps
-    uint32_t hint;                    // L2 eviction-priority stores (aux.k bit 8 = read next level)
-    uint32_t hint_ld;                 // ... and evict_first input loads
     uint32_t grid_blocks;             // wide path: cap the grid at the resident capacity (0 = off)
-    uint32_t bulk;                    // gather input rows with bulk copies (k_level_bulk)
     uint32_t sms;                     // multiprocessors of the device
 };
 
@@ -67,29 +64,6 @@ struct EndArgs {
     unsigned long long* trace;        // [trace_cap][n_po][ntw]
     uint32_t ntw, trace_cap;
     uint32_t pdl;
-};
-
-// Persistent slab-dataflow schedule of kernel A (kernels.cu, DESIGN.md §6 "kernel D"):
-// one launch per cycle runs every (lane slab, level, gate chunk) item; an item waits
-// only for the previous level of its own slab.
-struct DfArgs {
-    const uint4* din;
-    const GateAux* aux;
-    const uint4* dhi;                 // inputs 4..7 (gates with k > 4)
-    const uint4* dtt;                 // [n_eval][2] full 256-bit tables (programs with k > 6)
-    uint8_t* state;
-    uint64_t stride;
-    uint32_t row_gate0, qcur, qnext;
-    const uint32_t* lv_gate0;         // [nl + 1] exec-order first gate of compact level i
-    const uint32_t* lv_item0;         // [nl + 1] prefix sum of items per level (one slab)
-    uint32_t nl;                      // non-empty levels
-    uint32_t items_per_slab;          // lv_item0[nl]
-    uint32_t n_slabs, interleave;     // slabs; slabs walked level-by-level together
-    uint32_t slab_vec;                // 16-byte vectors per slab row (32 * VPL)
-    uint32_t gpw;                     // gates per warp per work item (item = 8 warps)
-    uint32_t total_items;
-    unsigned int* qhead;              // work-queue head (zeroed every cycle)
-    unsigned int* done;               // [n_slabs * nl] finished items (zeroed every cycle)
 };
 
 // Kernel T (kernels_tile.cu): one lane tile per CTA at a time, all levels x all cycles of
@@ -123,7 +97,6 @@ struct TileArgs {
     uint32_t ntw, trace_cap;
     uint64_t word_off;                // global 64-bit word of local lane 0
     uint32_t ncycles, n_tiles;
-    uint4* gslots;                    // desc_smem & 4: per-group slot regions [grid*NG][n_slots][TW/4]
 };
 size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
                        int desc_mode, uint32_t max_width);
@@ -131,14 +104,10 @@ cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_ev
                        int desc_smem, uint32_t max_width, uint32_t has_q, uint32_t* per_sm);
 cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s);
 
-cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s);
-// kernel A with bulk-copy staged gathers: chunk bytes used for rows of `words` 64-bit words
-// (slab of vslab 16-byte vectors when nonzero), 0 = rows not eligible
-uint32_t level_bulk_chunk(uint32_t words, uint32_t vslab);
-cudaError_t launch_level_bulk(const LevelArgs& a, cudaStream_t s);
+// *grid_stride (may be NULL) is set to 1 when the launch's grid was capped at the resident
+// capacity (the grid-stride branch), else 0
+cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s, uint32_t* grid_stride = nullptr);
 uint32_t level_lut_resident_blocks(int device);   // CTAs of k_level_lut_wide resident on the GPU
-cudaError_t launch_dataflow(const DfArgs& a, uint32_t grid, cudaStream_t s);
-cudaError_t dataflow_grid(uint32_t slab_vec, int device, uint32_t* grid);
 cudaError_t launch_level_poly(const LevelArgs& a, int check_only, cudaStream_t s);
 cudaError_t launch_stim(Ctl* ctl, uint8_t* state, uint64_t stride, uint32_t words, uint32_t row_pi0,
                         uint32_t n_pi, uint64_t word_off, uint32_t pdl, cudaStream_t s);

@@ -1,5 +1,5 @@
 // kernels_tile.cu — kernel T dispatch: plan-time setup and launch by tile width (the
-// template instantiations live in kernels_tile_tw{4,8,16,32}.cu).
+// template instantiations live in kernels_tile_tw{4,8,16,32,64}.cu).
 #include "kernels_tile.cuh"
 
 namespace gs {
@@ -8,9 +8,7 @@ static size_t lvl_bytes(uint32_t n_levels) { return (((size_t)n_levels + 1) * 4 
 
 size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
                        int desc_mode, uint32_t max_width) {
-    const bool sg = (desc_mode & 4) != 0;                // slots in global memory: MISR only
-    desc_mode &= 3;
-    size_t b = 0, g = ((sg ? 0 : (size_t)n_slots) + 64) * 4 * tw;
+    size_t b = 0, g = ((size_t)n_slots + 64) * 4 * tw;
     if (desc_mode == 1) b = (size_t)n_eval * 16 + lvl_bytes(n_levels);
     if (desc_mode == 2) {
         b = lvl_bytes(n_levels);

@@ -1,5 +1,5 @@
 // kernels_tile.cuh — kernel T: tile-resident simulation in shared memory (sm_100a).
-// Template definitions; instantiated per tile width in kernels_tile_tw{4,8,16,32}.cu
+// Template definitions; instantiated per tile width in kernels_tile_tw{4,8,16,32,64}.cu
 // (parallel compilation), dispatched by kernels_tile.cu.
 //
 // Stimuli are independent, so a tile of 32*TW lanes can run every level of
@@ -141,10 +141,9 @@ __device__ __forceinline__ void group_sync(uint32_t id, uint32_t nthreads) {
 // group simulates its own tile and synchronises only with itself (named barrier 1 + gid),
 // so one group's level barrier overlaps the other groups' work.  All groups share the
 // descriptor table in shared memory.
-template <int TW, bool HASQ, int NG, int DMS>
+template <int TW, bool HASQ, int NG, int DM>
 __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
-    constexpr int DM = DMS & 3;                          // descriptor mode (0 global, 1 resident, 2 TMA)
-    constexpr bool SG = (DMS & 4) != 0;                  // slots in global memory (L1/L2-resident), not smem
+    // DM: descriptor mode (0 global, 1 resident, 2 TMA)
     constexpr uint32_t V = TW / 4;                       // uint4 per slot
     constexpr uint32_t P = V >= 4 ? TILE_VPT : 1;        // 16-byte vectors per thread and gate
     constexpr uint32_t VS = V / P;                       // threads per gate (vector stride)
@@ -168,16 +167,12 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     }
     const uint32_t gid = threadIdx.x / GT, tid = threadIdx.x % GT, bd = GT;
     const uint32_t bar = 1 + gid;
-    // group region: [mbarriers + descriptor double buffer (mode 2)] [slots (unless SG)] [MISR]
-    uint4* greg = base + (size_t)gid * (((SG ? 0 : a.n_slots) + 64) * V + (DM == 2 ? 1 + 2 * a.max_width : 0));
+    // group region: [mbarriers + descriptor double buffer (mode 2)] [slots] [MISR]
+    uint4* greg = base + (size_t)gid * ((a.n_slots + 64) * V + (DM == 2 ? 1 + 2 * a.max_width : 0));
     uint64_t* mbar = reinterpret_cast<uint64_t*>(greg);
     uint4* dbuf = greg + 1;                                   // [2][max_width]
     uint4* gsm = DM == 2 ? greg + 1 + 2 * a.max_width : greg;
-    // SG: this group's slots are a private region of the workspace (one per resident group),
-    // kept close by L1 (the CTA uses almost no shared memory) and L2; a group's threads see
-    // each other's slot stores across the group barrier (bar.sync orders global memory
-    // within the CTA)
-    uint4* sl = SG ? a.gslots + ((size_t)blockIdx.x * NG + gid) * a.n_slots * V : gsm;
+    uint4* sl = gsm;
     if (DM == 2 && tid == 0) {
         mbar_init(mbar, 1);
         mbar_init(mbar + 1, 1);
@@ -187,7 +182,7 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     const uint32_t mbar_s = smem_u32(mbar);                   // mode 2: the two mbarriers (8 B apart)
     const uint32_t dbuf_s = smem_u32(dbuf);                   // mode 2: descriptor double buffer
     uint32_t* sw = reinterpret_cast<uint32_t*>(sl);          // slots as 32-bit words
-    uint32_t* mp = SG ? reinterpret_cast<uint32_t*>(gsm) : sw + (size_t)a.n_slots * TW;   // MISR planes [64][TW]
+    uint32_t* mp = sw + (size_t)a.n_slots * TW;              // MISR planes [64][TW]
     const unsigned long long c0 = a.ctl->cycle;
     const uint32_t R = a.n_reg, q0 = a.q0;
     const uint32_t w32_row = a.words * 2;                     // 32-bit words per state row

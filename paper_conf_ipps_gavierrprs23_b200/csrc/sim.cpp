@@ -23,49 +23,11 @@ size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 
 struct Layout {
     size_t ctl, state, din, aux, dhi, dtt, term_off, terms, po_rows, latch_src, latch_dst, reg_init,
-        trace_slot, misr, trace, lane_sigs, scratch, lv_gate0, lv_item0, dfctl, dfctl_bytes,
-        t_desc, t_desc_hi, t_po, t_lsrc, t_ldst, t_wbrow, t_wbslot, t_lvl, t_gslots, total;
+        trace_slot, misr, trace, lane_sigs, scratch, t_desc, t_desc_hi, t_po, t_lsrc, t_ldst, t_wbrow,
+        t_wbslot, t_lvl, total;
 };
-
-// Work-item plan of the DATAFLOW schedule (kernels.cu k_dataflow): non-empty levels only
-// (an empty level would break the "previous level done => all earlier levels done" chain).
-struct DfPlan {
-    uint32_t vpl = 0, n_slabs = 0, interleave = 0, gpw = 0, nl = 0;
-    std::vector<uint32_t> lv_gate0, lv_item0;
-};
-
-gs_status df_plan(const Program& p, const gs_sim_opts& o, DfPlan& d) {
-    if (o.kernel != GS_KERNEL_DATAFLOW) return GS_OK;
-    const uint64_t slabs = o.lane_slabs ? o.lane_slabs : o.lanes / 4096;
-    if (slabs == 0 || o.lanes % slabs)
-        return fail(GS_ERR_ARG, "DATAFLOW: lanes must be a multiple of lane_slabs (and of 4096)");
-    const uint64_t sl = o.lanes / slabs;
-    if (sl != 4096 && sl != 8192 && sl != 16384)
-        return fail(GS_ERR_ARG, "DATAFLOW: lanes / lane_slabs must be 4096, 8192 or 16384");
-    d.vpl = (uint32_t)(sl / 4096);
-    d.n_slabs = (uint32_t)slabs;
-    d.interleave = o.df_interleave ? o.df_interleave : 8;
-    if (d.interleave > d.n_slabs) d.interleave = d.n_slabs;
-    d.gpw = o.df_gates_per_warp ? o.df_gates_per_warp : 8;
-    if (d.gpw > 32) return fail(GS_ERR_ARG, "DATAFLOW: df_gates_per_warp must be <= 32");
-    const uint32_t gpi = 8 * d.gpw;              // one item = 8 warps x gpw gates
-    d.lv_gate0.clear();
-    d.lv_item0.assign(1, 0);
-    for (uint32_t l = 0; l < p.n_levels; ++l) {
-        const uint32_t w = p.level_off[l + 1] - p.level_off[l];
-        if (!w) continue;
-        d.lv_gate0.push_back(p.level_off[l]);
-        d.lv_item0.push_back(d.lv_item0.back() + (w + gpi - 1) / gpi);
-    }
-    d.nl = (uint32_t)d.lv_gate0.size();
-    d.lv_gate0.push_back(p.n_eval);
-    if ((uint64_t)d.lv_item0.back() * d.n_slabs >= (1ull << 32))
-        return fail(GS_ERR_ARG, "DATAFLOW: too many work items per cycle; raise df_gates_per_warp");
-    return GS_OK;
-}
 
 struct Plans {
-    DfPlan df;
     TilePlan tile;
     uint32_t tw = 0;                  // kernel T: 32-bit words per slot
     uint32_t ng = 0;                  // kernel T: thread groups (tiles) per CTA
@@ -76,7 +38,6 @@ struct Plans {
 constexpr size_t TILE_SMEM_MAX = 232448;   // 227 KB opt-in shared memory per CTA (sm_100a)
 
 gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
-    if (gs_status st = df_plan(p, o, pl.df)) return st;
     if (o.kernel != GS_KERNEL_TILE) return GS_OK;
     if (gs_status st = tile_plan(p, pl.tile)) return st;
     uint32_t maxw = 0;
@@ -106,7 +67,6 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
     // circuit runs 1.33x faster with TMA and 4x wider tiles than resident with narrow
     // ones), then wider tiles, then resident > TMA stream > global, then fewer groups
     const int forced = (o.flags & GS_SIM_TILE_DESC_GLOBAL) ? 0 : (o.flags & GS_SIM_TILE_DESC_TMA) ? 2 : -1;
-    const int sg = (o.flags & GS_SIM_TILE_SLOTS_GLOBAL) ? 4 : 0;   // slots in global memory
     uint64_t best = 0;
     for (int ds : {1, 2, 0}) {
         if (forced >= 0 && ds != forced) continue;
@@ -114,13 +74,12 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
             if (o.tile_groups && ng != o.tile_groups) continue;
             for (uint32_t tw : {4u, 8u, 16u, 32u, 64u}) {
                 if (o.tile_words && tw != o.tile_words) continue;
-                if (sg && tw > 8) continue;                  // global slots: 16/32-byte slot rows
-                if (o.lanes % (32ull * tw) || smem(tw, ng, ds | sg) > TILE_SMEM_MAX) continue;
+                if (o.lanes % (32ull * tw) || smem(tw, ng, ds) > TILE_SMEM_MAX) continue;
                 const uint64_t inflight = std::min<uint64_t>((uint64_t)ng * tw * 32 * sms, o.lanes);
                 const uint64_t pref = ds == 1 ? 2 : ds == 2 ? 1 : 0;
                 const uint64_t score = ((inflight << (ds == 1 ? 1 : 0)) << 24) | ((uint64_t)tw << 16) | (pref << 12) |
                                        ((8 - ng) << 8);
-                if (score > best) { best = score; pl.tw = tw; pl.ng = ng; pl.desc_smem = ds | sg; }
+                if (score > best) { best = score; pl.tw = tw; pl.ng = ng; pl.desc_smem = ds; }
             }
         }
     }
@@ -154,7 +113,6 @@ gs_sim_opts resolve_auto(const Program& p, const gs_sim_opts& o) {
 }
 
 Layout make_layout(const Program& p, const gs_sim_opts& o, const Plans& pl) {
-    const DfPlan& d = pl.df;
     const TilePlan& t = pl.tile;
     Layout L{};
     const uint64_t words = o.lanes / 64;
@@ -183,10 +141,6 @@ Layout make_layout(const Program& p, const gs_sim_opts& o, const Plans& pl) {
     L.trace = take((size_t)o.trace_cycles * p.n_po * o.n_trace_words * 8);
     L.lane_sigs = take((size_t)o.lanes * 8);
     L.scratch = take((size_t)p.n_po * words * 8);
-    L.lv_gate0 = take(d.lv_gate0.size() * 4);
-    L.lv_item0 = take(d.lv_item0.size() * 4);
-    L.dfctl_bytes = d.nl ? 4 + (size_t)d.n_slabs * d.nl * 4 : 0;
-    L.dfctl = take(L.dfctl_bytes);
     L.t_desc = take(t.desc.size() * sizeof(TileDesc));
     L.t_desc_hi = take(t.desc_hi.size() * 4);   // 48 B per gate when any k > 4
     L.t_po = take(t.po_slot.size() * 4);
@@ -195,9 +149,6 @@ Layout make_layout(const Program& p, const gs_sim_opts& o, const Plans& pl) {
     L.t_wbrow = take(t.wb_row.size() * 4);
     L.t_wbslot = take(t.wb_slot.size() * 4);
     L.t_lvl = take(pl.tw ? p.level_off.size() * 4 : 0);
-    // kernel T with global slots: one region of n_slots x tile bytes per tile (an upper bound
-    // on the resident groups) = n_slots x lanes / 8 bytes
-    L.t_gslots = take((pl.desc_smem & 4) ? (size_t)t.n_slots * (size_t)(o.lanes / 8) : 0);
     L.total = off;
     return L;
 }
@@ -212,7 +163,6 @@ struct gs_sim {
     uint8_t* ws = nullptr;
     cudaStream_t stream = nullptr, cap = nullptr;
     uint32_t words = 0;
-    uint32_t slabs = 1;
     uint64_t stride = 0;
     uint64_t cycle = 0;               // host mirror of Ctl::cycle
     int bound = 0;                    // 0 none, 1 generated, 2 host/device buffer
@@ -227,8 +177,6 @@ struct gs_sim {
     cudaStream_t copy = nullptr;
     cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
     cudaGraphExec_t exec[2] = {nullptr, nullptr};
-    DfPlan df;
-    uint32_t df_grid = 0;
     TilePlan tile;
     uint32_t tw = 0, tile_grid = 0;
     int desc_smem = 0;
@@ -237,14 +185,11 @@ struct gs_sim {
     uint32_t pdl = 1;                 // programmatic dependent launch between cycle kernels
     uint32_t min_warps = 0;           // kernel A auto-U threshold (2 waves of resident warps)
     uint32_t resident_blocks = 0;     // kernel A wide path: CTAs resident on the GPU
-    uint32_t grid_waves = 1;          // grid-stride grid = resident_blocks x this
     uint32_t sms = 148;
-    bool bulk = false;                // kernel A: bulk-copy staged gathers (k_level_bulk)
-    bool concurrent = false;          // lane groups: the slabs' level chains run concurrently
-    uint32_t branches = 1;            // concurrent lane groups; each runs slabs / branches slabs
-    std::vector<cudaStream_t> gstream;  // [slabs - 1] branch streams (group 0: the caller's)
-    std::vector<cudaEvent_t> gev;       // [0] fork, [1 .. slabs - 1] joins
-    std::vector<uint8_t> lv_bulk;     // [n_levels] every gate of the level has 1 <= k <= 4
+    uint32_t groups = 1;              // concurrent lane groups (kernel A), one graph branch each
+    std::vector<cudaStream_t> gstream;  // [groups - 1] branch streams (group 0: the caller's)
+    std::vector<cudaEvent_t> gev;       // [0] fork, [1 .. groups - 1] joins
+    uint64_t grid_stride_launches = 0;  // level launches whose grid was capped at residency
 
     Ctl* ctl() const { return reinterpret_cast<Ctl*>(ws + L.ctl); }
     uint8_t* state() const { return ws + L.state; }
@@ -278,10 +223,7 @@ static LevelArgs level_args(const gs_sim* s, uint32_t l, uint32_t parity) {
     a.ctl = s->ctl();
     a.pdl = s->pdl;
     a.min_warps = s->min_warps;
-    a.hint = (s->opts.flags & GS_SIM_L2_HINTS) ? 1u : 0u;
-    a.hint_ld = (s->opts.flags & GS_SIM_L2_HINT_LOADS) ? 1u : 0u;
-    a.grid_blocks = (s->opts.flags & GS_SIM_NO_GRID_STRIDE) ? 0u : s->resident_blocks * s->grid_waves;
-    a.bulk = (s->bulk && s->lv_bulk[l]) ? 1u : 0u;
+    a.grid_blocks = (s->opts.flags & GS_SIM_NO_GRID_STRIDE) ? 0u : s->resident_blocks;
     a.sms = s->sms;
     return a;
 }
@@ -311,53 +253,26 @@ static EndArgs end_args(const gs_sim* s, uint32_t parity) {
     return e;
 }
 
-static cudaError_t level_launch(const gs_sim* s, uint32_t l, uint32_t parity, cudaStream_t st,
-                                uint32_t slab = 0) {
+static cudaError_t level_launch(gs_sim* s, uint32_t l, uint32_t parity, cudaStream_t st, uint32_t group = 0) {
     LevelArgs a = level_args(s, l, parity);
     a.unroll = s->opts.lut_unroll;
-    if (s->slabs > 1) {
-        a.vslab = (s->words / 2) / s->slabs;
-        a.vec0 = slab * a.vslab;
+    if (s->groups > 1) {
+        a.vslab = (s->words / 2) / s->groups;
+        a.vec0 = group * a.vslab;
     }
+    uint32_t gs_flag = 0;
+    cudaError_t e = cudaSuccess;
     switch (s->opts.kernel) {
         case GS_KERNEL_POLY: return launch_level_poly(a, 0, st);
-        case GS_KERNEL_AB: {
-            cudaError_t e = launch_level_lut(a, st);
+        case GS_KERNEL_AB:
+            e = launch_level_lut(a, st, &gs_flag);
             if (e != cudaSuccess) return e;
-            return launch_level_poly(a, 1, st);
-        }
-        default: return launch_level_lut(a, st);
+            e = launch_level_poly(a, 1, st);
+            break;
+        default: e = launch_level_lut(a, st, &gs_flag); break;
     }
-}
-
-static cudaError_t dataflow_launch(const gs_sim* s, uint32_t parity, cudaStream_t st) {
-    const Program& p = *s->prog;
-    const DfPlan& d = s->df;
-    DfArgs a{};
-    a.din = s->at<const uint4>(s->L.din);
-    a.aux = s->at<const GateAux>(s->L.aux);
-    a.dhi = p.any_wide ? s->at<const uint4>(s->L.dhi) : nullptr;
-    a.dtt = p.max_k > GS_MAX_K_LUT64 ? s->at<const uint4>(s->L.dtt) : nullptr;
-    a.state = s->state();
-    a.stride = s->stride;
-    a.row_gate0 = p.row_gate0;
-    a.qcur = parity ? p.n_reg : 0;
-    a.qnext = parity ? 0 : p.n_reg;
-    a.lv_gate0 = s->at<const uint32_t>(s->L.lv_gate0);
-    a.lv_item0 = s->at<const uint32_t>(s->L.lv_item0);
-    a.nl = d.nl;
-    a.items_per_slab = d.lv_item0.back();
-    a.n_slabs = d.n_slabs;
-    a.interleave = d.interleave;
-    a.slab_vec = 32 * d.vpl;
-    a.gpw = d.gpw;
-    a.total_items = a.items_per_slab * d.n_slabs;
-    a.qhead = s->at<unsigned int>(s->L.dfctl);
-    a.done = a.qhead + 1;
-    if (!d.nl) return cudaSuccess;
-    cudaError_t e = cudaMemsetAsync(a.qhead, 0, s->L.dfctl_bytes, st);
-    if (e != cudaSuccess) return e;
-    return launch_dataflow(a, s->df_grid, st);
+    s->grid_stride_launches += gs_flag;
+    return e;
 }
 
 static cudaError_t tile_launch(const gs_sim* s, uint32_t ncycles, cudaStream_t st) {
@@ -371,7 +286,6 @@ static cudaError_t tile_launch(const gs_sim* s, uint32_t ncycles, cudaStream_t s
     a.n_levels = p.n_levels;
     a.desc_smem = (uint32_t)s->desc_smem;
     a.max_width = s->tile_max_width;
-    a.gslots = s->at<uint4>(s->L.t_gslots);
     a.po_slot = s->at<const uint32_t>(s->L.t_po);
     a.n_po = p.n_po;
     a.latch_src = s->at<const uint32_t>(s->L.t_lsrc);
@@ -399,49 +313,38 @@ static cudaError_t tile_launch(const gs_sim* s, uint32_t ncycles, cudaStream_t s
     return launch_tile(a, s->tw, s->tile_groups, s->tile_grid, st);
 }
 
-// evs (profiling): timing events around every level launch (or around the concurrent level
-// region); ext = the launches are being captured, record the events as graph nodes
-static cudaError_t cycle_launches(const gs_sim* s, uint32_t parity, cudaStream_t st,
+// evs (profiling): timing events around every level launch (one group), or around the
+// concurrent level region (lane groups); ext = the launches are being captured, record the
+// events as graph nodes
+static cudaError_t cycle_launches(gs_sim* s, uint32_t parity, cudaStream_t st,
                                   std::vector<cudaEvent_t>* evs = nullptr, bool ext = false) {
     const Program& p = *s->prog;
     cudaError_t e = launch_stim(s->ctl(), s->state(), s->stride, s->words, p.row_pi0, p.n_pi,
                                 s->opts.lane_offset / 64, s->pdl, st);
     if (e != cudaSuccess) return e;
-    if (s->opts.kernel == GS_KERNEL_DATAFLOW) {
-        if (evs) cudaEventRecord((*evs)[0], st);
-        e = dataflow_launch(s, parity, st);
-        if (evs) cudaEventRecord((*evs)[1], st);
-        if (e != cudaSuccess) return e;
-        return launch_end_cycle(end_args(s, parity), st);
-    }
-    if (s->concurrent) {
+    if (s->groups > 1) {
         // lane groups: one branch per group, forked after the stimulus kernel and joined
         // before the end-of-cycle kernel; the branches share nothing but the stimulus rows
         if (evs) cudaEventRecordWithFlags((*evs)[0], st, ext ? cudaEventRecordExternal : 0u);
         if ((e = cudaEventRecord(s->gev[0], st)) != cudaSuccess) return e;
-        const uint32_t per = s->slabs / s->branches;      // slabs of one group, run slab-major
-        for (uint32_t br = 0; br < s->branches; ++br) {
+        for (uint32_t br = 0; br < s->groups; ++br) {
             cudaStream_t b = br ? s->gstream[br - 1] : st;
             if (br && (e = cudaStreamWaitEvent(b, s->gev[0], 0)) != cudaSuccess) return e;
-            for (uint32_t j = 0; j < per; ++j)
-                for (uint32_t l = 0; l < p.n_levels; ++l)
-                    if ((e = level_launch(s, l, parity, b, br * per + j)) != cudaSuccess) return e;
+            for (uint32_t l = 0; l < p.n_levels; ++l)
+                if ((e = level_launch(s, l, parity, b, br)) != cudaSuccess) return e;
             if (br && (e = cudaEventRecord(s->gev[br], b)) != cudaSuccess) return e;
         }
-        for (uint32_t br = 1; br < s->branches; ++br)
+        for (uint32_t br = 1; br < s->groups; ++br)
             if ((e = cudaStreamWaitEvent(st, s->gev[br], 0)) != cudaSuccess) return e;
         if (evs) cudaEventRecordWithFlags((*evs)[1], st, ext ? cudaEventRecordExternal : 0u);
         return launch_end_cycle(end_args(s, parity), st);
     }
-    // slab-major order: every level on lanes [slab], then the next slab (lanes are
-    // independent; a slab's recent levels fit L2)
-    for (uint32_t sl = 0; sl < s->slabs; ++sl)
-        for (uint32_t l = 0; l < p.n_levels; ++l) {
-            if (evs) cudaEventRecord((*evs)[2 * ((size_t)sl * p.n_levels + l)], st);
-            e = level_launch(s, l, parity, st, sl);
-            if (e != cudaSuccess) return e;
-            if (evs) cudaEventRecord((*evs)[2 * ((size_t)sl * p.n_levels + l) + 1], st);
-        }
+    for (uint32_t l = 0; l < p.n_levels; ++l) {
+        if (evs) cudaEventRecord((*evs)[2 * (size_t)l], st);
+        e = level_launch(s, l, parity, st);
+        if (e != cudaSuccess) return e;
+        if (evs) cudaEventRecord((*evs)[2 * (size_t)l + 1], st);
+    }
     return launch_end_cycle(end_args(s, parity), st);
 }
 
@@ -467,7 +370,7 @@ static gs_status ensure_graph(gs_sim* s, uint32_t parity) {
 // algorithmic traffic (C5 shard: the level already fills the GPU for ~0.3 ms, and four
 // groups' 1 KB row segments lose more to short rows than the overlap gains).
 static uint32_t auto_lane_groups(const Program& p, const gs_sim_opts& o) {
-    if (o.kernel != GS_KERNEL_LUT || o.lane_slabs > 1 || o.lanes % 128) return 1;
+    if (o.kernel != GS_KERNEL_LUT || o.lanes % 128) return 1;
     const uint32_t vrow = (uint32_t)(o.lanes / 128);
     double bytes = 0;
     uint32_t nl = 0;
@@ -486,6 +389,21 @@ static void destroy_groups(gs_sim* s) {
         if (v) cudaEventDestroy(v);
     s->gstream.clear();
     s->gev.clear();
+}
+
+static void free_sim(gs_sim* s) {
+    if (!s) return;
+    destroy_groups(s);
+    for (auto& x : s->exec)
+        if (x) cudaGraphExecDestroy(x);
+    if (s->cap) cudaStreamDestroy(s->cap);
+    if (s->host_stage) cudaFree(s->host_stage);
+    if (s->copy) cudaStreamSynchronize(s->copy);
+    if (s->stream_buf) cudaFree(s->stream_buf);
+    for (auto& e : s->ev)
+        if (e) cudaEventDestroy(e);
+    if (s->copy) cudaStreamDestroy(s->copy);
+    delete s;
 }
 
 static gs_status check_sim(const gs_sim* s, const char* fn) {
@@ -507,12 +425,30 @@ static gs_status write_binding(gs_sim* s) {
     return GS_OK;
 }
 
-extern "C" {
+// flag bits of gs_sim_opts retired in 0.2.0 (L2 hints, bulk-copy gathers, global T slots)
+constexpr uint32_t GS_SIM_RETIRED_FLAGS = 2u | 4u | 64u | 128u | 256u;
+constexpr uint32_t GS_SIM_KNOWN_FLAGS = GS_SIM_NO_PDL | GS_SIM_NO_GRID_STRIDE | GS_SIM_TILE_DESC_GLOBAL |
+                                        GS_SIM_TILE_DESC_TMA;
 
-gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts, size_t* bytes) {
+static gs_status check_opts(const gs_sim_opts* o, const char* fn) {
+    if (o->lanes == 0 || o->lanes % 64) return fail(GS_ERR_ARG, std::string(fn) + ": lanes must be a positive multiple of 64");
+    if (o->lanes / 64 >= (1ull << 31)) return fail(GS_ERR_ARG, std::string(fn) + ": too many lanes");
+    if (o->lane_offset % 64) return fail(GS_ERR_ARG, std::string(fn) + ": lane_offset must be a multiple of 64");
+    if (o->kernel < GS_KERNEL_AUTO || o->kernel > GS_KERNEL_TILE || o->kernel == 4)
+        return fail(GS_ERR_ARG, std::string(fn) + ": bad kernel");
+    if (o->flags & GS_SIM_RETIRED_FLAGS)
+        return fail(GS_ERR_ARG, std::string(fn) + ": flag retired in 0.2.0 (L2 hints / bulk gathers / global T slots)");
+    if (o->flags & ~GS_SIM_KNOWN_FLAGS) return fail(GS_ERR_ARG, std::string(fn) + ": unknown flag");
+    if (o->n_trace_words && !o->trace_words) return fail(GS_ERR_ARG, std::string(fn) + ": trace_words is NULL");
+    return GS_OK;
+}
+
+// ======================================================================= ABI bodies
+// (each wrapped in GS_TRY by its extern "C" entry point below)
+
+static gs_status sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts, size_t* bytes) {
     if (!prog || !opts || !bytes) return fail(GS_ERR_ARG, "gs_sim_workspace_bytes: NULL argument");
-    if (opts->lanes == 0 || opts->lanes % 64) return fail(GS_ERR_ARG, "lanes must be a positive multiple of 64");
-    if (opts->lanes / 64 >= (1ull << 31)) return fail(GS_ERR_ARG, "too many lanes");
+    if (gs_status st = check_opts(opts, "gs_sim_workspace_bytes")) return st;
     const gs_sim_opts o = resolve_auto(*prog->p, *opts);
     Plans pl;
     if (gs_status st = make_plans(*prog->p, o, pl)) return st;
@@ -521,16 +457,14 @@ gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts
     return GS_OK;
 }
 
-gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void* dev_ws, size_t bytes, gs_sim** out) {
+static gs_status sim_reset(gs_sim* s);
+
+static gs_status sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void* dev_ws, size_t bytes, gs_sim** out) {
     NvtxRange nvtx("gs_sim_create");
     if (!prog || !opts_in || !out || !dev_ws) return fail(GS_ERR_ARG, "gs_sim_create: NULL argument");
+    if (gs_status st = check_opts(opts_in, "gs_sim_create")) return st;
     const gs_sim_opts resolved = resolve_auto(*prog->p, *opts_in);
     const gs_sim_opts* opts = &resolved;
-
-    if (opts->lanes == 0 || opts->lanes % 64) return fail(GS_ERR_ARG, "gs_sim_create: lanes must be a positive multiple of 64");
-    if (opts->lane_offset % 64) return fail(GS_ERR_ARG, "gs_sim_create: lane_offset must be a multiple of 64");
-    if (opts->kernel < GS_KERNEL_AUTO || opts->kernel > GS_KERNEL_TILE) return fail(GS_ERR_ARG, "gs_sim_create: bad kernel");
-    if (opts->n_trace_words && !opts->trace_words) return fail(GS_ERR_ARG, "gs_sim_create: trace_words is NULL");
     if ((reinterpret_cast<uintptr_t>(dev_ws) & 255) != 0) return fail(GS_ERR_ARG, "gs_sim_create: workspace must be 256-byte aligned");
     const Program& p = *prog->p;
     const uint32_t words = (uint32_t)(opts->lanes / 64);
@@ -538,11 +472,22 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
         if (opts->trace_words[i] >= words) return fail(GS_ERR_ARG, "gs_sim_create: trace word out of range");
     Plans pls;
     if (gs_status st = make_plans(p, *opts, pls)) return st;
-    const DfPlan& plan = pls.df;
     Layout L = make_layout(p, *opts, pls);
     if (bytes < L.total) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_create: workspace smaller than gs_sim_workspace_bytes");
+    uint32_t groups = opts->lane_groups;
+    if (groups == 0) groups = auto_lane_groups(p, *opts);
+    if (groups > 1) {
+        const uint32_t vrow = words / 2;
+        if (opts->kernel != GS_KERNEL_LUT || words % 2 || vrow % groups || (vrow / groups) % 32)
+            return fail(GS_ERR_ARG, "gs_sim_create: lane_groups needs kernel A, (lanes/128) % groups == 0 "
+                                    "and a multiple of 4096 lanes per group");
+    }
     CU(cudaSetDevice(opts->device));
     gs_sim* s = new gs_sim();
+    struct Guard {                        // frees the half-built sim on every early return
+        gs_sim*& s;
+        ~Guard() { free_sim(s); }
+    } guard{s};
     s->prog = &p;
     s->opts = *opts;
     s->trace_words.assign(opts->trace_words, opts->trace_words + opts->n_trace_words);
@@ -552,12 +497,12 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
     s->stream = static_cast<cudaStream_t>(opts->stream);
     s->words = words;
     s->stride = (uint64_t)words * 8;
-    s->df = plan;
     s->tile = pls.tile;
     s->tw = pls.tw;
     s->desc_smem = pls.desc_smem;
     s->tile_max_width = pls.max_width;
     s->pdl = (opts->flags & GS_SIM_NO_PDL) ? 0u : 1u;
+    s->groups = groups;
     {
         int sms = 148;
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, opts->device);
@@ -565,93 +510,33 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
         s->resident_blocks = level_lut_resident_blocks(opts->device);
         s->sms = (uint32_t)sms;
     }
-    {
-        // bulk-copy gathers: opt-in (measured slower than the register gathers)
-        s->bulk = (opts->flags & GS_SIM_LUT_BULK) && !(opts->flags & GS_SIM_LUT_NO_BULK);
-        s->lv_bulk.assign(p.n_levels, 1);
-        for (uint32_t l = 0; l < p.n_levels; ++l)
-            for (uint32_t g = p.level_off[l]; g < p.level_off[l + 1]; ++g) {
-                const uint32_t k = p.aux[g].k & 0xFFu;
-                if (k < 1 || k > 4) s->lv_bulk[l] = 0;
-            }
-    }
-    s->slabs = (opts->lane_slabs && s->opts.kernel != GS_KERNEL_DATAFLOW) ? opts->lane_slabs : 1;
-    uint32_t groups = opts->lane_groups;
-    if (groups == 0) groups = auto_lane_groups(p, *opts);
-    if (groups > 1) {
-        const uint32_t vrow = words / 2, G = groups;
-        const uint32_t S = std::max<uint32_t>(1, opts->lane_slabs);     // slabs per group
-        if (s->opts.kernel != GS_KERNEL_LUT || words % 2 || vrow % (G * S) || (vrow / (G * S)) % 32) {
-            delete s;
-            return fail(GS_ERR_ARG, "gs_sim_create: lane_groups needs kernel A, (lanes/128) % (groups x lane_slabs) "
-                                    "== 0 and a multiple of 4096 lanes per slab");
-        }
-        s->slabs = G * S;
-        s->branches = G;
-        s->concurrent = true;
-    }
-    if (s->slabs > 1) {
-        const uint32_t vrow = words / 2;
-        if (s->opts.kernel != GS_KERNEL_LUT || words % 2 || vrow % s->slabs || (vrow / s->slabs) % 32) {
-
-            delete s;
-            return fail(GS_ERR_ARG, "gs_sim_create: lane_slabs needs kernel A and (lanes/128) % slabs == 0 "
-                                    "with a multiple of 4096 lanes per slab");
-        }
-    }
-    auto cleanup = [&](gs_status st) {
-        if (s->cap) cudaStreamDestroy(s->cap);
-        delete s;
-        return st;
-    };
     cudaError_t e = cudaSuccess;
-    if (s->opts.kernel == GS_KERNEL_DATAFLOW) {
-        e = dataflow_grid(32 * plan.vpl, opts->device, &s->df_grid);
-        if (e != cudaSuccess) {
-            delete s;
-            return fail(GS_ERR_CUDA, std::string("dataflow occupancy: ") + cudaGetErrorString(e));
-        }
-    }
     if (s->opts.kernel == GS_KERNEL_TILE) {
         uint32_t per = 0;
-        int sms = 148;
         s->tile_groups = pls.ng;
         e = tile_setup(s->tw, s->tile_groups, s->tile.n_slots, p.n_eval, p.n_levels, s->desc_smem,
                        s->tile_max_width, p.n_reg > 0, &per);
-        if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, opts->device);
-        if (e != cudaSuccess || per == 0) {
-            delete s;
+        if (e != cudaSuccess || per == 0)
             return fail(e != cudaSuccess ? GS_ERR_CUDA : GS_ERR_ARG,
                         std::string("TILE: kernel setup: ") + (e != cudaSuccess ? cudaGetErrorString(e) : "0 CTAs fit an SM"));
-        }
         const uint32_t tiles = (uint32_t)(opts->lanes / (32ull * s->tw));
-        s->tile_grid = std::min<uint32_t>((tiles + s->tile_groups - 1) / s->tile_groups, per * (uint32_t)sms);
+        s->tile_grid = std::min<uint32_t>((tiles + s->tile_groups - 1) / s->tile_groups, per * s->sms);
     }
-    e = cudaStreamCreateWithFlags(&s->cap, cudaStreamNonBlocking);
-    if (e != cudaSuccess) return cleanup(fail(GS_ERR_CUDA, std::string("cudaStreamCreate: ") + cudaGetErrorString(e)));
-    if (s->concurrent) {
-        s->gstream.assign(s->branches - 1, nullptr);
-        s->gev.assign(s->branches, nullptr);
-        for (auto& b : s->gstream)
-            if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&b, cudaStreamNonBlocking);
-        for (auto& v : s->gev)
-            if (e == cudaSuccess) e = cudaEventCreateWithFlags(&v, cudaEventDisableTiming);
-        if (e != cudaSuccess) {
-            destroy_groups(s);
-            return cleanup(fail(GS_ERR_CUDA, std::string("lane groups: ") + cudaGetErrorString(e)));
-        }
+    CU(cudaStreamCreateWithFlags(&s->cap, cudaStreamNonBlocking));
+    if (s->groups > 1) {
+        s->gstream.assign(s->groups - 1, nullptr);
+        s->gev.assign(s->groups, nullptr);
+        for (auto& b : s->gstream) CU(cudaStreamCreateWithFlags(&b, cudaStreamNonBlocking));
+        for (auto& v : s->gev) CU(cudaEventCreateWithFlags(&v, cudaEventDisableTiming));
     }
     // upload the program (descriptors are device-resident for the sim's lifetime)
     struct Up { size_t off; const void* src; size_t n; };
     std::vector<int32_t> slot(words, -1);
     for (uint32_t i = 0; i < opts->n_trace_words; ++i) slot[opts->trace_words[i]] = (int32_t)i;
     const bool poly = s->opts.kernel == GS_KERNEL_POLY || s->opts.kernel == GS_KERNEL_AB;
-    // device aux: k | hot << 8 (kernels mask k with 0xFF)
-    std::vector<GateAux> aux_dev = p.aux;
-    for (size_t g = 0; g < aux_dev.size(); ++g) aux_dev[g].k |= (uint32_t)p.hot[g] << 8;
     std::vector<Up> ups = {
         {L.din, p.in_lo.data(), p.in_lo.size() * 4},
-        {L.aux, aux_dev.data(), aux_dev.size() * sizeof(GateAux)},
+        {L.aux, p.aux.data(), p.aux.size() * sizeof(GateAux)},
         {L.dhi, p.in_hi.data(), p.any_wide ? p.in_hi.size() * 4 : 0},
         {L.dtt, p.tt_full.data(), p.max_k > GS_MAX_K_LUT64 ? p.tt_full.size() * 8 : 0},
         {L.term_off, p.term_off.data(), poly ? p.term_off.size() * 4 : 0},
@@ -661,8 +546,6 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
         {L.latch_dst, p.latch_dst.data(), p.latch_dst.size() * 4},
         {L.reg_init, p.reg_init.data(), p.reg_init.size()},
         {L.trace_slot, slot.data(), slot.size() * 4},
-        {L.lv_gate0, plan.lv_gate0.data(), plan.lv_gate0.size() * 4},
-        {L.lv_item0, plan.lv_item0.data(), plan.lv_item0.size() * 4},
         {L.t_desc, s->tile.desc.data(), s->tile.desc.size() * sizeof(TileDesc)},
         {L.t_desc_hi, s->tile.desc_hi.data(), s->tile.desc_hi.size() * 4},
         {L.t_po, s->tile.po_slot.data(), s->tile.po_slot.size() * 4},
@@ -672,45 +555,23 @@ gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts_in, void
         {L.t_wbslot, s->tile.wb_slot.data(), s->tile.wb_slot.size() * 4},
         {L.t_lvl, p.level_off.data(), s->tw ? p.level_off.size() * 4 : 0},
     };
-    for (const Up& u : ups) {
-        if (!u.n) continue;
-        e = cudaMemcpyAsync(s->ws + u.off, u.src, u.n, cudaMemcpyHostToDevice, s->stream);
-        if (e != cudaSuccess) return cleanup(fail(GS_ERR_CUDA, std::string("upload: ") + cudaGetErrorString(e)));
-    }
-    e = cudaStreamSynchronize(s->stream);   // host vectors above are temporaries
-    if (e != cudaSuccess) return cleanup(fail(GS_ERR_CUDA, std::string("upload sync: ") + cudaGetErrorString(e)));
-    gs_status st = gs_sim_reset(s);
-    if (st != GS_OK) return cleanup(st);
+    for (const Up& u : ups)
+        if (u.n) CU(cudaMemcpyAsync(s->ws + u.off, u.src, u.n, cudaMemcpyHostToDevice, s->stream));
+    CU(cudaStreamSynchronize(s->stream));   // host vectors above are temporaries
+    if (gs_status st = sim_reset(s)) return st;
     *out = s;
+    s = nullptr;                            // ownership passes to the caller
     clear_error();
     return GS_OK;
 }
 
-gs_status gs_sim_destroy(gs_sim* s) {
-    if (!s) return GS_OK;
-    cudaSetDevice(s->opts.device);
-    cudaStreamSynchronize(s->stream);
-    destroy_groups(s);
-    for (auto& x : s->exec)
-        if (x) cudaGraphExecDestroy(x);
-    if (s->cap) cudaStreamDestroy(s->cap);
-    if (s->host_stage) cudaFree(s->host_stage);
-    if (s->copy) cudaStreamSynchronize(s->copy);
-    if (s->stream_buf) cudaFree(s->stream_buf);
-    for (auto& e : s->ev)
-        if (e) cudaEventDestroy(e);
-    if (s->copy) cudaStreamDestroy(s->copy);
-    delete s;
-    return GS_OK;
-}
-
-gs_status gs_sim_reset(gs_sim* s) {
+static gs_status sim_reset(gs_sim* s) {
     if (gs_status st = check_sim(s, "gs_sim_reset")) return st;
     const Program& p = *s->prog;
     CU(cudaSetDevice(s->opts.device));
     CU(cudaMemsetAsync(s->ws + s->L.ctl, 0, sizeof(Ctl), s->stream));
     CU(cudaMemsetAsync(s->ws + s->L.misr, 0, (size_t)2 * 64 * s->words * 8, s->stream));
-    if (s->L.lane_sigs != s->L.scratch) CU(cudaMemsetAsync(s->ws + s->L.lane_sigs, 0, (size_t)s->opts.lanes * 8, s->stream));
+    CU(cudaMemsetAsync(s->ws + s->L.lane_sigs, 0, (size_t)s->opts.lanes * 8, s->stream));
     size_t tbytes = (size_t)s->opts.trace_cycles * p.n_po * s->opts.n_trace_words * 8;
     if (tbytes) CU(cudaMemsetAsync(s->ws + s->L.trace, 0, tbytes, s->stream));
     CU(launch_fill_rows(s->state(), s->stride, s->words, 0, 1, nullptr, 0, s->stream));          // const0
@@ -725,7 +586,7 @@ gs_status gs_sim_reset(gs_sim* s) {
     return GS_OK;
 }
 
-gs_status gs_sim_set_lane_offset(gs_sim* s, uint64_t lane_offset) {
+static gs_status sim_set_lane_offset(gs_sim* s, uint64_t lane_offset) {
     if (gs_status st = check_sim(s, "gs_sim_set_lane_offset")) return st;
     if (lane_offset % 64) return fail(GS_ERR_ARG, "gs_sim_set_lane_offset: lane_offset must be a multiple of 64");
     CU(cudaSetDevice(s->opts.device));
@@ -739,10 +600,10 @@ gs_status gs_sim_set_lane_offset(gs_sim* s, uint64_t lane_offset) {
             }
         s->opts.lane_offset = lane_offset;
     }
-    return gs_sim_reset(s);
+    return sim_reset(s);
 }
 
-gs_status gs_sim_bind_stimulus_generated(gs_sim* s, uint64_t seed) {
+static gs_status sim_bind_generated(gs_sim* s, uint64_t seed) {
     if (gs_status st = check_sim(s, "gs_sim_bind_stimulus_generated")) return st;
     CU(cudaSetDevice(s->opts.device));
     s->bound = 1;
@@ -755,7 +616,7 @@ gs_status gs_sim_bind_stimulus_generated(gs_sim* s, uint64_t seed) {
     return GS_OK;
 }
 
-gs_status gs_sim_bind_stimulus_device(gs_sim* s, const uint64_t* dev_words, uint32_t cycles) {
+static gs_status sim_bind_device(gs_sim* s, const uint64_t* dev_words, uint32_t cycles) {
     if (gs_status st = check_sim(s, "gs_sim_bind_stimulus_device")) return st;
     if (!dev_words && cycles) return fail(GS_ERR_ARG, "gs_sim_bind_stimulus_device: NULL words");
     CU(cudaSetDevice(s->opts.device));
@@ -769,7 +630,7 @@ gs_status gs_sim_bind_stimulus_device(gs_sim* s, const uint64_t* dev_words, uint
     return GS_OK;
 }
 
-gs_status gs_sim_bind_stimulus_host(gs_sim* s, const uint64_t* words, uint32_t cycles) {
+static gs_status sim_bind_host(gs_sim* s, const uint64_t* words, uint32_t cycles) {
     if (gs_status st = check_sim(s, "gs_sim_bind_stimulus_host")) return st;
     if (!words && cycles) return fail(GS_ERR_ARG, "gs_sim_bind_stimulus_host: NULL words");
     CU(cudaSetDevice(s->opts.device));
@@ -793,7 +654,7 @@ gs_status gs_sim_bind_stimulus_host(gs_sim* s, const uint64_t* words, uint32_t c
     return GS_OK;
 }
 
-gs_status gs_sim_step(gs_sim* s, uint32_t n) {
+static gs_status sim_step(gs_sim* s, uint32_t n) {
     NvtxRange nvtx("gs_sim_step");
     if (gs_status st = check_sim(s, "gs_sim_step")) return st;
     if (!s->bound) return fail(GS_ERR_STATE, "gs_sim_step: no stimulus bound");
@@ -820,8 +681,8 @@ gs_status gs_sim_step(gs_sim* s, uint32_t n) {
     return GS_OK;
 }
 
-gs_status gs_sim_run_streamed(gs_sim* s, const uint64_t* host_stim, uint64_t* host_out, uint32_t ncycles,
-                              uint32_t chunk) {
+static gs_status sim_run_streamed(gs_sim* s, const uint64_t* host_stim, uint64_t* host_out, uint32_t ncycles,
+                                  uint32_t chunk) {
     NvtxRange nvtx("gs_sim_run_streamed");
     if (gs_status st = check_sim(s, "gs_sim_run_streamed")) return st;
     if (!host_stim && ncycles) return fail(GS_ERR_ARG, "gs_sim_run_streamed: NULL host_stim");
@@ -846,6 +707,8 @@ gs_status gs_sim_run_streamed(gs_sim* s, const uint64_t* host_stim, uint64_t* ho
         CU(cudaStreamCreateWithFlags(&s->copy, cudaStreamNonBlocking));
         for (auto& e : s->ev) CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     }
+    const int prev_bound = s->bound;
+    const uint64_t prev_seed = s->bound_seed;
     uint8_t* buf = static_cast<uint8_t*>(s->stream_buf);
     auto in_slot = [&](uint32_t i) { return buf + (i & 1) * in_b2; };
     auto out_slot = [&](uint32_t i) { return buf + 2 * in_b2 + (i & 1) * out_b2; };
@@ -881,7 +744,7 @@ gs_status gs_sim_run_streamed(gs_sim* s, const uint64_t* host_stim, uint64_t* ho
         s->bound_ptr = reinterpret_cast<uint64_t>(in_slot(i));
         s->bound_base = c0;
         s->bound_cycles = cc;
-        if (gs_status st = gs_sim_step(s, cc)) return st;
+        if (gs_status st = sim_step(s, cc)) return st;
         CU(cudaEventRecord(ev_comp[i & 1], s->stream));
         if (host_out) {
             CU(cudaStreamWaitEvent(s->copy, ev_comp[i & 1], 0));
@@ -890,36 +753,26 @@ gs_status gs_sim_run_streamed(gs_sim* s, const uint64_t* host_stim, uint64_t* ho
             CU(cudaEventRecord(ev_out[i & 1], s->copy));
         }
     }
-    // detach the sink; the sim's stream completes only after the last output copy
-    CU(launch_set_binding(s->ctl(), s->bound_ptr, s->bound_base, 1u, 0ull, 0ull, 0ull, s->stream));
+    // detach the sink and the staging slot: a generated binding from before the call is
+    // restored (the seed in Ctl is untouched by the streamed run), any other is cleared;
+    // the sim's stream completes only after the last output copy
+    if (prev_bound == 1) {
+        CU(launch_set_binding(s->ctl(), 0ull, 0ull, 0u, 0ull, 0ull, 0ull, s->stream));
+        s->bound = 1;
+        s->bound_seed = prev_seed;
+        s->bound_ptr = 0;
+        s->bound_cycles = 0;
+    } else {
+        CU(launch_set_binding(s->ctl(), s->bound_ptr, s->bound_base, 1u, 0ull, 0ull, 0ull, s->stream));
+        s->bound = 0;
+    }
     CU(cudaEventRecord(ev_in[0], s->copy));
     CU(cudaStreamWaitEvent(s->stream, ev_in[0], 0));
     clear_error();
     return GS_OK;
 }
 
-gs_status gs_sim_sync(gs_sim* s) {
-    if (gs_status st = check_sim(s, "gs_sim_sync")) return st;
-    CU(cudaSetDevice(s->opts.device));
-    CU(cudaStreamSynchronize(s->stream));
-    clear_error();
-    return GS_OK;
-}
-
-gs_status gs_sim_get_cycle(const gs_sim* s, uint64_t* cycle) {
-    if (!s || !cycle) return fail(GS_ERR_ARG, "gs_sim_get_cycle: NULL argument");
-    *cycle = s->cycle;
-    return GS_OK;
-}
-
-gs_status gs_sim_get_config(const gs_sim* s, int* kernel, uint32_t* lane_groups) {
-    if (!s || !kernel || !lane_groups) return fail(GS_ERR_ARG, "gs_sim_get_config: NULL argument");
-    *kernel = s->opts.kernel;
-    *lane_groups = s->concurrent ? s->branches : 1u;
-    return GS_OK;
-}
-
-gs_status gs_sim_read_outputs(gs_sim* s, uint64_t* host, size_t nwords) {
+static gs_status sim_read_outputs(gs_sim* s, uint64_t* host, size_t nwords) {
     if (gs_status st = check_sim(s, "gs_sim_read_outputs")) return st;
     const Program& p = *s->prog;
     const size_t need = (size_t)p.n_po * s->words;
@@ -936,37 +789,24 @@ gs_status gs_sim_read_outputs(gs_sim* s, uint64_t* host, size_t nwords) {
     return GS_OK;
 }
 
-gs_status gs_sim_read_registers(gs_sim* s, uint64_t* host, size_t nwords) {
-    if (gs_status st = check_sim(s, "gs_sim_read_registers")) return st;
+static gs_status sim_rw_registers(gs_sim* s, uint64_t* host_out, const uint64_t* host_in, size_t nwords) {
+    const char* fn = host_out ? "gs_sim_read_registers" : "gs_sim_write_registers";
+    if (gs_status st = check_sim(s, fn)) return st;
     const Program& p = *s->prog;
     const size_t need = (size_t)p.n_reg * s->words;
-    if (!host && need) return fail(GS_ERR_ARG, "gs_sim_read_registers: NULL buffer");
-    if (nwords < need) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_read_registers: need n_reg * lanes/64 words");
+    if (!host_out && !host_in && need) return fail(GS_ERR_ARG, std::string(fn) + ": NULL buffer");
+    if (nwords < need) return fail(GS_ERR_BUFFER_TOO_SMALL, std::string(fn) + ": need n_reg * lanes/64 words");
     CU(cudaSetDevice(s->opts.device));
     const uint32_t bank = (uint32_t)(s->cycle & 1);     // the bank the next cycle reads = Q(cycle)
-    const uint8_t* src = s->state() + (uint64_t)(p.row_q0 + bank * p.n_reg) * s->stride;
-    if (need) CU(cudaMemcpyAsync(host, src, need * 8, cudaMemcpyDeviceToHost, s->stream));
+    uint8_t* q = s->state() + (uint64_t)(p.row_q0 + bank * p.n_reg) * s->stride;
+    if (need && host_out) CU(cudaMemcpyAsync(host_out, q, need * 8, cudaMemcpyDeviceToHost, s->stream));
+    if (need && host_in) CU(cudaMemcpyAsync(q, host_in, need * 8, cudaMemcpyHostToDevice, s->stream));
     CU(cudaStreamSynchronize(s->stream));
     clear_error();
     return GS_OK;
 }
 
-gs_status gs_sim_write_registers(gs_sim* s, const uint64_t* host, size_t nwords) {
-    if (gs_status st = check_sim(s, "gs_sim_write_registers")) return st;
-    const Program& p = *s->prog;
-    const size_t need = (size_t)p.n_reg * s->words;
-    if (!host && need) return fail(GS_ERR_ARG, "gs_sim_write_registers: NULL buffer");
-    if (nwords < need) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_write_registers: need n_reg * lanes/64 words");
-    CU(cudaSetDevice(s->opts.device));
-    const uint32_t bank = (uint32_t)(s->cycle & 1);
-    uint8_t* dst = s->state() + (uint64_t)(p.row_q0 + bank * p.n_reg) * s->stride;
-    if (need) CU(cudaMemcpyAsync(dst, host, need * 8, cudaMemcpyHostToDevice, s->stream));
-    CU(cudaStreamSynchronize(s->stream));
-    clear_error();
-    return GS_OK;
-}
-
-gs_status gs_sim_read_trace(gs_sim* s, uint64_t* host, size_t nwords, uint32_t* cycles_recorded) {
+static gs_status sim_read_trace(gs_sim* s, uint64_t* host, size_t nwords, uint32_t* cycles_recorded) {
     if (gs_status st = check_sim(s, "gs_sim_read_trace")) return st;
     const Program& p = *s->prog;
     const uint64_t rec = s->cycle < s->opts.trace_cycles ? s->cycle : s->opts.trace_cycles;
@@ -989,7 +829,7 @@ static gs_status compute_lane_sigs(gs_sim* s) {
     return GS_OK;
 }
 
-gs_status gs_sim_read_lane_signatures(gs_sim* s, uint64_t* host, size_t nlanes) {
+static gs_status sim_read_lane_signatures(gs_sim* s, uint64_t* host, size_t nlanes) {
     if (gs_status st = check_sim(s, "gs_sim_read_lane_signatures")) return st;
     if (!host) return fail(GS_ERR_ARG, "gs_sim_read_lane_signatures: NULL buffer");
     if (nlanes < s->opts.lanes) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_read_lane_signatures: need `lanes` entries");
@@ -1001,7 +841,7 @@ gs_status gs_sim_read_lane_signatures(gs_sim* s, uint64_t* host, size_t nlanes) 
     return GS_OK;
 }
 
-gs_status gs_sim_read_signature(gs_sim* s, gs_signature* out) {
+static gs_status sim_read_signature(gs_sim* s, gs_signature* out) {
     if (gs_status st = check_sim(s, "gs_sim_read_signature")) return st;
     if (!out) return fail(GS_ERR_ARG, "gs_sim_read_signature: NULL out");
     CU(cudaSetDevice(s->opts.device));
@@ -1018,20 +858,17 @@ gs_status gs_sim_read_signature(gs_sim* s, gs_signature* out) {
     return GS_OK;
 }
 
-gs_status gs_sim_launches_per_cycle(const gs_sim* s, uint64_t* launches) {
-    if (!s || !launches) return fail(GS_ERR_ARG, "gs_sim_launches_per_cycle: NULL argument");
+static uint64_t launches_per_cycle(const gs_sim* s) {
     const Program& p = *s->prog;
+    if (s->opts.kernel == GS_KERNEL_TILE) return 1;      // per gs_sim_step call, not per cycle
     uint64_t lv = 0;
     for (uint32_t l = 0; l < p.n_levels; ++l)
         if (p.level_off[l + 1] > p.level_off[l]) lv++;
     const uint64_t per_level = s->opts.kernel == GS_KERNEL_AB ? 2 : 1;
-    if (s->opts.kernel == GS_KERNEL_TILE) *launches = 1;      // per gs_sim_step call, not per cycle
-    else if (s->opts.kernel == GS_KERNEL_DATAFLOW) lv = s->df.nl ? 1 : 0, *launches = (p.n_pi ? 1 : 0) + lv + 1;
-    else *launches = (p.n_pi ? 1 : 0) + lv * per_level * s->slabs + 1;
-    return GS_OK;
+    return (p.n_pi ? 1 : 0) + lv * per_level * s->groups + 1;
 }
 
-gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
+static gs_status sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
     if (gs_status st = check_sim(s, "gs_sim_profile_step")) return st;
     if (!out) return fail(GS_ERR_ARG, "gs_sim_profile_step: NULL out");
     if (!s->bound) return fail(GS_ERR_STATE, "gs_sim_profile_step: no stimulus bound");
@@ -1039,53 +876,66 @@ gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
         return fail(GS_ERR_STATE, "gs_sim_profile_step: stepping past the bound stimulus cycles");
     const Program& p = *s->prog;
     CU(cudaSetDevice(s->opts.device));
+    // algorithmic bytes of a level: every gate reads k input rows, writes its output row,
+    // plus the fused latch store (DESIGN.md §6 "algorithmic bytes")
+    std::vector<double> lb(p.n_levels, 0.0);
+    double all_bytes = 0;
+    for (uint32_t l = 0; l < p.n_levels; ++l) {
+        for (uint32_t g = p.level_off[l]; g < p.level_off[l + 1]; ++g)
+            lb[l] += (double)(p.aux[g].k + 1 + (p.aux[g].qdst != NONE32 ? 1 : 0)) * (double)s->stride;
+        all_bytes += lb[l];
+    }
+    std::memset(out, 0, sizeof(*out));
     if (s->opts.kernel == GS_KERNEL_TILE) {
         // one launch runs all n cycles; "level" bytes are the same algorithmic gather model
-        cudaEvent_t a0, a1;
-        CU(cudaEventCreate(&a0));
-        CU(cudaEventCreate(&a1));
-        cudaEventRecord(a0, s->stream);
-        cudaError_t e = tile_launch(s, n, s->stream);
-        cudaEventRecord(a1, s->stream);
+        cudaEvent_t a0 = nullptr, a1 = nullptr;
+        cudaError_t e = cudaEventCreate(&a0);
+        if (e == cudaSuccess) e = cudaEventCreate(&a1);
+        if (e == cudaSuccess) e = cudaEventRecord(a0, s->stream);
+        if (e == cudaSuccess) e = tile_launch(s, n, s->stream);
+        if (e == cudaSuccess) e = cudaEventRecord(a1, s->stream);
         if (e == cudaSuccess) e = cudaEventSynchronize(a1);
         float ms = 0;
         if (e == cudaSuccess) cudaEventElapsedTime(&ms, a0, a1);
-        cudaEventDestroy(a0);
-        cudaEventDestroy(a1);
+        if (a0) cudaEventDestroy(a0);
+        if (a1) cudaEventDestroy(a1);
         if (e != cudaSuccess) return fail(GS_ERR_CUDA, cudaGetErrorString(e));
         s->cycle += n;
-        double bytes = 0;
-        for (uint32_t g = 0; g < p.n_eval; ++g)
-            bytes += (double)(p.aux[g].k + 1 + (p.aux[g].qdst != NONE32 ? 1 : 0)) * (double)s->stride;
         out->level_ms = ms;
         out->total_ms = ms;
         out->level_launches = n ? 1 : 0;
         out->total_launches = n ? 1 : 0;
-        out->level_bytes = bytes * n;
+        out->level_bytes = all_bytes * n;
         clear_error();
         return GS_OK;
     }
-    std::vector<cudaEvent_t> evs(std::max<size_t>(2, 2 * (size_t)p.n_levels * s->slabs));
-    const bool df = s->opts.kernel == GS_KERNEL_DATAFLOW;
-    cudaEvent_t e0, e1;
+    std::vector<cudaEvent_t> evs(std::max<size_t>(2, 2 * (size_t)p.n_levels), nullptr);
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    cudaGraphExec_t px[2] = {nullptr, nullptr};
+    struct Cleanup {
+        std::vector<cudaEvent_t>& evs;
+        cudaEvent_t &e0, &e1;
+        cudaGraphExec_t* px;
+        ~Cleanup() {
+            for (auto& e : evs)
+                if (e) cudaEventDestroy(e);
+            if (e0) cudaEventDestroy(e0);
+            if (e1) cudaEventDestroy(e1);
+            for (int i = 0; i < 2; ++i)
+                if (px[i]) cudaGraphExecDestroy(px[i]);
+        }
+    } cleanup{evs, e0, e1, px};
     for (auto& e : evs) CU(cudaEventCreate(&e));
     CU(cudaEventCreate(&e0));
     CU(cudaEventCreate(&e1));
     double level_ms = 0, total_ms = 0, level_bytes = 0;
-    uint64_t lvl_launches = 0, launches = 0, per = 0;
-    gs_sim_launches_per_cycle(s, &per);
-    // algorithmic bytes of one level launch: every gate reads k input rows, writes its
-    // output row, plus the fused latch store
-    std::vector<double> lb(p.n_levels, 0.0);
-    for (uint32_t l = 0; l < p.n_levels; ++l)
-        for (uint32_t g = p.level_off[l]; g < p.level_off[l + 1]; ++g)
-            lb[l] += (double)(p.aux[g].k + 1 + (p.aux[g].qdst != NONE32 ? 1 : 0)) * (double)s->stride;
-    gs_status rc = GS_OK;
+    uint64_t lvl_launches = 0, launches = 0;
+    const uint64_t per = launches_per_cycle(s);
+    const uint64_t gs0 = s->grid_stride_launches;
     // concurrent lane groups: the branches only overlap as they do in gs_sim_step when the
     // cycle is replayed as its graph, so profile a graph of the cycle with timing-event
     // nodes at the fork and the join (eager launches of G x levels kernels would measure
     // the host's launch rate instead)
-    cudaGraphExec_t px[2] = {nullptr, nullptr};
     auto prof_graph = [&](uint32_t parity) -> cudaError_t {
         if (px[parity]) return cudaSuccess;
         cudaGraph_t g = nullptr;
@@ -1098,58 +948,152 @@ gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
         if (g) cudaGraphDestroy(g);
         return e;
     };
-    for (uint32_t i = 0; i < n && rc == GS_OK; ++i) {
+    for (uint32_t i = 0; i < n; ++i) {
         const uint32_t parity = (uint32_t)(s->cycle & 1);
-        cudaError_t e = cudaSuccess;
-        if (s->concurrent) {
-            e = prof_graph(parity);
-            if (e != cudaSuccess) { rc = fail(GS_ERR_CUDA, cudaGetErrorString(e)); break; }
-            cudaEventRecord(e0, s->stream);
-            e = cudaGraphLaunch(px[parity], s->stream);
+        if (s->groups > 1) {
+            CU(prof_graph(parity));
+            CU(cudaEventRecord(e0, s->stream));
+            CU(cudaGraphLaunch(px[parity], s->stream));
         } else {
-            cudaEventRecord(e0, s->stream);
-            e = cycle_launches(s, parity, s->stream, &evs);
+            CU(cudaEventRecord(e0, s->stream));
+            CU(cycle_launches(s, parity, s->stream, &evs));
         }
-        cudaEventRecord(e1, s->stream);
-        if (e != cudaSuccess) { rc = fail(GS_ERR_CUDA, cudaGetErrorString(e)); break; }
+        CU(cudaEventRecord(e1, s->stream));
         s->cycle++;
-        e = cudaEventSynchronize(e1);
-        if (e != cudaSuccess) { rc = fail(GS_ERR_CUDA, cudaGetErrorString(e)); break; }
+        CU(cudaEventSynchronize(e1));
         float ms = 0;
         cudaEventElapsedTime(&ms, e0, e1);
         total_ms += ms;
-        if (df || s->concurrent) {     // one persistent launch / concurrent branches cover every level
+        if (s->groups > 1) {           // concurrent branches cover every level
             cudaEventElapsedTime(&ms, evs[0], evs[1]);
             level_ms += ms;
-            for (uint32_t l = 0; l < p.n_levels; ++l) level_bytes += lb[l];
-            if (df) lvl_launches += s->df.nl ? 1 : 0;
-            else
-                for (uint32_t l = 0; l < p.n_levels; ++l) lvl_launches += p.level_off[l + 1] > p.level_off[l] ? s->slabs : 0;
-        } else
-        for (uint32_t sl = 0; sl < s->slabs; ++sl)
+            level_bytes += all_bytes;
+            for (uint32_t l = 0; l < p.n_levels; ++l) lvl_launches += p.level_off[l + 1] > p.level_off[l] ? s->groups : 0;
+        } else {
             for (uint32_t l = 0; l < p.n_levels; ++l) {
                 if (p.level_off[l + 1] == p.level_off[l]) continue;
-                const size_t ix = (size_t)sl * p.n_levels + l;
-                cudaEventElapsedTime(&ms, evs[2 * ix], evs[2 * ix + 1]);
+                cudaEventElapsedTime(&ms, evs[2 * (size_t)l], evs[2 * (size_t)l + 1]);
                 level_ms += ms;
-                level_bytes += lb[l] / s->slabs;
+                level_bytes += lb[l];
                 lvl_launches++;
             }
+        }
         launches += per;
     }
-    for (auto& x : px)
-        if (x) cudaGraphExecDestroy(x);
-    for (auto& e : evs) cudaEventDestroy(e);
-    cudaEventDestroy(e0);
-    cudaEventDestroy(e1);
-    if (rc != GS_OK) return rc;
     out->level_ms = level_ms;
     out->total_ms = total_ms;
     out->level_launches = lvl_launches;
     out->total_launches = launches;
     out->level_bytes = level_bytes;
+    // launch decisions of the host side: with lane groups they were taken once per captured
+    // graph (per parity), eagerly once per level launch otherwise
+    out->grid_stride_launches = s->grid_stride_launches - gs0;
     clear_error();
     return GS_OK;
 }
+
+extern "C" {
+
+gs_status gs_sim_workspace_bytes(const gs_program* prog, const gs_sim_opts* opts, size_t* bytes) {
+    GS_TRY(return sim_workspace_bytes(prog, opts, bytes);)
+}
+
+gs_status gs_sim_create(const gs_program* prog, const gs_sim_opts* opts, void* dev_ws, size_t bytes, gs_sim** out) {
+    GS_TRY(return sim_create(prog, opts, dev_ws, bytes, out);)
+}
+
+gs_status gs_sim_destroy(gs_sim* s) {
+    if (!s) return GS_OK;
+    GS_TRY({
+        cudaSetDevice(s->opts.device);
+        cudaStreamSynchronize(s->stream);
+        free_sim(s);
+        return GS_OK;
+    })
+}
+
+gs_status gs_sim_reset(gs_sim* s) { GS_TRY(return sim_reset(s);) }
+
+gs_status gs_sim_set_lane_offset(gs_sim* s, uint64_t lane_offset) { GS_TRY(return sim_set_lane_offset(s, lane_offset);) }
+
+gs_status gs_sim_bind_stimulus_generated(gs_sim* s, uint64_t seed) { GS_TRY(return sim_bind_generated(s, seed);) }
+
+gs_status gs_sim_bind_stimulus_device(gs_sim* s, const uint64_t* dev_words, uint32_t cycles) {
+    GS_TRY(return sim_bind_device(s, dev_words, cycles);)
+}
+
+gs_status gs_sim_bind_stimulus_host(gs_sim* s, const uint64_t* words, uint32_t cycles) {
+    GS_TRY(return sim_bind_host(s, words, cycles);)
+}
+
+gs_status gs_sim_step(gs_sim* s, uint32_t n) { GS_TRY(return sim_step(s, n);) }
+
+gs_status gs_sim_run_streamed(gs_sim* s, const uint64_t* host_stim, uint64_t* host_out, uint32_t ncycles,
+                              uint32_t chunk) {
+    GS_TRY(return sim_run_streamed(s, host_stim, host_out, ncycles, chunk);)
+}
+
+gs_status gs_sim_sync(gs_sim* s) {
+    GS_TRY({
+        if (gs_status st = check_sim(s, "gs_sim_sync")) return st;
+        CU(cudaSetDevice(s->opts.device));
+        CU(cudaStreamSynchronize(s->stream));
+        clear_error();
+        return GS_OK;
+    })
+}
+
+gs_status gs_sim_get_cycle(const gs_sim* s, uint64_t* cycle) {
+    GS_TRY({
+        if (!s || !cycle) return fail(GS_ERR_ARG, "gs_sim_get_cycle: NULL argument");
+        *cycle = s->cycle;
+        clear_error();
+        return GS_OK;
+    })
+}
+
+gs_status gs_sim_get_config(const gs_sim* s, int* kernel, uint32_t* lane_groups) {
+    GS_TRY({
+        if (!s || !kernel || !lane_groups) return fail(GS_ERR_ARG, "gs_sim_get_config: NULL argument");
+        *kernel = s->opts.kernel;
+        *lane_groups = s->groups;
+        clear_error();
+        return GS_OK;
+    })
+}
+
+gs_status gs_sim_read_outputs(gs_sim* s, uint64_t* host, size_t nwords) { GS_TRY(return sim_read_outputs(s, host, nwords);) }
+
+gs_status gs_sim_read_registers(gs_sim* s, uint64_t* host, size_t nwords) {
+    GS_TRY(return sim_rw_registers(s, host, nullptr, nwords);)
+}
+
+gs_status gs_sim_write_registers(gs_sim* s, const uint64_t* host, size_t nwords) {
+    GS_TRY({
+        if (!host && s && s->prog->n_reg) return fail(GS_ERR_ARG, "gs_sim_write_registers: NULL buffer");
+        return sim_rw_registers(s, nullptr, host, nwords);
+    })
+}
+
+gs_status gs_sim_read_trace(gs_sim* s, uint64_t* host, size_t nwords, uint32_t* cycles_recorded) {
+    GS_TRY(return sim_read_trace(s, host, nwords, cycles_recorded);)
+}
+
+gs_status gs_sim_read_lane_signatures(gs_sim* s, uint64_t* host, size_t nlanes) {
+    GS_TRY(return sim_read_lane_signatures(s, host, nlanes);)
+}
+
+gs_status gs_sim_read_signature(gs_sim* s, gs_signature* out) { GS_TRY(return sim_read_signature(s, out);) }
+
+gs_status gs_sim_launches_per_cycle(const gs_sim* s, uint64_t* launches) {
+    GS_TRY({
+        if (!s || !launches) return fail(GS_ERR_ARG, "gs_sim_launches_per_cycle: NULL argument");
+        *launches = launches_per_cycle(s);
+        clear_error();
+        return GS_OK;
+    })
+}
+
+gs_status gs_sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) { GS_TRY(return sim_profile_step(s, n, out);) }
 
 }  // extern "C"

@@ -24,7 +24,8 @@ def test_library_exports_every_header_symbol():
     for name in declared:
         assert hasattr(lib, name), name
     assert declared == set(gs.EXPORTED)
-    assert gs.version() == "0.1.0"
+    assert gs.version() == "0.2.0"
+    assert len(gs.build_id()) == 16 and gs.build_id() != "unknown"
 
 
 def _compile(nl, balance=True):
@@ -299,14 +300,47 @@ def test_program_save_load_round_trip(tmp_path):
             gs.Program.load(str(tmp_path / "flip.gsp"))
 
 
-def test_recency_order_is_a_permutation_within_levels():
-    """order = 1 keeps every gate's level and the level widths; only positions inside a level
-    move (gs_compile_opts.order)."""
-    nl = workloads.synthetic(20000, 800, 32, 48, 24, seed=12, name="s")
-    a = gs.Netlist.from_arrays(nl).compile()
-    b = gs.Netlist.from_arrays(nl).compile(order=1)
-    assert np.array_equal(a.level_widths(), b.level_widths())
-    assert np.array_equal(a.gate_levels(), b.gate_levels())
-    assert a.info["program_hash"] != b.info["program_hash"]
-    with pytest.raises(gs.GsError):
-        gs.Netlist.from_arrays(nl).compile(order=2)
+def _fnv(data: bytes) -> int:
+    h = 0xCBF29CE484222325
+    for b in data:
+        h = ((h ^ b) * 0x100000001B3) & ((1 << 64) - 1)
+    return h
+
+
+def test_program_load_validates_every_index(tmp_path):
+    """An edited program file whose checksum was recomputed must still be rejected when an
+    index is out of range (row refs, latch registers, offsets), and by the index
+    validation, before the program hash is even looked at."""
+    import struct
+    nl = workloads.random_tiny(3, n_pi=5, n_reg=4, n_gates=60, n_po=6, max_k=4)
+    p = gs.Netlist.from_arrays(nl).compile()
+    f = tmp_path / "p.gsp"
+    p.save(str(f))
+    data = bytearray(f.read_bytes())
+    hdr = 8 + 4 + 6 * 4 + 3 * 4 + 8 + 1 + 4               # magic, format, scalars
+    n_lv = struct.unpack_from("<Q", data, hdr)[0]
+    assert n_lv == p.info["n_levels"] + 1
+    in_lo = hdr + 8 + 4 * n_lv + 8                        # first element of in_lo
+    n_in = struct.unpack_from("<Q", data, in_lo - 8)[0]
+    assert n_in == 4 * p.info["n_eval_gates"]
+    aux = in_lo + 4 * n_in + 8 + 8                        # in_hi is empty (k <= 4): count only
+    last_gate = p.info["n_eval_gates"] - 1
+
+    def write(mut, name):
+        # edit, then recompute the FNV-1a checksum (over every byte before it) like an attacker
+        d = bytearray(data)
+        mut(d)
+        d[-8:] = struct.pack("<Q", _fnv(bytes(d[:-8])))
+        out = tmp_path / name
+        out.write_bytes(bytes(d))
+        with pytest.raises(gs.GsError) as e:
+            gs.Program.load(str(out))
+        return str(e.value)
+
+    msgs = [
+        write(lambda d: struct.pack_into("<I", d, in_lo + 16 * last_gate, 0x7FFFFFF0), "row.gsp"),
+        write(lambda d: struct.pack_into("<I", d, in_lo, p.info["n_rows"] - 1), "fwd.gsp"),
+        write(lambda d: struct.pack_into("<I", d, aux + 16 * last_gate + 8, 0x7000000), "qdst.gsp"),
+    ]
+    for m in msgs:
+        assert "inconsistent program (" in m and "hash mismatch" not in m, m

@@ -53,6 +53,35 @@ def build_netlist(name: str) -> Netlist:
     raise KeyError(name)
 
 
+def sample_lanes(lanes_total: int, shards: int = 1, per_shard: int = 256, seed: int = 0,
+                 groups: int = 4, lanes_per_word: int = 4) -> np.ndarray:
+    """Deterministic lane sample for the oracle comparison at full size (SURVEY §8(c) "Whole
+    engine"): ``per_shard`` lanes in every one of ``shards`` equal shards, grouped
+    ``lanes_per_word`` to a 64-lane word (so a trace of few words covers them), always
+    including each shard's first and last word, the words on both sides of every boundary
+    between ``groups`` equal lane groups of the shard, and bits 0 and 63 of every chosen
+    word.  Selection only: no method arithmetic."""
+    rng = np.random.default_rng(seed)
+    per = lanes_total // shards
+    W = per // 64
+    nw = max(1, per_shard // lanes_per_word)
+    out = []
+    for sh in range(shards):
+        must = {0, W - 1}
+        for g in range(1, groups):
+            if W % groups == 0:
+                must |= {g * W // groups - 1, g * W // groups}
+        must = sorted(w for w in must if 0 <= w < W)[:nw]
+        rest = np.setdiff1d(np.arange(W), must)
+        pick = list(must) + sorted(rng.choice(rest, size=min(nw - len(must), len(rest)), replace=False).tolist())
+        for w in sorted(pick):
+            bits = {0, 63} if lanes_per_word >= 2 else {0}
+            while len(bits) < min(lanes_per_word, 64):
+                bits.add(int(rng.integers(0, 64)))
+            out += [sh * per + 64 * w + b for b in sorted(bits)]
+    return np.array(out, dtype=np.int64)
+
+
 def random_host_stimulus(seed: int, cycles: int, n_pi: int, words: int) -> np.ndarray:
     """Paper-style host stimulus [cycle][pi][word] of uniform random uint64 words."""
     rng = np.random.default_rng(seed)
@@ -60,6 +89,6 @@ def random_host_stimulus(seed: int, cycles: int, n_pi: int, words: int) -> np.nd
                         dtype=np.uint64, endpoint=True)
 
 
-__all__ = ["Netlist", "Builder", "Config", "CONFIGS", "build_netlist", "adder",
+__all__ = ["Netlist", "Builder", "Config", "CONFIGS", "build_netlist", "adder", "sample_lanes",
            "array_multiplier", "synthetic", "probes_circuit", "register_edge_cases",
            "random_tiny", "random_host_stimulus", "LIBRARY", "tt_of"]
