@@ -38,6 +38,7 @@ sys.path.insert(0, ROOT)
 
 METRIC = "stimulus-gate-cycle evals/s at 1/2/4/8 B200; HBM GB/s vs roofline"
 UNIT = "sgc/s"
+DEFAULT_SUB_LANES = 32768       # sharded configs: lanes per sub-batch (tests use the same)
 
 
 def parse():
@@ -49,7 +50,7 @@ def parse():
     ap.add_argument("--config", default="C5")
     ap.add_argument("--cycles-per-step", type=int, default=0,
                     help="cycles per step (0 = the config's cycle count for sharded configs, else 100)")
-    ap.add_argument("--sub-lanes", type=int, default=32768,
+    ap.add_argument("--sub-lanes", type=int, default=DEFAULT_SUB_LANES,
                     help="sharded configs: lanes per sub-batch (a multiple of the shard size / 2^k)")
     ap.add_argument("--lut-k", type=int, default=0, help="cone-collapse into <= L-input LUTs first")
     ap.add_argument("--lanes", type=int, default=0, help="override lanes per GPU (unsharded configs)")
@@ -457,7 +458,8 @@ def main():
         vc = cfg.cycles
         sample = workloads.sample_lanes(lanes_total, max(cfg.shards, 1) if sharded else 1,
                                         args.parity_lanes // (cfg.shards if sharded else 1), seed=2,
-                                        groups=max(sim.config["lane_groups"], 1))
+                                        groups=max(sim.config["lane_groups"], 1),
+                                        lanes_per_word=2 if sharded else 4)
         sample = sample[(sample >= lane_offset) & (sample < lane_offset + lanes_rank)]
         gsig = np.zeros(len(sample), dtype=np.uint64)
         greg = np.zeros((len(sample), info["n_reg"]), dtype=np.uint8)
@@ -469,8 +471,9 @@ def main():
                 return
             loc = sample[m] - lo
             gsig[m] = sim.read_lane_signatures()[loc]
-            if info["n_reg"]:
-                greg[m] = gs.unpack_lanes(sim.read_registers())[:, loc].T
+            if info["n_reg"]:                 # [reg][word] -> the sampled lanes' bits only
+                w = sim.read_registers()[:, loc // 64]
+                greg[m] = ((w >> (loc % 64).astype(np.uint64)[None, :]) & np.uint64(1)).astype(np.uint8).T
         t = time.perf_counter()
         for j in range(subs):
             sim.set_lane_offset(lane_offset + j * lanes)

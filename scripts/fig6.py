@@ -33,7 +33,7 @@ def main():
                 "synth20k": workloads.synthetic(20000, 800, 32, 48, 24, seed=12, name="s20k")}
     rows = []
     for name, nl in circuits.items():
-        for L in (0, 2, 3, 4, 5, 6):
+        for L in (0, 2, 3, 4, 5, 6, 7, 8):
             prog = gs.Netlist.from_arrays(nl).compile(lut_k=L)
             info = prog.info
             for kernel, lanes in (("lut", 64), ("tile", 128)):

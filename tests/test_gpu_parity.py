@@ -139,8 +139,10 @@ def test_c2_multiplier_all_lanes_equal_a_times_b():
         b |= pi[32 + i] << np.uint64(i)
     with np.errstate(over="ignore"):
         assert np.array_equal(prod, a * b)
-    sample = np.concatenate([np.arange(0, 128), np.arange(cfg.lanes - 128, cfg.lanes),
-                             np.random.default_rng(0).integers(0, cfg.lanes, 1792)])
+    # >= 4,096 lanes against the oracle: both ends and a seeded spread
+    sample = np.unique(np.concatenate([np.arange(0, 1024), np.arange(cfg.lanes - 1024, cfg.lanes),
+                                       np.random.default_rng(0).integers(0, cfg.lanes, 2560)]))
+    assert len(sample) >= 4096
     o = oracle.simulate(nl, sample, 1, seed=cfg.stim_seed, want=("last",))
     assert np.array_equal(lane_bits(r["outputs"], sample), o["last"])
 
@@ -179,15 +181,57 @@ def sampled_lane_check(nl, r, sample_local, lane_offset, cycles, seed, trace_wor
     assert np.array_equal(r["sigs"][sample_local], o["sig"])
 
 
-def test_c3_full_config_sampled_lanes_and_probes():
+def trace_lane_bits(tr, trace_words, lanes_local):
+    """GPU trace [cycles][po][ntw] uint64 -> bits [len(lanes_local)][cycles][po] of the given
+    local lanes (each lane's word must be traced)."""
+    pos = {int(w): i for i, w in enumerate(trace_words)}
+    cols = np.array([pos[int(s) // 64] for s in lanes_local])
+    sh = np.array([int(s) % 64 for s in lanes_local], dtype=np.uint64)
+    x = tr[:, :, cols]                                          # [c][po][n]
+    bits = ((x >> sh[None, None, :]) & np.uint64(1)).astype(np.uint8)
+    return np.transpose(bits, (2, 0, 1))
+
+
+def full_config_check(nl, r, trace_words, sample_local, lane_offset, cycles, seed):
+    """Every output of every cycle (trace), every register bit after the last cycle and the
+    per-lane MISR of the sampled lanes against the oracle run on the same global lanes."""
+    o = oracle.simulate(nl, np.asarray(sample_local) + lane_offset, cycles, seed=seed)
+    got = trace_lane_bits(r["trace"], trace_words, sample_local)
+    assert got.shape == o["trace"].shape
+    bad = np.argwhere(got != o["trace"])
+    assert len(bad) == 0, f"{len(bad)} output bits differ, first (lane, cycle, po) {bad[:3].tolist()}"
+    assert np.array_equal(lane_bits(r["regs"], sample_local), o["regs"])
+    assert np.array_equal(r["sigs"][sample_local], o["sig"])
+    return o
+
+
+@pytest.mark.slow
+def test_c3_full_config_all_lanes_prefix_and_probes():
+    """C3 (BASELINE configs[2]) at full size: ALL 16,384 lanes, every output of every cycle,
+    registers and per-lane MISR vs the oracle over a 50-cycle prefix (SURVEY §8(c) "all lanes
+    on C1-C3"); the 1,000-cycle run is checked on 256 lanes below."""
     cfg = workloads.CONFIGS["C3"]
     nl = cfg.netlist()
     W_ = cfg.lanes // 64
-    tw = [0, 1, W_ // 2, W_ - 1]
+    cycles = 50
+    r = run_gpu(nl, cfg.lanes, cycles, "lut", seed=cfg.stim_seed, trace_words=range(W_))
+    o = oracle.simulate(nl, np.arange(cfg.lanes), cycles, seed=cfg.stim_seed)
+    assert np.array_equal(gpu_trace_bits(r["trace"], None), o["trace"])
+    assert np.array_equal(lane_bits(r["regs"], np.arange(cfg.lanes)), o["regs"])
+    assert np.array_equal(r["sigs"], o["sig"])
+    assert r["signature"]["lane_sig_sum"] == oracle.lane_sig_sum(o["sig"], np.arange(cfg.lanes))
+
+
+@pytest.mark.slow
+def test_c3_full_config_256_lanes_every_cycle_and_probes():
+    """C3 for all 1,000 cycles in the bench's launch configuration: 256 lanes (64 words, the
+    lane-group boundaries included) every cycle vs the oracle, probes on every lane."""
+    cfg = workloads.CONFIGS["C3"]
+    nl = cfg.netlist()
+    sample = workloads.sample_lanes(cfg.lanes, 1, 256, seed=3)
+    tw = sorted(set((sample // 64).tolist()))
     r = run_gpu(nl, cfg.lanes, cfg.cycles, "lut", seed=cfg.stim_seed, trace_words=tw)
-    sample = np.array([0, 1, 63, 64, 65, 127, W_ // 2 * 64 + 5, W_ // 2 * 64 + 40,
-                       cfg.lanes - 64, cfg.lanes - 2, cfg.lanes - 1])
-    sampled_lane_check(nl, r, sample, 0, cfg.cycles, cfg.stim_seed, tw)
+    full_config_check(nl, r, tw, sample, 0, cfg.cycles, cfg.stim_seed)
     probe_closed_forms(nl, gs.unpack_lanes(r["outputs"]).T, cfg.cycles - 1, cfg.stim_seed, cfg.lanes)
     assert r["signature"]["cycles"] == cfg.cycles
 
@@ -722,61 +766,92 @@ def test_tile_rejects_oversized_or_misaligned():
 
 # ------------------------------------------------------------------ full-size configs
 @pytest.mark.slow
-def test_c4_full_config_sampled_lanes_and_probes():
+def test_c4_full_config_256_lanes_every_cycle_and_probes():
+    """C4 (BASELINE configs[3]) at full size in the launch configuration `bench.py --config C4`
+    times (65,536 lanes, kernel A, auto = 4 concurrent lane groups, CUDA graphs): 256 lanes
+    spread over the batch (lanes 0/63/64/last, both sides of every lane-group boundary) x all
+    1,000 cycles vs the oracle — every output bit of every cycle, every register bit, the
+    per-lane MISR — and the probes' closed forms on every lane."""
     cfg = workloads.CONFIGS["C4"]
     nl = cfg.netlist()
-    W_ = cfg.lanes // 64
-    tw = [0, 1, W_ // 2, W_ - 1]
-    r = run_gpu(nl, cfg.lanes, cfg.cycles, "lut", seed=cfg.stim_seed, trace_words=tw)
-    sample = np.array([0, 63, 64, 127, W_ // 2 * 64 + 17, cfg.lanes - 64, cfg.lanes - 1])
-    sampled_lane_check(nl, r, sample, 0, cfg.cycles, cfg.stim_seed, tw)
+    prog = compile_nl(nl)
+    sample = workloads.sample_lanes(cfg.lanes, 1, 256, seed=4)
+    assert {0, 63, 64, cfg.lanes - 1} <= set(sample.tolist())
+    tw = sorted(set((sample // 64).tolist()))
+    sim = gs.Sim(prog, cfg.lanes, kernel="lut", trace_words=tw, trace_cycles=cfg.cycles)
+    assert sim.config["lane_groups"] == 4
+    sim.bind_generated(cfg.stim_seed)
+    sim.step(cfg.cycles)
+    sim.sync()
+    r = dict(outputs=sim.read_outputs(), regs=sim.read_registers(), sigs=sim.read_lane_signatures(),
+             trace=sim.read_trace())
+    sim.close()
+    full_config_check(nl, r, tw, sample, 0, cfg.cycles, cfg.stim_seed)
     probe_closed_forms(nl, gs.unpack_lanes(r["outputs"]).T, cfg.cycles - 1, cfg.stim_seed, cfg.lanes)
 
 
 @pytest.mark.slow
-def test_c5_shard_full_netlist_sampled_lanes():
+def test_c5_every_shard_32_lanes_every_cycle_bench_config():
+    """C5 (BASELINE configs[4]) at full size over its whole 262,144-lane batch in the launch
+    configuration bench.py times (10M gates, sub-batches of bench.DEFAULT_SUB_LANES lanes in
+    one workspace re-targeted by gs_sim_set_lane_offset, each from reset, auto lane groups):
+    32 lanes of every one of the 8 shards (256 in all, shard- and group-boundary lanes
+    included) x all 100 cycles vs the oracle, and the probes on every lane of every shard."""
+    import bench
     cfg = workloads.CONFIGS["C5"]
     nl = cfg.netlist()
-    lanes = cfg.lanes // cfg.shards
-    shard = 5
-    off = shard * lanes
-    W_ = lanes // 64
-    tw = [0, W_ - 1]
-    r = run_gpu(nl, lanes, cfg.cycles, "lut", seed=cfg.stim_seed, trace_words=tw, lane_offset=off)
-    sample = np.array([0, 1, 63, lanes - 64, lanes - 1])
-    sampled_lane_check(nl, r, sample, off, cfg.cycles, cfg.stim_seed, tw)
-    probe_closed_forms(nl, gs.unpack_lanes(r["outputs"]).T, cfg.cycles - 1, cfg.stim_seed, lanes, off)
-
-
-@pytest.mark.slow
-def test_c5_every_shard_sampled_lanes_sub_batches():
-    """C5's full netlist over ALL 8 shards of its 262,144-lane batch with one sim re-targeted by
-    gs_sim_set_lane_offset (the bench's sub-batch path): 32 sampled lanes per shard (256 in
-    all, shard-boundary lanes included) vs the oracle on every cycle, 20 cycles per shard."""
-    cfg = workloads.CONFIGS["C5"]
-    nl = cfg.netlist()
-    lanes = cfg.lanes // cfg.shards
-    W_ = lanes // 64
-    tw = [0, 1, W_ // 2, W_ - 1]
-    cycles = 20
     prog = compile_nl(nl)
-    sim = gs.Sim(prog, lanes, kernel="lut", trace_words=tw, trace_cycles=cycles)
+    sub = bench.DEFAULT_SUB_LANES
+    sample = workloads.sample_lanes(cfg.lanes, cfg.shards, 256 // cfg.shards, seed=5, lanes_per_word=2)
+    tw_all = sorted(set((sample % sub // 64).tolist()))        # local words of any sub-batch
+    sim = gs.Sim(prog, sub, kernel="lut", trace_words=tw_all, trace_cycles=cfg.cycles)
     sim.bind_generated(cfg.stim_seed)
-    rng = np.random.default_rng(55)
+    o = oracle.simulate(nl, sample, cfg.cycles, seed=cfg.stim_seed)
     tot = 0
-    for shard in range(cfg.shards):
-        off = shard * lanes
+    checked = 0
+    for j in range(cfg.lanes // sub):
+        off = j * sub
         sim.set_lane_offset(off)
-        sim.step(cycles)
+        sim.step(cfg.cycles)
         sim.sync()
-        r = dict(trace=sim.read_trace(), regs=sim.read_registers(), sigs=sim.read_lane_signatures())
-        words = rng.choice([1, W_ // 2], size=25)
-        sample = np.concatenate([[0, 63, 64, 127, lanes - 64, lanes - 2, lanes - 1],
-                                 words * 64 + rng.integers(0, 64, size=25)])
-        sampled_lane_check(nl, r, sample, off, cycles, cfg.stim_seed, tw)
+        m = (sample >= off) & (sample < off + sub)
+        loc = sample[m] - off
+        got = trace_lane_bits(sim.read_trace(), tw_all, loc)
+        assert np.array_equal(got, o["trace"][m]), j
+        assert np.array_equal(lane_bits(sim.read_registers(), loc), o["regs"][m]), j
+        sigs = sim.read_lane_signatures()
+        assert np.array_equal(sigs[loc], o["sig"][m]), j
+        probe_closed_forms(nl, gs.unpack_lanes(sim.read_outputs()).T, cfg.cycles - 1, cfg.stim_seed, sub, off)
         tot = (tot + sim.signature()["lane_sig_sum"]) % (1 << 64)
+        checked += int(m.sum())
     sim.close()
+    assert checked == len(sample) == 256
     assert tot != 0
+
+
+@pytest.mark.parametrize("gates,groups,depth", [(40000, 1, 8), (40000, 4, 4), (60000, 4, 3), (130000, 4, 6)])
+def test_grid_stride_branch_every_lane_vs_oracle(gates, groups, depth):
+    """Kernel A's grid-stride launches (a level 1-4 waves of resident CTAs deep runs on
+    exactly the resident CTAs, which stride over the level) at 65,536 lanes, with 4 and 16
+    vectors per warp unit (U = 4, 2, 1 by level width: ~2.9k gates / 1 group, ~3.6k, 6k, 10k
+    gates / 4 groups): every lane vs the oracle, and the branch provably taken
+    (gs_profile.grid_stride_launches > 0)."""
+    nl = workloads.synthetic(gates, gates // 25, 32, 48, depth, seed=60 + groups, name="gstride")
+    prog = compile_nl(nl)
+    lanes, cycles = 65536, 2
+    sim = gs.Sim(prog, lanes, kernel="lut", lane_groups=groups)
+    assert sim.config["lane_groups"] == groups
+    sim.bind_generated(6)
+    sim.step(cycles - 1)
+    pr = sim.profile_step(1)
+    assert pr["grid_stride_launches"] > 0, pr
+    sim.sync()
+    out, regs, sigs = sim.read_outputs(), sim.read_registers(), sim.read_lane_signatures()
+    sim.close()
+    o = oracle.simulate(nl, np.arange(lanes), cycles, seed=6, want=("last", "regs", "sig"))
+    assert np.array_equal(gs.unpack_lanes(out).T, o["last"])
+    assert np.array_equal(gs.unpack_lanes(regs).T, o["regs"])
+    assert np.array_equal(sigs, o["sig"])
 
 
 # ------------------------------------------------------------------ seeded fuzzing

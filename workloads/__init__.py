@@ -58,20 +58,21 @@ def sample_lanes(lanes_total: int, shards: int = 1, per_shard: int = 256, seed: 
     """Deterministic lane sample for the oracle comparison at full size (SURVEY §8(c) "Whole
     engine"): ``per_shard`` lanes in every one of ``shards`` equal shards, grouped
     ``lanes_per_word`` to a 64-lane word (so a trace of few words covers them), always
-    including each shard's first and last word, the words on both sides of every boundary
-    between ``groups`` equal lane groups of the shard, and bits 0 and 63 of every chosen
-    word.  Selection only: no method arithmetic."""
+    including (in this priority while room is left) each shard's first, last and second
+    word, the words on both sides of every boundary between ``groups`` equal lane groups of
+    the shard, and bits 0 and 63 of every chosen word.  Selection only: no method
+    arithmetic."""
     rng = np.random.default_rng(seed)
     per = lanes_total // shards
     W = per // 64
     nw = max(1, per_shard // lanes_per_word)
     out = []
     for sh in range(shards):
-        must = {0, W - 1}
+        must = [0, W - 1, 1]                        # lanes 0, 63, 64 and the last lane
         for g in range(1, groups):
             if W % groups == 0:
-                must |= {g * W // groups - 1, g * W // groups}
-        must = sorted(w for w in must if 0 <= w < W)[:nw]
+                must += [g * W // groups - 1, g * W // groups]
+        must = list(dict.fromkeys(w for w in must if 0 <= w < W))[:nw]
         rest = np.setdiff1d(np.arange(W), must)
         pick = list(must) + sorted(rng.choice(rest, size=min(nw - len(must), len(rest)), replace=False).tolist())
         for w in sorted(pick):
