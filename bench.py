@@ -54,10 +54,14 @@ def parse():
                     help="sharded configs: lanes per sub-batch (a multiple of the shard size / 2^k)")
     ap.add_argument("--lut-k", type=int, default=0, help="cone-collapse into <= L-input LUTs first")
     ap.add_argument("--lanes", type=int, default=0, help="override lanes per GPU (unsharded configs)")
-    ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab", "tile", "auto"])
+    ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab", "tile", "cluster", "auto"])
+    ap.add_argument("--cluster-size", type=int, default=0, help="kernel C: CTAs per cluster (0 = auto)")
+    ap.add_argument("--slab-lanes", type=int, default=0, help="kernel C: lanes per slab (0 = auto)")
     ap.add_argument("--no-balance", action="store_true", help="ASAP levels (balance-off A/B)")
     ap.add_argument("--tile-words", type=int, default=0, help="kernel T: 32-bit words per slot")
     ap.add_argument("--tile-groups", type=int, default=0, help="kernel T: thread groups per CTA")
+    ap.add_argument("--tile-desc", default="auto", choices=["auto", "tma", "global"],
+                    help="kernel T descriptor source (auto: resident if it fits, else TMA stream)")
     ap.add_argument("--lut-unroll", type=int, default=0, help="vectors per thread (0 = auto)")
     ap.add_argument("--lane-groups", type=int, default=0,
                     help="kernel A: concurrent lane groups per cycle (0 = library auto, 1 = off)")
@@ -317,10 +321,11 @@ def main():
     if world > 1:
         gdist.check_same_program(info["program_hash"])
     stream = torch.cuda.Stream(device=local)
-    flags = (8 if args.no_grid_stride else 0)
+    flags = (8 if args.no_grid_stride else 0) | {"auto": 0, "global": 16, "tma": 32}[args.tile_desc]
     sim = gs.Sim(prog, lanes, lane_offset=lane_offset, kernel=args.kernel, device=local, stream=stream,
                  lut_unroll=args.lut_unroll, pdl=not args.no_pdl, tile_words=args.tile_words,
-                 tile_groups=args.tile_groups, lane_groups=args.lane_groups, flags=flags)
+                 tile_groups=args.tile_groups, lane_groups=args.lane_groups, flags=flags,
+                 cluster_size=args.cluster_size, slab_lanes=args.slab_lanes)
     sim.bind_generated(cfg.stim_seed)
     launches_per_cycle = sim.launches_per_cycle()
 
@@ -498,6 +503,7 @@ def main():
                        "lut_unroll": args.lut_unroll, "lane_groups": sim.config["lane_groups"],
                        "pdl": not args.no_pdl, "tile_words": args.tile_words, "tile_groups": args.tile_groups,
                        "lut_k": args.lut_k, "grid_stride": not args.no_grid_stride,
+                       "launch": sim.launch,
                        "l2": "inputs larger than L2 (state %.1f GB per sub-batch)" % (info["n_rows"] * lanes / 8 / 1e9),
                        "step": (f"the whole batch: {subs} sub-batch(es) of {lanes} lanes per GPU, each from reset "
                                 f"for {C} cycles" if sharded else f"{C} more cycles over every lane of the GPU"),
@@ -506,7 +512,7 @@ def main():
                        "compile_s": round(compile_s, 2), "build_id": gs.build_id(),
                        "program_hash": str(info["program_hash"]),
                        "paper_style_gcps": value * (G + info["n_reg"]) / G},
-            "gpu_launches": int(launches_per_cycle * (1 if args.kernel == "tile" else C) * args.steps * subs),
+            "gpu_launches": int(launches_per_cycle * (1 if args.kernel in ("tile", "cluster") else C) * args.steps * subs),
             "signature": {k: str(v) for k, v in red.items()},
             "nccl": ({"nranks": nranks, "ok": nranks == world} if nranks is not None else None),
             "clocks": clk,

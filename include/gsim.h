@@ -145,7 +145,9 @@ gs_status gs_netlist_get_counts(const gs_netlist* nl, gs_netlist_counts* out);
 /* ======================================================================= compile */
 typedef struct {
     int balance;      /* 0: ASAP levels.  1: slack-based balancing within [ASAP, ALAP]
-                         (same depth; flattens the unbalanced level widths) */
+                         (same depth; flattens the unbalanced level widths).
+                         2: ALAP levels (same depth; shortest live ranges, so the fewest
+                         kernel-T shared-memory slots).  Results never depend on it.   */
     uint32_t max_k;   /* reject gates wider than this (0 = GS_MAX_K_POLY)             */
     uint32_t lut_k;   /* 0: evaluate the netlist's LUTs as given.  L in [2, max_k]: first
                          collapse cones into LUTs of at most L inputs (the paper's LUT
@@ -230,11 +232,18 @@ enum {
                              are counted                                            */
     GS_KERNEL_AB = 3,     /* A writes, B recomputes every level and counts mismatches      */
     /* 4: retired in 0.2.0 (an experimental persistent schedule, measured slower than A)   */
-    GS_KERNEL_TILE = 5     /* kernel T: each CTA owns a tile of 32*tile_words lanes and runs
+    GS_KERNEL_TILE = 5,    /* kernel T: each CTA owns a tile of 32*tile_words lanes and runs
                              every level of every cycle of a gs_sim_step in shared memory
                              (gate values in slots reused by live range); one launch per
                              step, HBM touched only for registers/MISR at step boundaries.
                              Needs the live slots of one tile to fit shared memory.          */
+    GS_KERNEL_CLUSTER = 6  /* kernel C: kernel A's state layout and gate evaluation, but a
+                             thread-block cluster owns a lane slab (slab_lanes lanes) and walks
+                             every level of every cycle of a gs_sim_step for it, the cluster's
+                             CTAs splitting each level, a hardware cluster barrier between
+                             levels; slabs from an atomic queue.  One launch per step; the
+                             lanes in flight are bounded so a level's rows are still in L2
+                             when the next levels read them.                               */
 };
 
 typedef struct {
@@ -259,6 +268,10 @@ typedef struct {
                                      ramp and drain overlap another's levels.  Needs
                                      (lanes/128) % groups == 0 and a multiple of 4096 lanes
                                      per group.  0 = auto, 1 = off.           */
+    uint32_t cluster_size;        /* CLUSTER: CTAs per thread-block cluster (1, 2, 4, 8 or 16;
+                                     0 = auto)                                             */
+    uint32_t slab_lanes;          /* CLUSTER: lanes per slab, a multiple of 128 dividing lanes
+                                     (0 = auto)                                            */
 } gs_sim_opts;
 /* flags: launch the per-cycle kernels WITHOUT programmatic dependent launch (by default a
  * level kernel may become resident while its predecessor drains; A/B measurement only). */
@@ -329,6 +342,18 @@ gs_status gs_sim_get_cycle(const gs_sim* sim, uint64_t* cycle);
 /* The resolved launch configuration: kernel (GS_KERNEL_*, AUTO resolved) and the number of
  * concurrent lane groups (1 = a single level chain per cycle). */
 gs_status gs_sim_get_config(const gs_sim* sim, int* kernel, uint32_t* lane_groups);
+
+/* The resolved launch plan of the sim (what gs_sim_step launches). */
+typedef struct {
+    int kernel;                   /* GS_KERNEL_* (AUTO resolved)                            */
+    uint32_t lane_groups;         /* kernel A: concurrent lane groups                       */
+    uint32_t tile_words, tile_groups, tile_desc;   /* kernel T: words per slot, thread groups
+                                     per CTA, descriptor source (0 global, 1 resident, 2 TMA) */
+    uint32_t grid;                /* kernels T / C: CTAs launched per step                  */
+    uint32_t cluster_size, slab_lanes;             /* kernel C                                 */
+    uint32_t live_slots;          /* kernel T: shared-memory slots per tile                 */
+} gs_launch_info;
+gs_status gs_sim_get_launch(const gs_sim* sim, gs_launch_info* out);
 
 /* Readback (synchronous).  Layouts, with W = lanes/64 local words:
  *   outputs   [po][W]  outputs of the last stepped cycle (before its latch, R4)

@@ -29,8 +29,9 @@ GS_SIM_NO_PDL = 1
 GS_SIM_NO_GRID_STRIDE = 8     # kernel A: one CTA per work chunk (A/B measurement only)
 GS_SIM_TILE_DESC_GLOBAL = 16  # kernel T: descriptors read from global memory
 GS_SIM_TILE_DESC_TMA = 32     # kernel T: descriptors TMA-streamed level by level
-GS_KERNEL_AUTO, GS_KERNEL_LUT, GS_KERNEL_POLY, GS_KERNEL_AB, GS_KERNEL_TILE = 0, 1, 2, 3, 5
-KERNELS = {"auto": 0, "lut": 1, "A": 1, "poly": 2, "B": 2, "ab": 3, "AB": 3, "tile": 5, "T": 5}
+GS_KERNEL_AUTO, GS_KERNEL_LUT, GS_KERNEL_POLY, GS_KERNEL_AB, GS_KERNEL_TILE, GS_KERNEL_CLUSTER = 0, 1, 2, 3, 5, 6
+KERNELS = {"auto": 0, "lut": 1, "A": 1, "poly": 2, "B": 2, "ab": 3, "AB": 3, "tile": 5, "T": 5,
+           "cluster": 6, "C": 6}
 
 
 class GsError(RuntimeError):
@@ -75,7 +76,8 @@ class gs_sim_opts(C.Structure):
                 ("lane_offset", C.c_uint64), ("kernel", C.c_int), ("n_trace_words", C.c_uint32),
                 ("trace_words", C.c_void_p), ("trace_cycles", C.c_uint32), ("use_graphs", C.c_int),
                 ("lut_unroll", C.c_uint32), ("flags", C.c_uint32), ("tile_words", C.c_uint32),
-                ("tile_groups", C.c_uint32), ("lane_groups", C.c_uint32)]
+                ("tile_groups", C.c_uint32), ("lane_groups", C.c_uint32), ("cluster_size", C.c_uint32),
+                ("slab_lanes", C.c_uint32)]
 
 
 class gs_signature(C.Structure):
@@ -85,6 +87,12 @@ class gs_signature(C.Structure):
 
     def as_dict(self):
         return {f: int(getattr(self, f)) for f, _ in self._fields_}
+
+
+class gs_launch_info(C.Structure):
+    _fields_ = [("kernel", C.c_int), ("lane_groups", C.c_uint32), ("tile_words", C.c_uint32),
+                ("tile_groups", C.c_uint32), ("tile_desc", C.c_uint32), ("grid", C.c_uint32),
+                ("cluster_size", C.c_uint32), ("slab_lanes", C.c_uint32), ("live_slots", C.c_uint32)]
 
 
 class gs_profile(C.Structure):
@@ -133,6 +141,7 @@ _SIGS = {
     "gs_sim_run_streamed": (C.c_int32, [_P, _P, _P, C.c_uint32, C.c_uint32]),
     "gs_sim_get_cycle": (C.c_int32, [_P, _P]),
     "gs_sim_get_config": (C.c_int32, [_P, _P, _P]),
+    "gs_sim_get_launch": (C.c_int32, [_P, _P]),
     "gs_sim_read_outputs": (C.c_int32, [_P, _P, C.c_size_t]),
     "gs_sim_read_registers": (C.c_int32, [_P, _P, C.c_size_t]),
     "gs_sim_write_registers": (C.c_int32, [_P, _P, C.c_size_t]),
@@ -248,16 +257,18 @@ class Netlist:
         _call("gs_netlist_get_counts", self.h, C.byref(c))
         return {f: int(getattr(c, f)) for f, _ in c._fields_}
 
-    def compile(self, balance: bool = True, max_k: int = 0, lut_k: int = 0, level_seed: int = 0) -> "Program":
+    def compile(self, balance=True, max_k: int = 0, lut_k: int = 0, level_seed: int = 0) -> "Program":
         return Program(self, balance, max_k, lut_k, level_seed=level_seed)
 
 
 class Program:
-    def __init__(self, netlist: Netlist | None, balance: bool = True, max_k: int = 0, lut_k: int = 0,
+    def __init__(self, netlist: Netlist | None, balance=True, max_k: int = 0, lut_k: int = 0,
                  _handle=None, level_seed: int = 0):
         if _handle is None:
             h = C.c_void_p()
-            o = gs_compile_opts(1 if balance else 0, max_k, lut_k, int(level_seed))
+            # balance: True/1 slack-balanced, False/0 ASAP, 2 or "alap" ALAP levels
+            b = 2 if balance in (2, "alap") else (1 if balance else 0)
+            o = gs_compile_opts(b, max_k, lut_k, int(level_seed))
             _call("gs_compile", netlist.h, C.byref(o), C.byref(h))
         else:
             h = _handle
@@ -315,7 +326,8 @@ class Sim:
     def __init__(self, program: Program, lanes: int, lane_offset: int = 0, kernel="lut",
                  device: int = 0, stream=None, trace_words=(), trace_cycles: int = 0,
                  use_graphs: bool = True, lut_unroll: int = 0, pdl: bool = True,
-                 tile_words: int = 0, tile_groups: int = 0, flags: int = 0, lane_groups: int = 0):
+                 tile_words: int = 0, tile_groups: int = 0, flags: int = 0, lane_groups: int = 0,
+                 cluster_size: int = 0, slab_lanes: int = 0):
         import torch
         self.program = program
         self.lanes, self.words = int(lanes), int(lanes) // 64
@@ -327,7 +339,7 @@ class Sim:
                         _p(self._tw) if len(self._tw) else None, int(trace_cycles),
                         1 if use_graphs else 0, int(lut_unroll),
                         (0 if pdl else GS_SIM_NO_PDL) | int(flags), int(tile_words), int(tile_groups),
-                        int(lane_groups))
+                        int(lane_groups), int(cluster_size), int(slab_lanes))
         nbytes = C.c_size_t()
         _call("gs_sim_workspace_bytes", program.h, C.byref(o), C.byref(nbytes))
         self.workspace = torch.empty(int(nbytes.value) + 256, dtype=torch.uint8, device=self.device)
@@ -392,6 +404,13 @@ class Sim:
         k, g = C.c_int32(), C.c_uint32()
         _call("gs_sim_get_config", self.h, C.byref(k), C.byref(g))
         return {"kernel": k.value, "lane_groups": g.value}
+
+    @property
+    def launch(self) -> dict:
+        """Resolved launch plan (gs_sim_get_launch)."""
+        li = gs_launch_info()
+        _call("gs_sim_get_launch", self.h, C.byref(li))
+        return {f: int(getattr(li, f)) for f, _ in li._fields_}
 
     @property
     def cycle(self) -> int:

@@ -143,6 +143,33 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
             alap[g] = a;
         }
     }
+    // peak number of gate values live at one level boundary for a level assignment: a value
+    // lives from its level to its last reader's level (outputs and leftover latch sources:
+    // to the end of the cycle), the quantity tile.cpp's interval colouring allocates
+    auto peak_live = [&](const std::vector<uint32_t>& lv) -> uint64_t {
+        std::vector<int64_t> diff(D + 3, 0);
+        std::vector<uint32_t> last(G, 0);
+        for (uint32_t g = 0; g < G; ++g)
+            if (nl.gate_k[g] > 0) last[g] = lv[g];
+        for (uint32_t g = 0; g < G; ++g)
+            for (uint32_t e = cons_off[g]; e < cons_off[g + 1]; ++e) last[g] = std::max(last[g], lv[cons[e]]);
+        for (uint32_t o = 0; o < O; ++o) {
+            const uint32_t n = nl.po_net[o];
+            if (is_eval_gate_net(n)) last[nl.net_index[n]] = D + 1;
+        }
+        for (uint32_t r = 0; r < R; ++r) {
+            const uint32_t n = nl.reg_d[r];
+            if (is_eval_gate_net(n)) last[nl.net_index[n]] = D + 1;
+        }
+        for (uint32_t g = 0; g < G; ++g)
+            if (nl.gate_k[g] > 0) {
+                diff[lv[g]] += 1;
+                diff[last[g] + 1] -= 1;
+            }
+        int64_t cur = 0, peak = 0;
+        for (uint32_t l = 0; l < D + 3; ++l) peak = std::max(peak, cur += diff[l]);
+        return (uint64_t)peak;
+    };
     if (opts.level_seed && n_eval > 0) {
         // seeded random valid levels: in topological order, uniform in [1 + max input level,
         // ALAP]; the upper end stays >= the lower one because every input's level is <= its
@@ -160,6 +187,11 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
             z ^= z >> 31;
             level[g] = lo + (uint32_t)(z % (uint64_t)(alap[g] - lo + 1));
         }
+    } else if (opts.balance == 2 && n_eval > 0) {
+        // ALAP: every gate as late as its consumers allow (same depth); a value is produced
+        // right before it is needed, which shortens live ranges (kernel T's shared-memory
+        // slots, tile.cpp) at the price of uneven widths
+        level = alap;
     } else if (opts.balance && n_eval > 0) {
         // list scheduling, level by level: least slack (smallest ALAP) first, must place
         // every gate whose ALAP is this level, otherwise fill up to the mean width.
@@ -187,6 +219,13 @@ gs_status compile(const Netlist& nl, const gs_compile_opts& opts, Program*& out)
                 }
         }
         if (!ready.empty()) return fail(GS_ERR_STATE, "gs_compile: internal balancing error");
+        // Filling levels up to the mean width moves gates with large slack (the partial
+        // products of a multiplier) early, where their values stay live for many levels.
+        // Where ALAP levels hold markedly fewer values live at once (kernel T keeps every live
+        // value of a tile in shared memory, so fewer live values = more lanes per SM), take ALAP
+        // instead: C2 (32x32 multiplier) 752 -> 256 peak live values; synthetic circuits keep
+        // the balanced levels (ALAP raises their peak).
+        if (peak_live(level) * 4 > peak_live(alap) * 5) level = alap;
     } else {
         level = asap;
     }

@@ -2,11 +2,14 @@
 #pragma once
 
 #include <cstdint>
+#include <vector>
 #include <cuda_runtime.h>
 
 #include "internal.h"
 
 namespace gs {
+
+constexpr uint32_t GS_TILE_CHUNK = 256;   // kernel T: most descriptors per TMA-streamed step
 
 // Device control block (first 256 B of the workspace).
 struct Ctl {
@@ -23,6 +26,8 @@ struct Ctl {
     unsigned long long sink_ptr;     // 0, or device [cycle - sink_base][po][word] every output
     unsigned long long sink_base;    //   of every cycle is written to (gs_sim_run_streamed)
     unsigned long long sink_cycles;  //   capacity in cycles
+    unsigned int tile_next;          // kernel T: next tile of the launch's queue (zeroed per launch)
+    unsigned int pad_;
 };
 
 struct LevelArgs {
@@ -72,12 +77,11 @@ struct EndArgs {
 struct TileArgs {
     const TileDesc* desc;             // [n_eval]
     const uint4* desc_hi;             // [n_eval] (k > 4 only)
-    const uint32_t* level_off;        // [n_levels + 1]
-    uint32_t n_eval, n_levels;
+    const uint2* steps;               // [n_steps] {first gate, gates}: one per non-empty level
+                                      // (chunks of <= TILE_CHUNK gates when TMA-streamed)
+    uint32_t n_eval, n_steps;
     uint32_t desc_smem;               // 0: descriptors read from global; 1: resident in shared
-                                      // memory; 2: TMA-streamed level by level (double buffer);
-                                      // | 4: slots in global memory instead of shared memory
-    uint32_t max_width;               // widest level (mode 2 buffer size, in descriptors)
+                                      // memory; 2: TMA-streamed step by step (double buffer)
     const uint32_t* po_slot;
     uint32_t n_po;
     const uint32_t* latch_src;
@@ -91,6 +95,7 @@ struct TileArgs {
     uint32_t words;                   // 64-bit words per state row (lanes / 64)
     uint32_t row_q0;
     Ctl* ctl;
+    unsigned int* tile_next;          // &ctl->tile_next (the tile queue)
     unsigned long long* misr;         // 2 x [64][words] (buffer = cycle parity)
     const int32_t* trace_slot;
     unsigned long long* trace;
@@ -98,14 +103,49 @@ struct TileArgs {
     uint64_t word_off;                // global 64-bit word of local lane 0
     uint32_t ncycles, n_tiles;
 };
-size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
-                       int desc_mode, uint32_t max_width);
-cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
-                       int desc_smem, uint32_t max_width, uint32_t has_q, uint32_t* per_sm);
+// steps of a program for kernel T: one per non-empty level, levels wider than `chunk` gates
+// cut into chunks (chunk = 0: no cutting)
+void tile_steps(const uint32_t* level_off, uint32_t n_levels, uint32_t chunk, std::vector<uint2>& out);
+size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_steps,
+                       int desc_mode);
+cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_steps,
+                       int desc_smem, uint32_t has_q, uint32_t* per_sm);
 cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s);
 
 // *grid_stride (may be NULL) is set to 1 when the launch's grid was capped at the resident
 // capacity (the grid-stride branch), else 0
+// Kernel C (kernels_cluster.cu): a thread-block cluster owns a lane slab and walks every
+// level of every cycle of a step for it, cluster barrier between levels.
+struct ClusterArgs {
+    const uint4* din;
+    const GateAux* aux;
+    const uint4* dhi;                 // inputs 4..7 (gates with k > 4)
+    const uint4* dtt;                 // [n_eval][2] full 256-bit tables (programs with k > 6)
+    const uint2* steps;               // [n_steps] {first gate, gates} of every non-empty level
+    uint32_t n_steps;
+    uint8_t* state;
+    uint64_t stride;                  // bytes per state row
+    uint32_t words;                   // 64-bit words per row
+    uint32_t row_gate0, row_pi0, n_pi, row_q0, n_reg;
+    const uint32_t* latch_src;
+    const uint32_t* latch_dst;
+    uint32_t n_latch;
+    const uint32_t* po_rows;
+    uint32_t n_po;
+    unsigned long long* misr;         // 2 x [64][words] (buffer = cycle parity)
+    const int32_t* trace_slot;        // [words]
+    unsigned long long* trace;
+    uint32_t ntw, trace_cap;
+    Ctl* ctl;
+    unsigned int* tile_next;          // &ctl->tile_next (the slab queue)
+    uint64_t word_off;                // global 64-bit word of local lane 0
+    uint32_t ncycles;
+    uint32_t slab_vec, n_slabs;       // 16-byte vectors per slab row; slabs = lanes / (128 slab_vec)
+};
+uint32_t cluster_vpt(uint32_t slab_vec);
+cudaError_t cluster_max_active(uint32_t slab_vec, uint32_t cs, uint32_t* clusters);
+cudaError_t launch_cluster(const ClusterArgs& a, uint32_t clusters, uint32_t cs, cudaStream_t s);
+
 cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s, uint32_t* grid_stride = nullptr);
 uint32_t level_lut_resident_blocks(int device);   // CTAs of k_level_lut_wide resident on the GPU
 cudaError_t launch_level_poly(const LevelArgs& a, int check_only, cudaStream_t s);

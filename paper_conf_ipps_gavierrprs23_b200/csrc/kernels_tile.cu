@@ -1,25 +1,32 @@
 // kernels_tile.cu — kernel T dispatch: plan-time setup and launch by tile width (the
 // template instantiations live in kernels_tile_tw{4,8,16,32,64}.cu).
+#include <algorithm>
+
 #include "kernels_tile.cuh"
 
 namespace gs {
 
-static size_t lvl_bytes(uint32_t n_levels) { return (((size_t)n_levels + 1) * 4 + 15) / 16 * 16; }
+void tile_steps(const uint32_t* level_off, uint32_t n_levels, uint32_t chunk, std::vector<uint2>& out) {
+    out.clear();
+    for (uint32_t l = 0; l < n_levels; ++l)
+        for (uint32_t g = level_off[l]; g < level_off[l + 1];) {
+            const uint32_t n = chunk ? std::min(chunk, level_off[l + 1] - g) : level_off[l + 1] - g;
+            out.push_back(make_uint2(g, n));
+            g += n;
+        }
+}
 
-size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
-                       int desc_mode, uint32_t max_width) {
-    size_t b = 0, g = ((size_t)n_slots + 64) * 4 * tw;
-    if (desc_mode == 1) b = (size_t)n_eval * 16 + lvl_bytes(n_levels);
-    if (desc_mode == 2) {
-        b = lvl_bytes(n_levels);
-        g += 16 + 2 * (size_t)max_width * 16;
-    }
+size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_steps,
+                       int desc_mode) {
+    size_t b = ((size_t)n_steps + 1) / 2 * 16;
+    if (desc_mode == 1) b += (size_t)n_eval * 16;
+    const size_t g = 32 + (desc_mode == 2 ? 2 * (size_t)TILE_CHUNK * 16 : 0) + ((size_t)n_slots + 64) * 4 * tw;
     return b + (size_t)ng * g;
 }
 
-cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_levels,
-                       int desc_smem, uint32_t max_width, uint32_t has_q, uint32_t* per_sm) {
-    const size_t smem = tile_smem_bytes(tw, ng, n_slots, n_eval, n_levels, desc_smem, max_width);
+cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_steps,
+                       int desc_smem, uint32_t has_q, uint32_t* per_sm) {
+    const size_t smem = tile_smem_bytes(tw, ng, n_slots, n_eval, n_steps, desc_smem);
     int per = 0;
     cudaError_t e;
     switch (tw) {
@@ -36,7 +43,9 @@ cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_ev
 
 cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s) {
     if (a.n_tiles == 0 || a.ncycles == 0) return cudaSuccess;
-    const size_t smem = tile_smem_bytes(tw, ng, a.n_slots, a.n_eval, a.n_levels, a.desc_smem, a.max_width);
+    const size_t smem = tile_smem_bytes(tw, ng, a.n_slots, a.n_eval, a.n_steps, a.desc_smem);
+    cudaError_t e = cudaMemsetAsync(a.tile_next, 0, sizeof(unsigned int), s);   // empty the tile queue
+    if (e != cudaSuccess) return e;
     switch (tw) {
         case 4: return launch_tile_tw<4>(a, ng, grid, smem, s);
         case 8: return launch_tile_tw<8>(a, ng, grid, smem, s);

@@ -30,12 +30,8 @@ constexpr uint32_t TILE_CTA = 512;                   // threads per CTA (one CTA
 #endif
 constexpr uint32_t TILE_VPT = GS_TILE_VPT;          // 16-byte vectors per thread and gate (TW >= 16)
 constexpr unsigned long long TILE_MISR_POLY = 0x42F0E1EBA9EA3693ULL;   // CRC-64/ECMA-182
+constexpr uint32_t TILE_CHUNK = GS_TILE_CHUNK;      // TMA-streamed descriptors per step (max)
 
-// Shared memory by descriptor mode:
-//   1 (resident): [desc: 16 B x n_eval] [level_off: 4 B x (n_levels + 1), padded to 16 B]
-//   2 (TMA-streamed): [level_off] then per group [2 mbarriers, 16 B][2 x max_width x 16 B]
-//   0 (global): nothing
-// then per thread group: [slots: n_slots x TW words] [MISR: 64 x TW words].
 // ---- TMA bulk copy (cp.async.bulk) of a level's descriptors into shared memory, completion
 // signalled on an mbarrier (expect_tx / complete_tx), consumers wait on the phase parity
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -137,54 +133,67 @@ __device__ __forceinline__ void group_sync(uint32_t id, uint32_t nthreads) {
 
 // TW = 32-bit words per slot (tile = 32 * TW lanes).  A thread evaluates one gate on P
 // 16-byte groups of 4 words (128 lanes each; P = TILE_VPT when TW >= 16): P*k 16-byte
-// shared-memory loads, P*4*(2^k - 1) LOP3, P 16-byte stores.  The CTA (TILE_CTA threads) is split into NG independent groups; each
-// group simulates its own tile and synchronises only with itself (named barrier 1 + gid),
-// so one group's level barrier overlaps the other groups' work.  All groups share the
-// descriptor table in shared memory.
+// shared-memory loads, P*4*(2^k - 1) LOP3, P 16-byte stores.  The CTA (TILE_CTA threads) is
+// split into NG independent groups; each group simulates its own tile and synchronises only
+// with itself (named barrier 1 + gid), so one group's level barrier overlaps the other
+// groups' work.  Tiles are handed out by an atomic queue (Ctl::tile_next), one per group at a
+// time.
+//
+// The level loop walks a per-program STEP table in shared memory: one step per non-empty
+// level (resident descriptors), or per chunk of at most TILE_CHUNK gates of a level
+// (TMA-streamed descriptors: chunk t+1 is copied into the other half of a fixed double
+// buffer while chunk t is evaluated).  Every step ends with the group barrier.  Everything
+// loop-invariant (Ctl fields, shared-memory addresses) is read once per launch, so a step
+// costs a handful of instructions besides its gates.
 template <int TW, bool HASQ, int NG, int DM>
 __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
-    // DM: descriptor mode (0 global, 1 resident, 2 TMA)
+    // DM: descriptor mode (0 global, 1 resident, 2 TMA-streamed chunks)
     constexpr uint32_t V = TW / 4;                       // uint4 per slot
     constexpr uint32_t P = V >= 4 ? TILE_VPT : 1;        // 16-byte vectors per thread and gate
     constexpr uint32_t VS = V / P;                       // threads per gate (vector stride)
+    constexpr uint32_t VSH = VS == 1 ? 0 : VS == 2 ? 1 : VS == 4 ? 2 : VS == 8 ? 3 : 4;
+    static_assert((1u << VSH) == VS, "VS must be a power of two <= 16");
     constexpr uint32_t GT = TILE_CTA / NG;               // threads per group
     extern __shared__ uint4 smem[];
-    const uint4* dsm = DM == 1 ? smem : reinterpret_cast<const uint4*>(a.desc);
-    const uint32_t* lvl = a.level_off;
+    // ---- shared layout: [resident descriptors (DM 1)] [steps: uint2 x n_steps, padded]
+    //      then per group: [2 mbarriers (16 B)] [tile id (16 B)] [2 x TILE_CHUNK descriptors
+    //                      (DM 2)] [slots: n_slots x V uint4] [MISR: 64 x V uint4]
     uint4* base = smem;
     if (DM == 1) {
-        uint32_t* lv = reinterpret_cast<uint32_t*>(smem + a.n_eval);
         const uint4* gd = reinterpret_cast<const uint4*>(a.desc);
         for (uint32_t i = threadIdx.x; i < a.n_eval; i += blockDim.x) smem[i] = __ldg(gd + i);
-        for (uint32_t i = threadIdx.x; i <= a.n_levels; i += blockDim.x) lv[i] = __ldg(a.level_off + i);
-        lvl = lv;
-        base = smem + a.n_eval + ((a.n_levels + 1) * 4 + 15) / 16;
-    } else if (DM == 2) {
-        uint32_t* lv = reinterpret_cast<uint32_t*>(smem);
-        for (uint32_t i = threadIdx.x; i <= a.n_levels; i += blockDim.x) lv[i] = __ldg(a.level_off + i);
-        lvl = lv;
-        base = smem + ((a.n_levels + 1) * 4 + 15) / 16;
+        base += a.n_eval;
     }
-    const uint32_t gid = threadIdx.x / GT, tid = threadIdx.x % GT, bd = GT;
+    uint2* steps = reinterpret_cast<uint2*>(base);
+    for (uint32_t i = threadIdx.x; i < a.n_steps; i += blockDim.x) steps[i] = __ldg(a.steps + i);
+    base += (a.n_steps + 1) / 2;
+    const uint32_t gid = threadIdx.x / GT, tid = threadIdx.x % GT;
     const uint32_t bar = 1 + gid;
-    // group region: [mbarriers + descriptor double buffer (mode 2)] [slots] [MISR]
-    uint4* greg = base + (size_t)gid * ((a.n_slots + 64) * V + (DM == 2 ? 1 + 2 * a.max_width : 0));
+    uint4* greg = base + (size_t)gid * (2 + (DM == 2 ? 2 * TILE_CHUNK : 0) + (a.n_slots + 64) * V);
     uint64_t* mbar = reinterpret_cast<uint64_t*>(greg);
-    uint4* dbuf = greg + 1;                                   // [2][max_width]
-    uint4* gsm = DM == 2 ? greg + 1 + 2 * a.max_width : greg;
-    uint4* sl = gsm;
+    volatile uint32_t* tile_slot = reinterpret_cast<volatile uint32_t*>(greg + 1);
+    uint4* dbuf = greg + 2;                                   // DM 2: [2][TILE_CHUNK]
+    uint4* sl = greg + 2 + (DM == 2 ? 2 * TILE_CHUNK : 0);    // slots
+    const uint4* dsm = DM == 1 ? smem : reinterpret_cast<const uint4*>(a.desc);
     if (DM == 2 && tid == 0) {
         mbar_init(mbar, 1);
         mbar_init(mbar + 1, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
-    const uint32_t mbar_s = smem_u32(mbar);                   // mode 2: the two mbarriers (8 B apart)
-    const uint32_t dbuf_s = smem_u32(dbuf);                   // mode 2: descriptor double buffer
+    const uint32_t mbar_s = smem_u32(mbar);
+    const uint32_t dbuf_s = smem_u32(dbuf);
     uint32_t* sw = reinterpret_cast<uint32_t*>(sl);          // slots as 32-bit words
     uint32_t* mp = sw + (size_t)a.n_slots * TW;              // MISR planes [64][TW]
+    // loop-invariant control state, read once
     const unsigned long long c0 = a.ctl->cycle;
-    const uint32_t R = a.n_reg, q0 = a.q0;
+    const unsigned long long seed = a.ctl->seed;
+    const uint32_t stim_mode = a.ctl->stim_mode;
+    const unsigned long long* stim_src = reinterpret_cast<const unsigned long long*>(a.ctl->stim_ptr);
+    const unsigned long long stim_base = a.ctl->stim_base;
+    const unsigned long long sink_ptr = a.ctl->sink_ptr, sink_base = a.ctl->sink_base,
+                             sink_cycles = a.ctl->sink_cycles;
+    const uint32_t R = a.n_reg, q0 = a.q0, n_steps = a.n_steps;
     const uint32_t w32_row = a.words * 2;                     // 32-bit words per state row
     const uint32_t* st32 = reinterpret_cast<const uint32_t*>(a.state);
     uint32_t* st32w = reinterpret_cast<uint32_t*>(a.state);
@@ -193,143 +202,150 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     const uint32_t* misr_in = reinterpret_cast<const uint32_t*>(a.misr + (size_t)(c0 & 1) * 64 * a.words);
     uint32_t* misr_out = reinterpret_cast<uint32_t*>(a.misr + (size_t)((c0 + a.ncycles) & 1) * 64 * a.words);
     unsigned long long pop = 0;
-    // mode 2: the group's descriptor stream, one level per step, double-buffered: while
-    // level l is evaluated from buffer (step & 1), the TMA engine fetches the next level
-    // (the same sequence repeats every cycle and every tile)
-    uint32_t step = 0;
-    if (DM == 2 && tid == 0 && blockIdx.x * NG + gid < a.n_tiles)
-        tma_load_1d(dbuf_s, a.desc + lvl[0], (lvl[1] - lvl[0]) * 16, mbar_s);
+    uint32_t step = 0;                                        // DM 2: chunks consumed by this group
 
-    for (uint32_t tile = blockIdx.x * NG + gid; tile < a.n_tiles; tile += gridDim.x * NG) {
-        const bool last_tile = tile + gridDim.x * NG >= a.n_tiles;
+    // first tile of the group (the queue is zeroed before every launch)
+    if (tid == 0) *tile_slot = atomicAdd(a.tile_next, 1u);
+    group_sync(bar, GT);
+    uint32_t tile = *tile_slot;
+    if (DM == 2 && tid == 0 && tile < a.n_tiles && n_steps) {
+        const uint2 s0 = steps[0];
+        tma_load_1d(dbuf_s, a.desc + s0.x, s0.y * 16, mbar_s);
+    }
+    while (tile < a.n_tiles) {
+        // claim the next tile now, so the descriptor stream knows whether to continue
+        if (tid == 0) *tile_slot = atomicAdd(a.tile_next, 1u);
         const uint32_t t0 = tile * TW;                    // first 32-bit word of the tile (shard-local)
         // ---- load: constants, both register banks, MISR planes
-        for (uint32_t u = tid; u < TW; u += bd) {
+        for (uint32_t u = tid; u < TW; u += GT) {
             sw[u] = 0u;
             sw[TW + u] = 0xFFFFFFFFu;
         }
         // register slots: bank 0 always holds the CURRENT Q (state bank c0 & 1), bank 1 the
         // next one; inputs never resolve banks — bank 1 is copied into bank 0 after each cycle
-        for (uint32_t u = tid; u < 2 * R * TW; u += bd) {
+        for (uint32_t u = tid; u < 2 * R * TW; u += GT) {
             const uint32_t r = u / TW, w = u % TW;
             const uint32_t sb = (r < R ? (uint32_t)(c0 & 1) : (uint32_t)((c0 + 1) & 1)) * R + (r < R ? r : r - R);
             sw[(size_t)(q0 + r) * TW + w] = st32[(uint64_t)(a.row_q0 + sb) * w32_row + t0 + w];
         }
-        for (uint32_t u = tid; u < 64 * TW; u += bd) {
+        for (uint32_t u = tid; u < 64 * TW; u += GT) {
             const uint32_t j = u / TW, w = u % TW;
             mp[u] = misr_in[(uint64_t)j * w32_row + t0 + w];
         }
         group_sync(bar, GT);
+        const uint32_t next_tile = *tile_slot;           // (written before the barrier above)
         for (uint32_t c = 0; c < a.ncycles; ++c) {
             const unsigned long long cyc = c0 + c;
-            const uint32_t qnext = R;
             // ---- primary inputs of this cycle (R2): one 64-bit hash per pair of words
-            for (uint32_t u = tid; u < a.n_pi * (TW / 2); u += bd) {
+            for (uint32_t u = tid; u < a.n_pi * (TW / 2); u += GT) {
                 const uint32_t p = u / (TW / 2), w2 = u % (TW / 2);
                 const uint32_t g64 = (t0 >> 1) + w2;      // shard-local 64-bit word
-                unsigned long long v;
-                if (a.ctl->stim_mode == 0) {
-                    v = dmix64(dmix64(dmix64(a.ctl->seed ^ p) ^ cyc) ^ (a.word_off + g64));
-                } else {
-                    const unsigned long long* src = reinterpret_cast<const unsigned long long*>(a.ctl->stim_ptr);
-                    v = src[((cyc - a.ctl->stim_base) * a.n_pi + p) * a.words + g64];
-                }
+                const unsigned long long v =
+                    stim_mode == 0 ? dmix64(dmix64(dmix64(seed ^ p) ^ cyc) ^ (a.word_off + g64))
+                                   : stim_src[((cyc - stim_base) * a.n_pi + p) * a.words + g64];
                 reinterpret_cast<unsigned long long*>(sw + (size_t)(2 + p) * TW)[w2] = v;
             }
             group_sync(bar, GT);
-            // ---- levels: every (gate, 16-byte group) unit of the level, then a barrier
-            for (uint32_t l = 0; l < a.n_levels; ++l) {
-                const uint32_t g0 = lvl[l], n = (lvl[l + 1] - g0) * VS;
-                const uint4* dl = dsm + g0;
+            // ---- steps: every (gate, vector group) unit of the step, then the group barrier
+            const bool more = c + 1 < a.ncycles || next_tile < a.n_tiles;   // stream continues
+#pragma unroll 1
+            for (uint32_t si = 0; si < n_steps; ++si) {
+                const uint2 st = steps[si];
+                const uint4* dl = dsm + st.x;
                 if (DM == 2) {
                     const uint32_t b = step & 1;
-                    if (tid == 0 && !(last_tile && c + 1 == a.ncycles && l + 1 == a.n_levels)) {
-                        const uint32_t ln = l + 1 == a.n_levels ? 0 : l + 1;
-                        tma_load_1d(dbuf_s + (b ^ 1) * a.max_width * 16, a.desc + lvl[ln],
-                                    (lvl[ln + 1] - lvl[ln]) * 16, mbar_s + 8 * (b ^ 1));
+                    if (tid == 0 && (si + 1 < n_steps || more)) {
+                        const uint2 sn = steps[si + 1 < n_steps ? si + 1 : 0];
+                        tma_load_1d(dbuf_s + (b ^ 1) * (TILE_CHUNK * 16), a.desc + sn.x, sn.y * 16,
+                                    mbar_s + 8 * (b ^ 1));
                     }
                     mbar_wait(mbar_s + 8 * b, (step >> 1) & 1);
-                    dl = dbuf + b * a.max_width;
+                    dl = dbuf + b * TILE_CHUNK;
                     ++step;
                 }
-                for (uint32_t u = tid; u < n; u += bd) {
-                    const uint32_t gi = u / VS, v = u % VS;
-                    const uint32_t g = g0 + gi;
+                const uint32_t n = st.y << VSH;
+#pragma unroll 1
+                for (uint32_t u = tid; u < n; u += GT) {
+                    const uint32_t gi = u >> VSH, v = u & (VS - 1);
+                    const uint32_t g = st.x + gi;
                     const uint4 d = dl[gi];
                     // k: warp-uniform except at k-group edges; the common 2-4-input gates are
                     // tested first (a compare and branch each instead of the jump table)
                     const uint32_t k = d.w & 15u;
-                    if (k == 2) tile_gate<2, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext);
-                    else if (k == 3) tile_gate<3, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext);
-                    else if (k == 4) tile_gate<4, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext);
+                    if (k == 2) tile_gate<2, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R);
+                    else if (k == 3) tile_gate<3, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R);
+                    else if (k == 4) tile_gate<4, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R);
                     else switch (k) {
-                        case 1: tile_gate<1, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext); break;
-                        case 5: tile_gate<5, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext); break;
-                        case 6: tile_gate<6, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext); break;
-                        case 7: tile_gate<7, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext); break;
-                        default: tile_gate<8, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, qnext); break;
+                        case 1: tile_gate<1, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R); break;
+                        case 5: tile_gate<5, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R); break;
+                        case 6: tile_gate<6, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R); break;
+                        case 7: tile_gate<7, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R); break;
+                        default: tile_gate<8, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R); break;
                     }
                 }
                 group_sync(bar, GT);
             }
             // ---- leftover latches into the next bank; MISR / popcount / trace of the POs
-            for (uint32_t u = tid; u < a.n_latch * V; u += bd) {
+            for (uint32_t u = tid; u < a.n_latch * V; u += GT) {
                 const uint32_t e = u / V, v = u % V;
                 const uint32_t s = __ldg(a.latch_src + e);
-                sl[(size_t)(q0 + __ldg(a.latch_dst + e) + qnext) * V + v] = sl[(size_t)s * V + v];
+                sl[(size_t)(q0 + __ldg(a.latch_dst + e) + R) * V + v] = sl[(size_t)s * V + v];
             }
             constexpr uint32_t NP = (64 * TW + GT - 1) / GT;    // MISR plane words per thread
             uint32_t newp[NP];
             const bool tr = a.trace && cyc < a.trace_cap;
+            // full per-cycle output stream: a boolean, never a null pointer plus an offset
+            const bool to_sink = sink_ptr && cyc - sink_base < sink_cycles;
+            uint32_t* sink = reinterpret_cast<uint32_t*>(sink_ptr) +
+                             (to_sink ? (cyc - sink_base) * a.n_po * (uint64_t)w32_row : 0ull);
 #pragma unroll
             for (uint32_t i = 0; i < NP; ++i) {
-                const uint32_t u = tid + i * bd;
-                if (u >= 64 * TW) break;
-                const uint32_t j = u / TW, w = u % TW;
-                const uint32_t g32 = t0 + w;
-                const int32_t tslot = tr ? __ldg(a.trace_slot + (g32 >> 1)) : -1;
-                // full per-cycle output stream: a boolean, never a null pointer plus an offset
-                const bool to_sink = a.ctl->sink_ptr && cyc - a.ctl->sink_base < a.ctl->sink_cycles;
-                uint32_t* sink = reinterpret_cast<uint32_t*>(a.ctl->sink_ptr) +
-                                 (to_sink ? (cyc - a.ctl->sink_base) * a.n_po * (uint64_t)w32_row : 0ull);
-                uint32_t vv = 0;
-                for (uint32_t o = j; o < a.n_po; o += 64) {
-                    const uint32_t x = sw[(size_t)__ldg(a.po_slot + o) * TW + w];
-                    vv ^= x;
-                    pop += __popc(x);
-                    if (tslot >= 0)
-                        reinterpret_cast<uint32_t*>(a.trace)[(((uint64_t)cyc * a.n_po + o) * a.ntw + tslot) * 2 +
-                                                             (g32 & 1)] = x;
-                    if (to_sink) sink[(uint64_t)o * w32_row + g32] = x;
+                const uint32_t u = tid + i * GT;
+                newp[i] = 0u;
+                if (u < 64 * TW) {
+                    const uint32_t j = u / TW, w = u % TW;
+                    const uint32_t g32 = t0 + w;
+                    const int32_t tslot = tr ? __ldg(a.trace_slot + (g32 >> 1)) : -1;
+                    uint32_t vv = 0;
+                    for (uint32_t o = j; o < a.n_po; o += 64) {
+                        const uint32_t x = sw[(size_t)__ldg(a.po_slot + o) * TW + w];
+                        vv ^= x;
+                        pop += __popc(x);
+                        if (tslot >= 0)
+                            reinterpret_cast<uint32_t*>(a.trace)[(((uint64_t)cyc * a.n_po + o) * a.ntw + tslot) * 2 +
+                                                                 (g32 & 1)] = x;
+                        if (to_sink) sink[(uint64_t)o * w32_row + g32] = x;
+                    }
+                    const uint32_t prev = j ? mp[(j - 1) * TW + w] : 0u;
+                    const uint32_t fb = ((TILE_MISR_POLY >> j) & 1ULL) ? mp[63 * TW + w] : 0u;
+                    newp[i] = prev ^ fb ^ vv;
                 }
-                const uint32_t prev = j ? mp[(j - 1) * TW + w] : 0u;
-                const uint32_t fb = ((TILE_MISR_POLY >> j) & 1ULL) ? mp[63 * TW + w] : 0u;
-                newp[i] = prev ^ fb ^ vv;
             }
             group_sync(bar, GT);
 #pragma unroll
             for (uint32_t i = 0; i < NP; ++i)
-                if (tid + i * bd < 64 * TW) mp[tid + i * bd] = newp[i];
+                if (tid + i * GT < 64 * TW) mp[tid + i * GT] = newp[i];
             if (HASQ && c + 1 < a.ncycles)                    // the clock edge: Q := next Q
-                for (uint32_t u = tid; u < R * V; u += bd) sl[(size_t)q0 * V + u] = sl[(size_t)(q0 + R) * V + u];
+                for (uint32_t u = tid; u < R * V; u += GT) sl[(size_t)q0 * V + u] = sl[(size_t)(q0 + R) * V + u];
             group_sync(bar, GT);
         }
         // ---- write back: Q of the last cycle (bank 0) to state bank (last & 1), the latched
         // next Q (bank 1) to the other bank; PO rows (read_outputs); MISR planes
         const uint32_t lastp = (uint32_t)((c0 + a.ncycles - 1) & 1);
-        for (uint32_t u = tid; u < 2 * R * TW; u += bd) {
+        for (uint32_t u = tid; u < 2 * R * TW; u += GT) {
             const uint32_t r = u / TW, w = u % TW;
             const uint32_t sb = (r < R ? lastp : lastp ^ 1u) * R + (r < R ? r : r - R);
             st32w[(uint64_t)(a.row_q0 + sb) * w32_row + t0 + w] = sw[(size_t)(q0 + r) * TW + w];
         }
-        for (uint32_t u = tid; u < a.n_wb * TW; u += bd) {
+        for (uint32_t u = tid; u < a.n_wb * TW; u += GT) {
             const uint32_t e = u / TW, w = u % TW;
             st32w[(uint64_t)__ldg(a.wb_row + e) * w32_row + t0 + w] = sw[(size_t)__ldg(a.wb_slot + e) * TW + w];
         }
-        for (uint32_t u = tid; u < 64 * TW; u += bd) {
+        for (uint32_t u = tid; u < 64 * TW; u += GT) {
             const uint32_t j = u / TW, w = u % TW;
             misr_out[(uint64_t)j * w32_row + t0 + w] = mp[u];
         }
+        tile = next_tile;
         group_sync(bar, GT);                              // before the next tile reuses smem
     }
     // ---- counters; the last CTA advances the device clock

@@ -24,7 +24,7 @@ size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 struct Layout {
     size_t ctl, state, din, aux, dhi, dtt, term_off, terms, po_rows, latch_src, latch_dst, reg_init,
         trace_slot, misr, trace, lane_sigs, scratch, t_desc, t_desc_hi, t_po, t_lsrc, t_ldst, t_wbrow,
-        t_wbslot, t_lvl, total;
+        t_wbslot, t_steps, total;
 };
 
 struct Plans {
@@ -32,25 +32,27 @@ struct Plans {
     uint32_t tw = 0;                  // kernel T: 32-bit words per slot
     uint32_t ng = 0;                  // kernel T: thread groups (tiles) per CTA
     int desc_smem = 0;                // kernel T: descriptors 0 global, 1 resident, 2 TMA-streamed
-    uint32_t max_width = 0;           // kernel T: widest level
+    std::vector<uint2> steps;         // kernel T: level steps (chunks when TMA-streamed)
 };
 
 constexpr size_t TILE_SMEM_MAX = 232448;   // 227 KB opt-in shared memory per CTA (sm_100a)
 
 gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
+    if (o.kernel == GS_KERNEL_CLUSTER) {
+        const uint64_t sl = o.slab_lanes ? o.slab_lanes : 256;
+        if (sl % 128 || o.lanes % sl)
+            return fail(GS_ERR_ARG, "CLUSTER: slab_lanes must be a multiple of 128 dividing lanes");
+        const uint32_t cs = o.cluster_size ? o.cluster_size : 2;
+        if (cs != 1 && cs != 2 && cs != 4 && cs != 8 && cs != 16)
+            return fail(GS_ERR_ARG, "CLUSTER: cluster_size must be 1, 2, 4, 8 or 16");
+        tile_steps(p.level_off.data(), p.n_levels, 0, pl.steps);
+        return GS_OK;
+    }
     if (o.kernel != GS_KERNEL_TILE) return GS_OK;
     if (gs_status st = tile_plan(p, pl.tile)) return st;
-    uint32_t maxw = 0;
-    bool empty_level = false;
-    for (uint32_t l = 0; l < p.n_levels; ++l) {
-        maxw = std::max(maxw, p.level_off[l + 1] - p.level_off[l]);
-        empty_level = empty_level || p.level_off[l + 1] == p.level_off[l];
-    }
-    pl.max_width = maxw;
-    auto smem = [&](uint32_t tw, uint32_t ng, int ds) {
-        if (ds == 2 && empty_level) return (size_t)-1;             // TMA stream needs non-empty levels
-        return tile_smem_bytes(tw, ng, pl.tile.n_slots, p.n_eval, p.n_levels, ds, maxw);
-    };
+    std::vector<uint2> st_level, st_chunk;
+    tile_steps(p.level_off.data(), p.n_levels, 0, st_level);
+    tile_steps(p.level_off.data(), p.n_levels, GS_TILE_CHUNK, st_chunk);
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, o.device);
     if (o.tile_words && (o.tile_words != 4 && o.tile_words != 8 && o.tile_words != 16 && o.tile_words != 32 &&
@@ -60,30 +62,38 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
         return fail(GS_ERR_ARG, "TILE: tile_groups must be 1, 2 or 4");
     if (o.tile_words && o.lanes % (32ull * o.tile_words))
         return fail(GS_ERR_ARG, "TILE: lanes must be a multiple of 32 * tile_words");
-    // choose (descriptor mode, tile words, groups per CTA): the most lanes in flight on the
-    // GPU (groups x tile lanes x SMs, capped by the batch), counting a resident descriptor
-    // table as worth 2x the lanes (measured: C2 runs 1.08x faster with one group and a
-    // resident table than with two groups and TMA-streamed descriptors, while a 10k-gate
-    // circuit runs 1.33x faster with TMA and 4x wider tiles than resident with narrow
-    // ones), then wider tiles, then resident > TMA stream > global, then fewer groups
+    // choose (descriptor mode, tile words, groups per CTA).  Kernel T is latency-bound per
+    // tile (a level barrier per step), so a launch takes ~ waves x tile time with waves =
+    // ceil(tiles / (groups x SMs)): score = lanes per wave (quantisation included), resident
+    // descriptors weighted 4/3, then wider tiles, then resident > TMA stream > global, then
+    // more groups.  C2 (256 live slots): 2 groups x 2,048-lane tiles, TMA stream, 3.0e13 vs
+    // 2.56e13 for 1 group with resident descriptors (profiles/r02_kernelT_configs_C2.txt)
     const int forced = (o.flags & GS_SIM_TILE_DESC_GLOBAL) ? 0 : (o.flags & GS_SIM_TILE_DESC_TMA) ? 2 : -1;
     uint64_t best = 0;
     for (int ds : {1, 2, 0}) {
         if (forced >= 0 && ds != forced) continue;
+        const uint32_t nsteps = (uint32_t)(ds == 2 ? st_chunk.size() : st_level.size());
         for (uint32_t ng : {4u, 2u, 1u}) {
             if (o.tile_groups && ng != o.tile_groups) continue;
             for (uint32_t tw : {4u, 8u, 16u, 32u, 64u}) {
                 if (o.tile_words && tw != o.tile_words) continue;
-                if (o.lanes % (32ull * tw) || smem(tw, ng, ds) > TILE_SMEM_MAX) continue;
-                const uint64_t inflight = std::min<uint64_t>((uint64_t)ng * tw * 32 * sms, o.lanes);
+                if (o.lanes % (32ull * tw)) continue;
+                if (tile_smem_bytes(tw, ng, pl.tile.n_slots, p.n_eval, nsteps, ds) > TILE_SMEM_MAX) continue;
+                const uint64_t tiles = o.lanes / (32ull * tw);
+                const uint64_t slots = (uint64_t)ng * (uint64_t)sms;
+                const uint64_t waves = (tiles + slots - 1) / slots;
+                const uint64_t per_wave = o.lanes / waves;
                 const uint64_t pref = ds == 1 ? 2 : ds == 2 ? 1 : 0;
-                const uint64_t score = ((inflight << (ds == 1 ? 1 : 0)) << 24) | ((uint64_t)tw << 16) | (pref << 12) |
-                                       ((8 - ng) << 8);
+                // resident descriptors counted 4/3 (no per-step TMA wait): measured on C2 at
+                // 2,048-lane tiles, resident 2.56e13 vs TMA-streamed 1.92e13
+                const uint64_t score = ((per_wave * (ds == 1 ? 4 : 3)) << 24) | ((uint64_t)tw << 16) |
+                                       (pref << 12) | ((uint64_t)ng << 8);
                 if (score > best) { best = score; pl.tw = tw; pl.ng = ng; pl.desc_smem = ds; }
             }
         }
     }
     if (!best) return fail(GS_ERR_ARG, "TILE: live state of a 128-lane tile exceeds shared memory (or lanes % 128)");
+    pl.steps = pl.desc_smem == 2 ? st_chunk : st_level;
     return GS_OK;
 }
 
@@ -148,7 +158,7 @@ Layout make_layout(const Program& p, const gs_sim_opts& o, const Plans& pl) {
     L.t_ldst = take(t.latch_dst.size() * 4);
     L.t_wbrow = take(t.wb_row.size() * 4);
     L.t_wbslot = take(t.wb_slot.size() * 4);
-    L.t_lvl = take(pl.tw ? p.level_off.size() * 4 : 0);
+    L.t_steps = take(pl.steps.size() * sizeof(uint2));
     L.total = off;
     return L;
 }
@@ -181,7 +191,7 @@ struct gs_sim {
     uint32_t tw = 0, tile_grid = 0;
     int desc_smem = 0;
     uint32_t tile_groups = 1;
-    uint32_t tile_max_width = 0;
+    std::vector<uint2> tile_steps;    // kernel T: level steps (uploaded to L.t_steps)
     uint32_t pdl = 1;                 // programmatic dependent launch between cycle kernels
     uint32_t min_warps = 0;           // kernel A auto-U threshold (2 waves of resident warps)
     uint32_t resident_blocks = 0;     // kernel A wide path: CTAs resident on the GPU
@@ -190,6 +200,7 @@ struct gs_sim {
     std::vector<cudaStream_t> gstream;  // [groups - 1] branch streams (group 0: the caller's)
     std::vector<cudaEvent_t> gev;       // [0] fork, [1 .. groups - 1] joins
     uint64_t grid_stride_launches = 0;  // level launches whose grid was capped at residency
+    uint32_t cluster_size = 0, clusters = 0, slab_vec = 0, n_slabs = 0;   // kernel C
 
     Ctl* ctl() const { return reinterpret_cast<Ctl*>(ws + L.ctl); }
     uint8_t* state() const { return ws + L.state; }
@@ -281,11 +292,10 @@ static cudaError_t tile_launch(const gs_sim* s, uint32_t ncycles, cudaStream_t s
     TileArgs a{};
     a.desc = s->at<const TileDesc>(s->L.t_desc);
     a.desc_hi = s->at<const uint4>(s->L.t_desc_hi);
-    a.level_off = s->at<const uint32_t>(s->L.t_lvl);
+    a.steps = s->at<const uint2>(s->L.t_steps);
     a.n_eval = p.n_eval;
-    a.n_levels = p.n_levels;
+    a.n_steps = (uint32_t)s->tile_steps.size();
     a.desc_smem = (uint32_t)s->desc_smem;
-    a.max_width = s->tile_max_width;
     a.po_slot = s->at<const uint32_t>(s->L.t_po);
     a.n_po = p.n_po;
     a.latch_src = s->at<const uint32_t>(s->L.t_lsrc);
@@ -302,6 +312,7 @@ static cudaError_t tile_launch(const gs_sim* s, uint32_t ncycles, cudaStream_t s
     a.words = s->words;
     a.row_q0 = p.row_q0;
     a.ctl = s->ctl();
+    a.tile_next = &s->ctl()->tile_next;
     a.misr = s->at<unsigned long long>(s->L.misr);
     a.trace_slot = s->at<const int32_t>(s->L.trace_slot);
     a.trace = (s->opts.n_trace_words && s->opts.trace_cycles) ? s->at<unsigned long long>(s->L.trace) : nullptr;
@@ -311,6 +322,42 @@ static cudaError_t tile_launch(const gs_sim* s, uint32_t ncycles, cudaStream_t s
     a.ncycles = ncycles;
     a.n_tiles = (uint32_t)(s->opts.lanes / (32ull * s->tw));
     return launch_tile(a, s->tw, s->tile_groups, s->tile_grid, st);
+}
+
+static cudaError_t cluster_launch(const gs_sim* s, uint32_t ncycles, cudaStream_t st) {
+    const Program& p = *s->prog;
+    ClusterArgs a{};
+    a.din = s->at<const uint4>(s->L.din);
+    a.aux = s->at<const GateAux>(s->L.aux);
+    a.dhi = p.any_wide ? s->at<const uint4>(s->L.dhi) : nullptr;
+    a.dtt = p.max_k > GS_MAX_K_LUT64 ? s->at<const uint4>(s->L.dtt) : nullptr;
+    a.steps = s->at<const uint2>(s->L.t_steps);
+    a.n_steps = (uint32_t)s->tile_steps.size();
+    a.state = s->state();
+    a.stride = s->stride;
+    a.words = s->words;
+    a.row_gate0 = p.row_gate0;
+    a.row_pi0 = p.row_pi0;
+    a.n_pi = p.n_pi;
+    a.row_q0 = p.row_q0;
+    a.n_reg = p.n_reg;
+    a.latch_src = s->at<const uint32_t>(s->L.latch_src);
+    a.latch_dst = s->at<const uint32_t>(s->L.latch_dst);
+    a.n_latch = (uint32_t)p.latch_src.size();
+    a.po_rows = s->at<const uint32_t>(s->L.po_rows);
+    a.n_po = p.n_po;
+    a.misr = s->at<unsigned long long>(s->L.misr);
+    a.trace_slot = s->at<const int32_t>(s->L.trace_slot);
+    a.trace = (s->opts.n_trace_words && s->opts.trace_cycles) ? s->at<unsigned long long>(s->L.trace) : nullptr;
+    a.ntw = s->opts.n_trace_words;
+    a.trace_cap = s->opts.trace_cycles;
+    a.ctl = s->ctl();
+    a.tile_next = &s->ctl()->tile_next;
+    a.word_off = s->opts.lane_offset / 64;
+    a.ncycles = ncycles;
+    a.slab_vec = s->slab_vec;
+    a.n_slabs = s->n_slabs;
+    return launch_cluster(a, s->clusters, s->cluster_size, st);
 }
 
 // evs (profiling): timing events around every level launch (one group), or around the
@@ -434,7 +481,7 @@ static gs_status check_opts(const gs_sim_opts* o, const char* fn) {
     if (o->lanes == 0 || o->lanes % 64) return fail(GS_ERR_ARG, std::string(fn) + ": lanes must be a positive multiple of 64");
     if (o->lanes / 64 >= (1ull << 31)) return fail(GS_ERR_ARG, std::string(fn) + ": too many lanes");
     if (o->lane_offset % 64) return fail(GS_ERR_ARG, std::string(fn) + ": lane_offset must be a multiple of 64");
-    if (o->kernel < GS_KERNEL_AUTO || o->kernel > GS_KERNEL_TILE || o->kernel == 4)
+    if (o->kernel < GS_KERNEL_AUTO || o->kernel > GS_KERNEL_CLUSTER || o->kernel == 4)
         return fail(GS_ERR_ARG, std::string(fn) + ": bad kernel");
     if (o->flags & GS_SIM_RETIRED_FLAGS)
         return fail(GS_ERR_ARG, std::string(fn) + ": flag retired in 0.2.0 (L2 hints / bulk gathers / global T slots)");
@@ -500,7 +547,7 @@ static gs_status sim_create(const gs_program* prog, const gs_sim_opts* opts_in, 
     s->tile = pls.tile;
     s->tw = pls.tw;
     s->desc_smem = pls.desc_smem;
-    s->tile_max_width = pls.max_width;
+    s->tile_steps = pls.steps;
     s->pdl = (opts->flags & GS_SIM_NO_PDL) ? 0u : 1u;
     s->groups = groups;
     {
@@ -514,13 +561,26 @@ static gs_status sim_create(const gs_program* prog, const gs_sim_opts* opts_in, 
     if (s->opts.kernel == GS_KERNEL_TILE) {
         uint32_t per = 0;
         s->tile_groups = pls.ng;
-        e = tile_setup(s->tw, s->tile_groups, s->tile.n_slots, p.n_eval, p.n_levels, s->desc_smem,
-                       s->tile_max_width, p.n_reg > 0, &per);
+        e = tile_setup(s->tw, s->tile_groups, s->tile.n_slots, p.n_eval, (uint32_t)s->tile_steps.size(),
+                       s->desc_smem, p.n_reg > 0, &per);
         if (e != cudaSuccess || per == 0)
             return fail(e != cudaSuccess ? GS_ERR_CUDA : GS_ERR_ARG,
                         std::string("TILE: kernel setup: ") + (e != cudaSuccess ? cudaGetErrorString(e) : "0 CTAs fit an SM"));
         const uint32_t tiles = (uint32_t)(opts->lanes / (32ull * s->tw));
         s->tile_grid = std::min<uint32_t>((tiles + s->tile_groups - 1) / s->tile_groups, per * s->sms);
+    }
+    if (s->opts.kernel == GS_KERNEL_CLUSTER) {
+        const uint64_t sl = opts->slab_lanes ? opts->slab_lanes : 256;
+        s->cluster_size = opts->cluster_size ? opts->cluster_size : 2;
+        s->slab_vec = (uint32_t)(sl / 128);
+        s->n_slabs = (uint32_t)(opts->lanes / sl);
+        uint32_t maxc = 0;
+        e = cluster_max_active(s->slab_vec, s->cluster_size, &maxc);
+        if (e != cudaSuccess || maxc == 0)
+            return fail(e != cudaSuccess ? GS_ERR_CUDA : GS_ERR_ARG,
+                        std::string("CLUSTER: no cluster fits: ") + (e != cudaSuccess ? cudaGetErrorString(e) : "0 active"));
+        s->clusters = std::min(maxc, s->n_slabs);
+        s->tile_steps = pls.steps;
     }
     CU(cudaStreamCreateWithFlags(&s->cap, cudaStreamNonBlocking));
     if (s->groups > 1) {
@@ -553,7 +613,7 @@ static gs_status sim_create(const gs_program* prog, const gs_sim_opts* opts_in, 
         {L.t_ldst, s->tile.latch_dst.data(), s->tile.latch_dst.size() * 4},
         {L.t_wbrow, s->tile.wb_row.data(), s->tile.wb_row.size() * 4},
         {L.t_wbslot, s->tile.wb_slot.data(), s->tile.wb_slot.size() * 4},
-        {L.t_lvl, p.level_off.data(), s->tw ? p.level_off.size() * 4 : 0},
+        {L.t_steps, s->tile_steps.data(), s->tile_steps.size() * sizeof(uint2)},
     };
     for (const Up& u : ups)
         if (u.n) CU(cudaMemcpyAsync(s->ws + u.off, u.src, u.n, cudaMemcpyHostToDevice, s->stream));
@@ -661,8 +721,9 @@ static gs_status sim_step(gs_sim* s, uint32_t n) {
     if (s->bound == 2 && s->cycle + n > s->bound_base + s->bound_cycles)
         return fail(GS_ERR_STATE, "gs_sim_step: stepping past the bound stimulus cycles");
     CU(cudaSetDevice(s->opts.device));
-    if (s->opts.kernel == GS_KERNEL_TILE) {       // every cycle of the step in one launch
-        CU(tile_launch(s, n, s->stream));
+    if (s->opts.kernel == GS_KERNEL_TILE || s->opts.kernel == GS_KERNEL_CLUSTER) {
+        // every cycle of the step in one launch
+        CU(s->opts.kernel == GS_KERNEL_TILE ? tile_launch(s, n, s->stream) : cluster_launch(s, n, s->stream));
         s->cycle += n;
         clear_error();
         return GS_OK;
@@ -860,7 +921,8 @@ static gs_status sim_read_signature(gs_sim* s, gs_signature* out) {
 
 static uint64_t launches_per_cycle(const gs_sim* s) {
     const Program& p = *s->prog;
-    if (s->opts.kernel == GS_KERNEL_TILE) return 1;      // per gs_sim_step call, not per cycle
+    if (s->opts.kernel == GS_KERNEL_TILE || s->opts.kernel == GS_KERNEL_CLUSTER)
+        return 1;                                          // per gs_sim_step call, not per cycle
     uint64_t lv = 0;
     for (uint32_t l = 0; l < p.n_levels; ++l)
         if (p.level_off[l + 1] > p.level_off[l]) lv++;
@@ -886,13 +948,14 @@ static gs_status sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
         all_bytes += lb[l];
     }
     std::memset(out, 0, sizeof(*out));
-    if (s->opts.kernel == GS_KERNEL_TILE) {
+    if (s->opts.kernel == GS_KERNEL_TILE || s->opts.kernel == GS_KERNEL_CLUSTER) {
         // one launch runs all n cycles; "level" bytes are the same algorithmic gather model
         cudaEvent_t a0 = nullptr, a1 = nullptr;
         cudaError_t e = cudaEventCreate(&a0);
         if (e == cudaSuccess) e = cudaEventCreate(&a1);
         if (e == cudaSuccess) e = cudaEventRecord(a0, s->stream);
-        if (e == cudaSuccess) e = tile_launch(s, n, s->stream);
+        if (e == cudaSuccess)
+            e = s->opts.kernel == GS_KERNEL_TILE ? tile_launch(s, n, s->stream) : cluster_launch(s, n, s->stream);
         if (e == cudaSuccess) e = cudaEventRecord(a1, s->stream);
         if (e == cudaSuccess) e = cudaEventSynchronize(a1);
         float ms = 0;
@@ -1057,6 +1120,25 @@ gs_status gs_sim_get_config(const gs_sim* s, int* kernel, uint32_t* lane_groups)
         if (!s || !kernel || !lane_groups) return fail(GS_ERR_ARG, "gs_sim_get_config: NULL argument");
         *kernel = s->opts.kernel;
         *lane_groups = s->groups;
+        clear_error();
+        return GS_OK;
+    })
+}
+
+gs_status gs_sim_get_launch(const gs_sim* s, gs_launch_info* out) {
+    GS_TRY({
+        if (!s || !out) return fail(GS_ERR_ARG, "gs_sim_get_launch: NULL argument");
+        std::memset(out, 0, sizeof(*out));
+        out->kernel = s->opts.kernel;
+        out->lane_groups = s->groups;
+        out->tile_words = s->tw;
+        out->tile_groups = s->opts.kernel == GS_KERNEL_TILE ? s->tile_groups : 0;
+        out->tile_desc = (uint32_t)s->desc_smem;
+        out->grid = s->opts.kernel == GS_KERNEL_TILE ? s->tile_grid
+                    : s->opts.kernel == GS_KERNEL_CLUSTER ? s->clusters * s->cluster_size : 0;
+        out->cluster_size = s->cluster_size;
+        out->slab_lanes = s->slab_vec * 128;
+        out->live_slots = s->opts.kernel == GS_KERNEL_TILE ? s->tile.n_slots : 0;
         clear_error();
         return GS_OK;
     })

@@ -516,6 +516,72 @@ def test_lane_groups_reject_bad_shapes():
         assert e.value.code == gs.GS_ERR_ARG
 
 
+# ------------------------------------------------------------------ kernel C (cluster slabs)
+@pytest.mark.parametrize("cs,slab,lanes", [(1, 128, 4096), (2, 256, 8192), (4, 512, 16384), (2, 128, 2048),
+                                            (8, 256, 8192), (2, 384, 12288)])
+def test_cluster_kernel_every_lane_vs_oracle(cs, slab, lanes):
+    """Kernel C (a thread-block cluster owns a lane slab and walks every level of every cycle
+    of the step, cluster barrier between levels): a sequential netlist with fused latches, Q
+    inputs, 5-6-input LUTs and leftover latches; every lane's outputs, registers, signature
+    and the trace of boundary words vs the oracle; steps split over several launches; a lane
+    offset; identical to kernel A."""
+    nls = [workloads.synthetic(3000, 120, 20, 32, 16, seed=23, name="cl"),
+           workloads.random_tiny(5, n_pi=6, n_reg=5, n_gates=300, n_po=12, max_k=6),
+           workloads.register_edge_cases()]
+    for nl in nls:
+        prog = compile_nl(nl)
+        W_ = lanes // 64
+        tw = [0, slab // 64 - 1, slab // 64, W_ - 1]
+        sim = gs.Sim(prog, lanes, kernel="cluster", cluster_size=cs, slab_lanes=slab, trace_words=tw,
+                     trace_cycles=11, lane_offset=64 * 31)
+        sim.bind_generated(8)
+        for n in (1, 3, 7):
+            sim.step(n)
+        sim.sync()
+        o = oracle.simulate(nl, np.arange(lanes) + 64 * 31, 11, seed=8)
+        assert np.array_equal(gs.unpack_lanes(sim.read_outputs()).T, o["last"])
+        assert np.array_equal(gs.unpack_lanes(sim.read_registers()).T, o["regs"])
+        assert np.array_equal(sim.read_lane_signatures(), o["sig"])
+        sel = np.concatenate([np.arange(64) + 64 * w for w in tw])
+        assert np.array_equal(gpu_trace_bits(sim.read_trace(), None), o["trace"][sel])
+        sig = sim.signature()
+        assert sig["cycles"] == 11 and sig["out_popcount"] == int(o["trace"].sum())
+        sim.close()
+
+
+def test_cluster_kernel_c3_equals_lut_and_streamed_io():
+    """Kernel C on C3 (100k gates, 4k registers) at 16,384 lanes == kernel A on every lane;
+    and gs_sim_run_streamed (host stimuli in, every output out) through kernel C == kernel A."""
+    cfg = workloads.CONFIGS["C3"]
+    nl = cfg.netlist()
+    prog = compile_nl(nl)
+    c = run_gpu(nl, cfg.lanes, 30, "cluster", seed=3, prog=prog)
+    a = run_gpu(nl, cfg.lanes, 30, "lut", seed=3, prog=prog)
+    for key in ("outputs", "regs", "sigs"):
+        assert np.array_equal(c[key], a[key]), key
+    assert c["signature"]["lane_sig_sum"] == a["signature"]["lane_sig_sum"]
+    assert c["signature"]["out_popcount"] == a["signature"]["out_popcount"]
+    W_ = 4096 // 64
+    stim = workloads.random_host_stimulus(9, 12, nl.n_pi, W_)
+    outs = []
+    for kernel in ("cluster", "lut"):
+        sim = gs.Sim(prog, 4096, kernel=kernel)
+        out = np.zeros((12, nl.n_po, W_), dtype=np.uint64)
+        sim.run_streamed(stim, out, chunk=5)
+        sim.sync()
+        outs.append((out, sim.read_lane_signatures()))
+        sim.close()
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+
+
+def test_cluster_kernel_rejects_bad_shapes():
+    prog = compile_nl(workloads.adder(8))
+    for kw in (dict(slab_lanes=192), dict(slab_lanes=2048), dict(cluster_size=3)):
+        with pytest.raises(gs.GsError) as e:
+            gs.Sim(prog, 1024, kernel="cluster", **kw)
+        assert e.value.code == gs.GS_ERR_ARG
+
+
 # ------------------------------------------------------------------ cone collapsing (lut_k)
 @pytest.mark.parametrize("L", [3, 6])
 @pytest.mark.parametrize("kernel", ["lut", "poly", "ab", "tile"])
@@ -881,8 +947,9 @@ def test_fuzz_every_kernel_all_lanes_vs_oracle(case):
     lut_k = int(rng.choice([0, 0, 3, 4, 6, 8]))
     prog = gs.Netlist.from_arrays(nl).compile(balance=balance, lut_k=lut_k)
     o = oracle.simulate(nl, np.arange(lanes) + offset, cycles, seed=seed, want=("last", "regs", "sig"))
-    kernels = ["lut", "poly", "ab", "auto"] + (["tile"] if lanes % 128 == 0 else [])
-    runs = [(k, {}) for k in kernels]
+    kernels = ["lut", "poly", "ab", "auto"] + (["tile", "cluster"] if lanes % 128 == 0 else [])
+    runs = [(k, {}) if k != "cluster" else (k, dict(slab_lanes=128, cluster_size=[1, 2, 4][case % 3]))
+            for k in kernels]
     # opt-in launch options: one pick per case for kernel A, one descriptor source for T
     opt = [dict(flags=gs.GS_SIM_NO_PDL), dict(flags=gs.GS_SIM_NO_GRID_STRIDE), dict(lane_groups=1),
            dict(lane_groups=2)][case % 4]
