@@ -39,6 +39,11 @@ sys.path.insert(0, ROOT)
 METRIC = "stimulus-gate-cycle evals/s at 1/2/4/8 B200; HBM GB/s vs roofline"
 UNIT = "sgc/s"
 DEFAULT_SUB_LANES = 32768       # sharded configs: lanes per sub-batch (tests use the same)
+# level assignment per workload (bench --levels auto), from the round-2 A/B
+# (profiles/r02_levels_ab.txt): the DRAM-bound configs run faster on ASAP levels (a producer
+# and its readers stay closer in time, so more inputs hit L2: C4 +8 %, C5 +3 %), the
+# launch-bound C3 on balanced levels (ASAP -8 %: narrow levels)
+AUTO_LEVELS = {"C4": "asap", "C5": "asap"}
 
 
 def parse():
@@ -57,7 +62,9 @@ def parse():
     ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab", "tile", "cluster", "auto"])
     ap.add_argument("--cluster-size", type=int, default=0, help="kernel C: CTAs per cluster (0 = auto)")
     ap.add_argument("--slab-lanes", type=int, default=0, help="kernel C: lanes per slab (0 = auto)")
-    ap.add_argument("--no-balance", action="store_true", help="ASAP levels (balance-off A/B)")
+    ap.add_argument("--levels", default="auto", choices=["auto", "balanced", "asap", "alap"],
+                    help="level assignment (auto: the workload's measured best, DESIGN.md §6)")
+    ap.add_argument("--no-balance", action="store_true", help="= --levels asap")
     ap.add_argument("--tile-words", type=int, default=0, help="kernel T: 32-bit words per slot")
     ap.add_argument("--tile-groups", type=int, default=0, help="kernel T: thread groups per CTA")
     ap.add_argument("--tile-desc", default="auto", choices=["auto", "tma", "global"],
@@ -314,7 +321,11 @@ def main():
         lane_offset = rank * lanes                      # weak scaling: own global range per rank
     lanes_total = lanes_rank * world
     t0 = time.perf_counter()
-    prog = gs.Netlist.from_arrays(nl).compile(balance=not args.no_balance, lut_k=args.lut_k)
+    levels = "asap" if args.no_balance else args.levels
+    if levels == "auto":
+        levels = AUTO_LEVELS.get(cfg.name, "balanced")
+    prog = gs.Netlist.from_arrays(nl).compile(balance={"balanced": 1, "asap": 0, "alap": 2}[levels],
+                                              lut_k=args.lut_k)
     compile_s = time.perf_counter() - t0
     info = prog.info
     G = info["n_eval_gates"]
@@ -499,7 +510,7 @@ def main():
             "config": {"workload": f"{cfg.name}: {cfg.label}", "gates": G, "registers": info["n_reg"],
                        "levels": info["n_levels"], "lanes_total": lanes_total, "lanes_per_gpu": lanes_rank,
                        "sub_batches_per_gpu": subs, "lanes_per_sub_batch": lanes,
-                       "cycles_per_step": C, "kernel": args.kernel, "balance": not args.no_balance,
+                       "cycles_per_step": C, "kernel": args.kernel, "level_assignment": levels,
                        "lut_unroll": args.lut_unroll, "lane_groups": sim.config["lane_groups"],
                        "pdl": not args.no_pdl, "tile_words": args.tile_words, "tile_groups": args.tile_groups,
                        "lut_k": args.lut_k, "grid_stride": not args.no_grid_stride,

@@ -31,7 +31,13 @@
 
 namespace gs {
 
-constexpr uint32_t CLUSTER_CTA = 512;
+#ifndef GS_CLUSTER_CTA
+#define GS_CLUSTER_CTA 256
+#endif
+#ifndef GS_CLUSTER_MINB
+#define GS_CLUSTER_MINB 4
+#endif
+constexpr uint32_t CLUSTER_CTA = GS_CLUSTER_CTA;   // threads per CTA (several CTAs per SM)
 constexpr unsigned long long C_MISR_POLY = 0x42F0E1EBA9EA3693ULL;   // CRC-64/ECMA-182
 
 __device__ __forceinline__ void cluster_sync_all() {
@@ -114,7 +120,7 @@ __device__ __forceinline__ void c_gate(const ClusterArgs& a, uint32_t gate, cons
 }
 
 template <int VPT>
-__global__ void __launch_bounds__(CLUSTER_CTA, 1) k_cluster(ClusterArgs a) {
+__global__ void __launch_bounds__(CLUSTER_CTA, GS_CLUSTER_MINB) k_cluster(ClusterArgs a) {
     __shared__ uint32_t s_slab;
     const uint32_t rank = cluster_rank(), ncta = cluster_ncta();
     const uint32_t gtid = rank * blockDim.x + threadIdx.x, gtot = ncta * blockDim.x;
@@ -128,7 +134,8 @@ __global__ void __launch_bounds__(CLUSTER_CTA, 1) k_cluster(ClusterArgs a) {
                              sink_cycles = a.ctl->sink_cycles;
     const uint32_t SV = a.slab_vec;                  // 16-byte vectors per slab row
     const uint32_t SW = SV * 2;                      // 64-bit words per slab row
-    const uint32_t VG = SV / VPT;                    // threads per gate
+    const uint32_t VG = SV / VPT;                    // threads per gate (a power of two)
+    const uint32_t vgs = 31u - __clz(VG);
     unsigned long long pop = 0;
     for (;;) {
         // ---- next slab of the cluster: CTA 0 claims it, every CTA reads it over DSMEM
@@ -160,7 +167,7 @@ __global__ void __launch_bounds__(CLUSTER_CTA, 1) k_cluster(ClusterArgs a) {
                 const uint32_t n = st.y * VG;
 #pragma unroll 1
                 for (uint32_t u = gtid; u < n; u += gtot) {
-                    const uint32_t gi = u / VG, vgi = u - gi * VG;
+                    const uint32_t gi = u >> vgs, vgi = u & (VG - 1);
                     const uint32_t gate = st.x + gi;
                     const uint4 in = __ldg(a.din + gate);
                     const uint4 au = __ldg(reinterpret_cast<const uint4*>(a.aux) + gate);

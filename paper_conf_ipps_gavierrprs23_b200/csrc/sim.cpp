@@ -40,8 +40,8 @@ constexpr size_t TILE_SMEM_MAX = 232448;   // 227 KB opt-in shared memory per CT
 gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
     if (o.kernel == GS_KERNEL_CLUSTER) {
         const uint64_t sl = o.slab_lanes ? o.slab_lanes : 256;
-        if (sl % 128 || o.lanes % sl)
-            return fail(GS_ERR_ARG, "CLUSTER: slab_lanes must be a multiple of 128 dividing lanes");
+        if (sl % 128 || o.lanes % sl || ((sl / 128) & (sl / 128 - 1)))
+            return fail(GS_ERR_ARG, "CLUSTER: slab_lanes must be 128 x a power of two dividing lanes");
         const uint32_t cs = o.cluster_size ? o.cluster_size : 2;
         if (cs != 1 && cs != 2 && cs != 4 && cs != 8 && cs != 16)
             return fail(GS_ERR_ARG, "CLUSTER: cluster_size must be 1, 2, 4, 8 or 16");
@@ -65,9 +65,9 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
     // choose (descriptor mode, tile words, groups per CTA).  Kernel T is latency-bound per
     // tile (a level barrier per step), so a launch takes ~ waves x tile time with waves =
     // ceil(tiles / (groups x SMs)): score = lanes per wave (quantisation included), resident
-    // descriptors weighted 4/3, then wider tiles, then resident > TMA stream > global, then
-    // more groups.  C2 (256 live slots): 2 groups x 2,048-lane tiles, TMA stream, 3.0e13 vs
-    // 2.56e13 for 1 group with resident descriptors (profiles/r02_kernelT_configs_C2.txt)
+    // descriptors weighted 4/3 over a TMA stream, then wider tiles, then resident > TMA stream
+    // > global, then more groups.  C2 (256 live slots): 2 groups x 2,048-lane tiles with the
+    // small descriptor table read through L1/L2, 3.18e13 (profiles/r02_kernelT_configs_C2.txt)
     const int forced = (o.flags & GS_SIM_TILE_DESC_GLOBAL) ? 0 : (o.flags & GS_SIM_TILE_DESC_TMA) ? 2 : -1;
     uint64_t best = 0;
     for (int ds : {1, 2, 0}) {
@@ -83,11 +83,15 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
                 const uint64_t slots = (uint64_t)ng * (uint64_t)sms;
                 const uint64_t waves = (tiles + slots - 1) / slots;
                 const uint64_t per_wave = o.lanes / waves;
+                // descriptor source weights (measured on C2, 2,048-lane tiles): resident 2.56e13
+                // vs TMA-streamed 1.92e13 (1 group); with 2 groups, global (L1/L2-cached) 3.18e13
+                // vs TMA 3.04e13 — a small table (<= 128 KB) stays cache-resident, a large one
+                // is better streamed (mid-size circuits, round 1)
+                const bool small_table = (uint64_t)p.n_eval * 16 <= 131072;
+                const uint64_t wgt = ds == 1 ? 40 : ds == 2 ? 30 : small_table ? 32 : 28;
                 const uint64_t pref = ds == 1 ? 2 : ds == 2 ? 1 : 0;
-                // resident descriptors counted 4/3 (no per-step TMA wait): measured on C2 at
-                // 2,048-lane tiles, resident 2.56e13 vs TMA-streamed 1.92e13
-                const uint64_t score = ((per_wave * (ds == 1 ? 4 : 3)) << 24) | ((uint64_t)tw << 16) |
-                                       (pref << 12) | ((uint64_t)ng << 8);
+                const uint64_t score = ((per_wave * wgt) << 20) | ((uint64_t)tw << 12) | (pref << 8) |
+                                       ((uint64_t)ng << 4);
                 if (score > best) { best = score; pl.tw = tw; pl.ng = ng; pl.desc_smem = ds; }
             }
         }

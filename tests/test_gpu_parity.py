@@ -56,6 +56,7 @@ def lane_bits(words_2d, lanes_idx):
 
 
 KERNELS = ["lut", "poly", "ab"]
+BENCH_BALANCE = {"balanced": 1, "asap": 0, "alap": 2}      # bench.py --levels -> gs_compile_opts.balance
 
 
 # ------------------------------------------------------------------ C1: adder
@@ -518,7 +519,7 @@ def test_lane_groups_reject_bad_shapes():
 
 # ------------------------------------------------------------------ kernel C (cluster slabs)
 @pytest.mark.parametrize("cs,slab,lanes", [(1, 128, 4096), (2, 256, 8192), (4, 512, 16384), (2, 128, 2048),
-                                            (8, 256, 8192), (2, 384, 12288)])
+                                            (8, 256, 8192), (2, 1024, 16384)])
 def test_cluster_kernel_every_lane_vs_oracle(cs, slab, lanes):
     """Kernel C (a thread-block cluster owns a lane slab and walks every level of every cycle
     of the step, cluster barrier between levels): a sequential netlist with fused latches, Q
@@ -576,7 +577,7 @@ def test_cluster_kernel_c3_equals_lut_and_streamed_io():
 
 def test_cluster_kernel_rejects_bad_shapes():
     prog = compile_nl(workloads.adder(8))
-    for kw in (dict(slab_lanes=192), dict(slab_lanes=2048), dict(cluster_size=3)):
+    for kw in (dict(slab_lanes=192), dict(slab_lanes=384), dict(slab_lanes=2048), dict(cluster_size=3)):
         with pytest.raises(gs.GsError) as e:
             gs.Sim(prog, 1024, kernel="cluster", **kw)
         assert e.value.code == gs.GS_ERR_ARG
@@ -838,9 +839,10 @@ def test_c4_full_config_256_lanes_every_cycle_and_probes():
     spread over the batch (lanes 0/63/64/last, both sides of every lane-group boundary) x all
     1,000 cycles vs the oracle — every output bit of every cycle, every register bit, the
     per-lane MISR — and the probes' closed forms on every lane."""
+    import bench
     cfg = workloads.CONFIGS["C4"]
     nl = cfg.netlist()
-    prog = compile_nl(nl)
+    prog = gs.Netlist.from_arrays(nl).compile(balance=BENCH_BALANCE[bench.AUTO_LEVELS.get("C4", "balanced")])
     sample = workloads.sample_lanes(cfg.lanes, 1, 256, seed=4)
     assert {0, 63, 64, cfg.lanes - 1} <= set(sample.tolist())
     tw = sorted(set((sample // 64).tolist()))
@@ -866,7 +868,7 @@ def test_c5_every_shard_32_lanes_every_cycle_bench_config():
     import bench
     cfg = workloads.CONFIGS["C5"]
     nl = cfg.netlist()
-    prog = compile_nl(nl)
+    prog = gs.Netlist.from_arrays(nl).compile(balance=BENCH_BALANCE[bench.AUTO_LEVELS.get("C5", "balanced")])
     sub = bench.DEFAULT_SUB_LANES
     sample = workloads.sample_lanes(cfg.lanes, cfg.shards, 256 // cfg.shards, seed=5, lanes_per_word=2)
     tw_all = sorted(set((sample % sub // 64).tolist()))        # local words of any sub-batch
