@@ -66,7 +66,7 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
     // tile (a level barrier per step), so a launch takes ~ waves x tile time with waves =
     // ceil(tiles / (groups x SMs)): score = lanes per wave (quantisation included), resident
     // descriptors weighted 4/3 over a TMA stream, then wider tiles, then resident > TMA stream
-    // > global, then more groups.  C2 (256 live slots): 2 groups x 2,048-lane tiles with the
+    // > global, then fewer groups (more threads per tile).  C2 (256 live slots): 2 groups x 2,048-lane tiles with the
     // small descriptor table read through L1/L2, 3.18e13 (profiles/r02_kernelT_configs_C2.txt)
     const int forced = (o.flags & GS_SIM_TILE_DESC_GLOBAL) ? 0 : (o.flags & GS_SIM_TILE_DESC_TMA) ? 2 : -1;
     uint64_t best = 0;
@@ -90,8 +90,11 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
                 const bool small_table = (uint64_t)p.n_eval * 16 <= 131072;
                 const uint64_t wgt = ds == 1 ? 40 : ds == 2 ? 30 : small_table ? 32 : 28;
                 const uint64_t pref = ds == 1 ? 2 : ds == 2 ? 1 : 0;
-                const uint64_t score = ((per_wave * wgt) << 20) | ((uint64_t)tw << 12) | (pref << 8) |
-                                       ((uint64_t)ng << 4);
+                // ties (e.g. every plan fits one wave): more SMs busy, then wider tiles (C1,
+                // 1,024 lanes: 8 tiles of 128 lanes 1.03e10 vs one 1,024-lane tile 7.8e9)
+                const uint64_t busy = std::min<uint64_t>((tiles + ng - 1) / ng, (uint64_t)sms);
+                const uint64_t score = (((per_wave / 64) * wgt) << 28) | (busy << 16) | ((uint64_t)tw << 8) |
+                                       (pref << 4) | (uint64_t)(8 - ng);
                 if (score > best) { best = score; pl.tw = tw; pl.ng = ng; pl.desc_smem = ds; }
             }
         }
@@ -121,7 +124,10 @@ gs_sim_opts resolve_auto(const Program& p, const gs_sim_opts& o) {
     r.kernel = GS_KERNEL_TILE;
     Plans pl;
     const std::string saved = gs_last_error();
-    if (p.n_eval == 0 || make_plans(p, r, pl) != GS_OK || pl.desc_smem == 0) r.kernel = GS_KERNEL_LUT;
+    // (a large descriptor table read from global memory is slow: T only with resident or
+    // TMA-streamed descriptors, or a table small enough to stay cache-resident)
+    if (p.n_eval == 0 || make_plans(p, r, pl) != GS_OK || (pl.desc_smem == 0 && (uint64_t)p.n_eval * 16 > 131072))
+        r.kernel = GS_KERNEL_LUT;
     set_error(saved);
     return r;
 }

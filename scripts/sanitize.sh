@@ -13,7 +13,10 @@ prog = gs.Netlist.from_arrays(nl).compile()
 lanes = 16384 if kernel.startswith("lut_") else 2048
 extra = {"lut_groups": dict(lane_groups=4),                              # concurrent graph branches
          "lut_u4": dict(lane_groups=1, lut_unroll=4),                    # U = 4 wide path
-         "tile_tma": dict(flags=gs.GS_SIM_TILE_DESC_TMA)}.get(kernel, {})
+         "tile_tma": dict(flags=gs.GS_SIM_TILE_DESC_TMA, tile_groups=2),  # chunked TMA stream, 2 groups
+         "tile_global": dict(flags=gs.GS_SIM_TILE_DESC_GLOBAL, tile_groups=4),
+         "cluster_2": dict(cluster_size=2, slab_lanes=256),             # kernel C, DSMEM slab broadcast
+         "cluster_8": dict(cluster_size=8, slab_lanes=256)}.get(kernel, {})
 if kernel == "lut_u4":
     lanes = 65536
 sim = gs.Sim(prog, lanes, kernel=kernel.split("_")[0], trace_words=[0, 5], trace_cycles=4,
@@ -27,7 +30,7 @@ sim.read_outputs(); sim.read_registers(); sim.read_lane_signatures(); sim.signat
 sim.close()
 print("ok", kernel)
 PY
-for k in ${KERNELS:-lut poly ab tile lut_groups lut_u4 tile_tma}; do
+for k in ${KERNELS:-lut poly ab tile lut_groups lut_u4 tile_tma tile_global cluster_2 cluster_8}; do
   for tool in memcheck racecheck synccheck; do
     timeout 600 compute-sanitizer --tool $tool --error-exitcode 9 python /tmp/san_run.py $k > $OUT/${k}_${tool}.log 2>&1
     echo "$k $tool rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY' $OUT/${k}_${tool}.log | tr '\n' ' ')" >> $OUT/summary.txt
