@@ -103,9 +103,13 @@ struct TileArgs {
     uint64_t word_off;                // global 64-bit word of local lane 0
     uint32_t ncycles, n_tiles;
 };
-// steps of a program for kernel T: one per non-empty level, levels wider than `chunk` gates
-// cut into chunks (chunk = 0: no cutting)
-void tile_steps(const uint32_t* level_off, uint32_t n_levels, uint32_t chunk, std::vector<uint2>& out);
+// Steps of a program for kernels T and C: {first gate, n | k << 24 | level_end << 31}.  One
+// step per run of equal fan-in k inside a non-empty level (aux != NULL; k = 0 when aux is
+// NULL: one step per level), runs longer than `chunk` gates cut (chunk = 0: no cutting);
+// level_end marks the last step of a level (the level barrier follows it).
+constexpr uint32_t STEP_N_MASK = 0xFFFFFFu;
+void tile_steps(const uint32_t* level_off, uint32_t n_levels, const GateAux* aux, uint32_t chunk,
+                std::vector<uint2>& out);
 size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_steps,
                        int desc_mode);
 cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_steps,

@@ -164,7 +164,7 @@ __global__ void __launch_bounds__(CLUSTER_CTA, GS_CLUSTER_MINB) k_cluster(Cluste
 #pragma unroll 1
             for (uint32_t si = 0; si < a.n_steps; ++si) {
                 const uint2 st = __ldg(a.steps + si);
-                const uint32_t n = st.y * VG;
+                const uint32_t n = (st.y & STEP_N_MASK) * VG;
 #pragma unroll 1
                 for (uint32_t u = gtid; u < n; u += gtot) {
                     const uint32_t gi = u >> vgs, vgi = u & (VG - 1);

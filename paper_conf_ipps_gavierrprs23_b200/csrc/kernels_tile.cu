@@ -6,13 +6,18 @@
 
 namespace gs {
 
-void tile_steps(const uint32_t* level_off, uint32_t n_levels, uint32_t chunk, std::vector<uint2>& out) {
+void tile_steps(const uint32_t* level_off, uint32_t n_levels, const GateAux* aux, uint32_t chunk,
+                std::vector<uint2>& out) {
     out.clear();
+    const uint32_t cap = chunk ? std::min(chunk, STEP_N_MASK) : STEP_N_MASK;
     for (uint32_t l = 0; l < n_levels; ++l)
         for (uint32_t g = level_off[l]; g < level_off[l + 1];) {
-            const uint32_t n = chunk ? std::min(chunk, level_off[l + 1] - g) : level_off[l + 1] - g;
-            out.push_back(make_uint2(g, n));
-            g += n;
+            const uint32_t k = aux ? (aux[g].k & 0xFFu) : 0u;
+            uint32_t e = g + 1;                      // run of equal k (gates are k-grouped per level)
+            while (e < level_off[l + 1] && e - g < cap && (!aux || (aux[e].k & 0xFFu) == k)) ++e;
+            const bool end = e == level_off[l + 1];
+            out.push_back(make_uint2(g, (e - g) | (k << 24) | (end ? 0x80000000u : 0u)));
+            g = e;
         }
 }
 

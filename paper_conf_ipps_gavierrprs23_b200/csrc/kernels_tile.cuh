@@ -127,6 +127,21 @@ __device__ __forceinline__ void tile_gate(uint4* sl, uint32_t V, uint32_t v, uin
     }
 }
 
+// All (gate, vector group) units of one step, every gate with fan-in K.  d0 = the descriptor of
+// the thread's first unit, already loaded (prefetched before the previous barrier).
+template <int K, bool HASQ, int P, uint32_t VS, uint32_t VSH, uint32_t GT>
+__device__ __forceinline__ void tile_step(uint4* sl, uint32_t V, const uint4* dl, uint32_t g0, uint32_t n,
+                                          uint32_t tid, const uint4* desc_hi, uint32_t q0, uint32_t R,
+                                          const uint4& d0) {
+    if (tid >= n) return;
+    tile_gate<K, HASQ, P>(sl, V, tid & (VS - 1), VS, d0, desc_hi, g0 + (tid >> VSH), q0, R);
+#pragma unroll 1
+    for (uint32_t u = tid + GT; u < n; u += GT) {
+        const uint32_t gi = u >> VSH, v = u & (VS - 1);
+        tile_gate<K, HASQ, P>(sl, V, v, VS, dl[gi], desc_hi, g0 + gi, q0, R);
+    }
+}
+
 __device__ __forceinline__ void group_sync(uint32_t id, uint32_t nthreads) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
@@ -208,9 +223,10 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     if (tid == 0) *tile_slot = atomicAdd(a.tile_next, 1u);
     group_sync(bar, GT);
     uint32_t tile = *tile_slot;
+    group_sync(bar, GT);                                  // every thread has read it before the next claim
     if (DM == 2 && tid == 0 && tile < a.n_tiles && n_steps) {
         const uint2 s0 = steps[0];
-        tma_load_1d(dbuf_s, a.desc + s0.x, s0.y * 16, mbar_s);
+        tma_load_1d(dbuf_s, a.desc + s0.x, (s0.y & STEP_N_MASK) * 16, mbar_s);
     }
     while (tile < a.n_tiles) {
         // claim the next tile now, so the descriptor stream knows whether to continue
@@ -248,42 +264,48 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
             group_sync(bar, GT);
             // ---- steps: every (gate, vector group) unit of the step, then the group barrier
             const bool more = c + 1 < a.ncycles || next_tile < a.n_tiles;   // stream continues
+            // descriptor of this thread's first unit of step 0 (resident / global modes: the
+            // next step's is prefetched before each barrier, so its latency overlaps the wait)
+            uint4 dpre = make_uint4(0, 0, 0, 0);
+            if (DM != 2 && n_steps && (tid >> VSH) < (steps[0].y & STEP_N_MASK)) dpre = dsm[steps[0].x + (tid >> VSH)];
 #pragma unroll 1
             for (uint32_t si = 0; si < n_steps; ++si) {
                 const uint2 st = steps[si];
+                const uint32_t sn_gates = st.y & STEP_N_MASK;
                 const uint4* dl = dsm + st.x;
                 if (DM == 2) {
                     const uint32_t b = step & 1;
                     if (tid == 0 && (si + 1 < n_steps || more)) {
                         const uint2 sn = steps[si + 1 < n_steps ? si + 1 : 0];
-                        tma_load_1d(dbuf_s + (b ^ 1) * (TILE_CHUNK * 16), a.desc + sn.x, sn.y * 16,
+                        tma_load_1d(dbuf_s + (b ^ 1) * (TILE_CHUNK * 16), a.desc + sn.x, (sn.y & STEP_N_MASK) * 16,
                                     mbar_s + 8 * (b ^ 1));
                     }
                     mbar_wait(mbar_s + 8 * b, (step >> 1) & 1);
                     dl = dbuf + b * TILE_CHUNK;
                     ++step;
+                    if ((tid >> VSH) < sn_gates) dpre = dl[tid >> VSH];
                 }
-                const uint32_t n = st.y << VSH;
-#pragma unroll 1
-                for (uint32_t u = tid; u < n; u += GT) {
-                    const uint32_t gi = u >> VSH, v = u & (VS - 1);
-                    const uint32_t g = st.x + gi;
-                    const uint4 d = dl[gi];
-                    // k: warp-uniform except at k-group edges; the common 2-4-input gates are
-                    // tested first (a compare and branch each instead of the jump table)
-                    const uint32_t k = d.w & 15u;
-                    if (k == 2) tile_gate<2, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R);
-                    else if (k == 3) tile_gate<3, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R);
-                    else if (k == 4) tile_gate<4, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R);
-                    else switch (k) {
-                        case 1: tile_gate<1, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R); break;
-                        case 5: tile_gate<5, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R); break;
-                        case 6: tile_gate<6, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R); break;
-                        case 7: tile_gate<7, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R); break;
-                        default: tile_gate<8, HASQ, P>(sl, V, v, VS, d, a.desc_hi, g, q0, R); break;
-                    }
+                // every gate of a step has the same fan-in k (steps are cut at k changes), so the
+                // dispatch happens once per step, not per gate
+                const uint32_t n = sn_gates << VSH;
+                const uint4 d0 = dpre;
+                switch ((st.y >> 24) & 15u) {
+                    case 2: tile_step<2, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
+                    case 3: tile_step<3, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
+                    case 4: tile_step<4, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
+                    case 1: tile_step<1, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
+                    case 5: tile_step<5, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
+                    case 6: tile_step<6, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
+                    case 7: tile_step<7, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
+                    default: tile_step<8, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
                 }
-                group_sync(bar, GT);
+                if (DM != 2) {                            // prefetch the next step's first descriptor
+                    const uint2 nx = steps[si + 1 < n_steps ? si + 1 : 0];
+                    if ((tid >> VSH) < (nx.y & STEP_N_MASK)) dpre = dsm[nx.x + (tid >> VSH)];
+                }
+                // the level barrier; TMA mode also needs it between the chunks of a level (the
+                // next chunk's copy reuses the buffer the previous chunk was read from)
+                if (DM == 2 || (st.y >> 31)) group_sync(bar, GT);
             }
             // ---- leftover latches into the next bank; MISR / popcount / trace of the POs
             for (uint32_t u = tid; u < a.n_latch * V; u += GT) {

@@ -45,14 +45,14 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
         const uint32_t cs = o.cluster_size ? o.cluster_size : 2;
         if (cs != 1 && cs != 2 && cs != 4 && cs != 8 && cs != 16)
             return fail(GS_ERR_ARG, "CLUSTER: cluster_size must be 1, 2, 4, 8 or 16");
-        tile_steps(p.level_off.data(), p.n_levels, 0, pl.steps);
+        tile_steps(p.level_off.data(), p.n_levels, nullptr, 0, pl.steps);
         return GS_OK;
     }
     if (o.kernel != GS_KERNEL_TILE) return GS_OK;
     if (gs_status st = tile_plan(p, pl.tile)) return st;
     std::vector<uint2> st_level, st_chunk;
-    tile_steps(p.level_off.data(), p.n_levels, 0, st_level);
-    tile_steps(p.level_off.data(), p.n_levels, GS_TILE_CHUNK, st_chunk);
+    tile_steps(p.level_off.data(), p.n_levels, p.aux.data(), 0, st_level);
+    tile_steps(p.level_off.data(), p.n_levels, p.aux.data(), GS_TILE_CHUNK, st_chunk);
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, o.device);
     if (o.tile_words && (o.tile_words != 4 && o.tile_words != 8 && o.tile_words != 16 && o.tile_words != 32 &&

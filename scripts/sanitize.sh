@@ -32,7 +32,7 @@ print("ok", kernel)
 PY
 for k in ${KERNELS:-lut poly ab tile lut_groups lut_u4 tile_tma tile_global cluster_2 cluster_8}; do
   for tool in memcheck racecheck synccheck; do
-    timeout 600 compute-sanitizer --tool $tool --error-exitcode 9 python /tmp/san_run.py $k > $OUT/${k}_${tool}.log 2>&1
+    timeout 1500 compute-sanitizer --tool $tool --error-exitcode 9 python /tmp/san_run.py $k > $OUT/${k}_${tool}.log 2>&1
     echo "$k $tool rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY' $OUT/${k}_${tool}.log | tr '\n' ' ')" >> $OUT/summary.txt
   done
 done
