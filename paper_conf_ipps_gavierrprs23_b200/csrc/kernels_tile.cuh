@@ -127,16 +127,12 @@ __device__ __forceinline__ void tile_gate(uint4* sl, uint32_t V, uint32_t v, uin
     }
 }
 
-// All (gate, vector group) units of one step, every gate with fan-in K.  d0 = the descriptor of
-// the thread's first unit, already loaded (prefetched before the previous barrier).
+// All (gate, vector group) units of one step, every gate with fan-in K.
 template <int K, bool HASQ, int P, uint32_t VS, uint32_t VSH, uint32_t GT>
 __device__ __forceinline__ void tile_step(uint4* sl, uint32_t V, const uint4* dl, uint32_t g0, uint32_t n,
-                                          uint32_t tid, const uint4* desc_hi, uint32_t q0, uint32_t R,
-                                          const uint4& d0) {
-    if (tid >= n) return;
-    tile_gate<K, HASQ, P>(sl, V, tid & (VS - 1), VS, d0, desc_hi, g0 + (tid >> VSH), q0, R);
+                                          uint32_t tid, const uint4* desc_hi, uint32_t q0, uint32_t R) {
 #pragma unroll 1
-    for (uint32_t u = tid + GT; u < n; u += GT) {
+    for (uint32_t u = tid; u < n; u += GT) {
         const uint32_t gi = u >> VSH, v = u & (VS - 1);
         tile_gate<K, HASQ, P>(sl, V, v, VS, dl[gi], desc_hi, g0 + gi, q0, R);
     }
@@ -264,10 +260,6 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
             group_sync(bar, GT);
             // ---- steps: every (gate, vector group) unit of the step, then the group barrier
             const bool more = c + 1 < a.ncycles || next_tile < a.n_tiles;   // stream continues
-            // descriptor of this thread's first unit of step 0 (resident / global modes: the
-            // next step's is prefetched before each barrier, so its latency overlaps the wait)
-            uint4 dpre = make_uint4(0, 0, 0, 0);
-            if (DM != 2 && n_steps && (tid >> VSH) < (steps[0].y & STEP_N_MASK)) dpre = dsm[steps[0].x + (tid >> VSH)];
 #pragma unroll 1
             for (uint32_t si = 0; si < n_steps; ++si) {
                 const uint2 st = steps[si];
@@ -283,25 +275,19 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
                     mbar_wait(mbar_s + 8 * b, (step >> 1) & 1);
                     dl = dbuf + b * TILE_CHUNK;
                     ++step;
-                    if ((tid >> VSH) < sn_gates) dpre = dl[tid >> VSH];
                 }
                 // every gate of a step has the same fan-in k (steps are cut at k changes), so the
                 // dispatch happens once per step, not per gate
                 const uint32_t n = sn_gates << VSH;
-                const uint4 d0 = dpre;
                 switch ((st.y >> 24) & 15u) {
-                    case 2: tile_step<2, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
-                    case 3: tile_step<3, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
-                    case 4: tile_step<4, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
-                    case 1: tile_step<1, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
-                    case 5: tile_step<5, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
-                    case 6: tile_step<6, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
-                    case 7: tile_step<7, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
-                    default: tile_step<8, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R, d0); break;
-                }
-                if (DM != 2) {                            // prefetch the next step's first descriptor
-                    const uint2 nx = steps[si + 1 < n_steps ? si + 1 : 0];
-                    if ((tid >> VSH) < (nx.y & STEP_N_MASK)) dpre = dsm[nx.x + (tid >> VSH)];
+                    case 2: tile_step<2, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R); break;
+                    case 3: tile_step<3, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R); break;
+                    case 4: tile_step<4, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R); break;
+                    case 1: tile_step<1, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R); break;
+                    case 5: tile_step<5, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R); break;
+                    case 6: tile_step<6, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R); break;
+                    case 7: tile_step<7, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R); break;
+                    default: tile_step<8, HASQ, P, VS, VSH, GT>(sl, V, dl, st.x, n, tid, a.desc_hi, q0, R); break;
                 }
                 // the level barrier; TMA mode also needs it between the chunks of a level (the
                 // next chunk's copy reuses the buffer the previous chunk was read from)
