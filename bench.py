@@ -67,7 +67,7 @@ def parse():
     ap.add_argument("--no-balance", action="store_true", help="= --levels asap")
     ap.add_argument("--tile-words", type=int, default=0, help="kernel T: 32-bit words per slot")
     ap.add_argument("--tile-groups", type=int, default=0, help="kernel T: thread groups per CTA")
-    ap.add_argument("--tile-desc", default="auto", choices=["auto", "tma", "global"],
+    ap.add_argument("--tile-desc", default="auto", choices=["auto", "tma", "global", "resident"],
                     help="kernel T descriptor source (auto: resident if it fits, else TMA stream)")
     ap.add_argument("--lut-unroll", type=int, default=0, help="vectors per thread (0 = auto)")
     ap.add_argument("--lane-groups", type=int, default=0,
@@ -332,7 +332,7 @@ def main():
     if world > 1:
         gdist.check_same_program(info["program_hash"])
     stream = torch.cuda.Stream(device=local)
-    flags = (8 if args.no_grid_stride else 0) | {"auto": 0, "global": 16, "tma": 32}[args.tile_desc]
+    flags = (8 if args.no_grid_stride else 0) | {"auto": 0, "global": 16, "tma": 32, "resident": 512}[args.tile_desc]
     sim = gs.Sim(prog, lanes, lane_offset=lane_offset, kernel=args.kernel, device=local, stream=stream,
                  lut_unroll=args.lut_unroll, pdl=not args.no_pdl, tile_words=args.tile_words,
                  tile_groups=args.tile_groups, lane_groups=args.lane_groups, flags=flags,
@@ -523,7 +523,10 @@ def main():
                        "compile_s": round(compile_s, 2), "build_id": gs.build_id(),
                        "program_hash": str(info["program_hash"]),
                        "paper_style_gcps": value * (G + info["n_reg"]) / G},
-            "gpu_launches": int(launches_per_cycle * (1 if args.kernel in ("tile", "cluster") else C) * args.steps * subs),
+            # per cycle: stim + level launches + end-of-cycle (kernels T / C: one launch per step);
+            # sharded: per sub-batch also the reset's 3 row fills and the signature's k_lane_sigs
+            "gpu_launches": int(args.steps * subs * (launches_per_cycle * (1 if args.kernel in ("tile", "cluster") else C)
+                                                     + (4 if sharded else 0))),
             "signature": {k: str(v) for k, v in red.items()},
             "nccl": ({"nranks": nranks, "ok": nranks == world} if nranks is not None else None),
             "clocks": clk,

@@ -279,11 +279,12 @@ typedef struct {
 /* flags: kernel A launches one CTA per work chunk instead of a grid-stride grid sized to
  * the resident capacity (A/B measurement only). */
 #define GS_SIM_NO_GRID_STRIDE 8u
-/* flags (kernel T): force the descriptor source — global memory (L2), or a TMA bulk-copy
- * stream of one level at a time into a shared-memory double buffer.  Default: resident in
- * shared memory if the whole table fits, else the TMA stream, else global. */
+/* flags (kernel T): force the descriptor source — global memory (L1/L2), a TMA bulk-copy
+ * stream of <= 256 descriptors per step into a shared-memory double buffer, or the whole
+ * table resident in shared memory.  Default: the planner's choice (sim.cpp make_plans). */
 #define GS_SIM_TILE_DESC_GLOBAL 16u
 #define GS_SIM_TILE_DESC_TMA 32u
+#define GS_SIM_TILE_DESC_RESIDENT 512u   /* force the resident table (A/B measurement)        */
 /* Retired in 0.2.0 (measured slower, DESIGN.md §6 "removed"): flag bits 2, 4 (L2 eviction
  * hints), 64, 128 (bulk-copy gathers) and 256 (kernel T slots in global memory) are rejected
  * with GS_ERR_ARG. */

@@ -29,6 +29,7 @@ GS_SIM_NO_PDL = 1
 GS_SIM_NO_GRID_STRIDE = 8     # kernel A: one CTA per work chunk (A/B measurement only)
 GS_SIM_TILE_DESC_GLOBAL = 16  # kernel T: descriptors read from global memory
 GS_SIM_TILE_DESC_TMA = 32     # kernel T: descriptors TMA-streamed level by level
+GS_SIM_TILE_DESC_RESIDENT = 512  # kernel T: descriptor table resident in shared memory
 GS_KERNEL_AUTO, GS_KERNEL_LUT, GS_KERNEL_POLY, GS_KERNEL_AB, GS_KERNEL_TILE, GS_KERNEL_CLUSTER = 0, 1, 2, 3, 5, 6
 KERNELS = {"auto": 0, "lut": 1, "A": 1, "poly": 2, "B": 2, "ab": 3, "AB": 3, "tile": 5, "T": 5,
            "cluster": 6, "C": 6}

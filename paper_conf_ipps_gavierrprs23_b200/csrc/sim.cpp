@@ -64,11 +64,11 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
         return fail(GS_ERR_ARG, "TILE: lanes must be a multiple of 32 * tile_words");
     // choose (descriptor mode, tile words, groups per CTA).  Kernel T is latency-bound per
     // tile (a level barrier per step), so a launch takes ~ waves x tile time with waves =
-    // ceil(tiles / (groups x SMs)): score = lanes per wave (quantisation included), resident
-    // descriptors weighted 4/3 over a TMA stream, then wider tiles, then resident > TMA stream
-    // > global, then fewer groups (more threads per tile).  C2 (256 live slots): 2 groups x 2,048-lane tiles with the
+    // ceil(tiles / (groups x SMs)): score = lanes per wave (quantisation included) x a
+    // descriptor-source weight, then more SMs busy, then wider tiles, then fewer groups.  C2 (256 live slots): 2 groups x 2,048-lane tiles with the
     // small descriptor table read through L1/L2, 3.18e13 (profiles/r02_kernelT_configs_C2.txt)
-    const int forced = (o.flags & GS_SIM_TILE_DESC_GLOBAL) ? 0 : (o.flags & GS_SIM_TILE_DESC_TMA) ? 2 : -1;
+    const int forced = (o.flags & GS_SIM_TILE_DESC_GLOBAL) ? 0 : (o.flags & GS_SIM_TILE_DESC_TMA) ? 2
+                       : (o.flags & GS_SIM_TILE_DESC_RESIDENT) ? 1 : -1;
     uint64_t best = 0;
     for (int ds : {1, 2, 0}) {
         if (forced >= 0 && ds != forced) continue;
@@ -83,13 +83,14 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
                 const uint64_t slots = (uint64_t)ng * (uint64_t)sms;
                 const uint64_t waves = (tiles + slots - 1) / slots;
                 const uint64_t per_wave = o.lanes / waves;
-                // descriptor source weights (measured on C2, 2,048-lane tiles): resident 2.56e13
-                // vs TMA-streamed 1.92e13 (1 group); with 2 groups, global (L1/L2-cached) 3.18e13
-                // vs TMA 3.04e13 — a small table (<= 128 KB) stays cache-resident, a large one
-                // is better streamed (mid-size circuits, round 1)
+                // descriptor source weights (profiles/r02_kernelT_configs_C2.txt,
+                // r02_mid_size_kernelT.txt): a small table (<= 128 KB) read through L1/L2 beats the
+                // same table resident in shared memory (5k gates: 9.5e12 vs 5.1e12 at 512-lane
+                // tiles; C2 2 groups 3.4e13) — the descriptor reads stay off the shared-memory
+                // port the slots saturate; a large table is best TMA-streamed (10k gates)
                 const bool small_table = (uint64_t)p.n_eval * 16 <= 131072;
-                const uint64_t wgt = ds == 1 ? 40 : ds == 2 ? 30 : small_table ? 32 : 28;
-                const uint64_t pref = ds == 1 ? 2 : ds == 2 ? 1 : 0;
+                const uint64_t wgt = ds == 0 ? (small_table ? 40 : 28) : ds == 1 ? 36 : 32;
+                const uint64_t pref = ds == 0 && small_table ? 3 : ds == 1 ? 2 : ds == 2 ? 1 : 0;
                 // ties (e.g. every plan fits one wave): more SMs busy, then wider tiles (C1,
                 // 1,024 lanes: 8 tiles of 128 lanes 1.03e10 vs one 1,024-lane tile 7.8e9)
                 const uint64_t busy = std::min<uint64_t>((tiles + ng - 1) / ng, (uint64_t)sms);
@@ -485,7 +486,7 @@ static gs_status write_binding(gs_sim* s) {
 // flag bits of gs_sim_opts retired in 0.2.0 (L2 hints, bulk-copy gathers, global T slots)
 constexpr uint32_t GS_SIM_RETIRED_FLAGS = 2u | 4u | 64u | 128u | 256u;
 constexpr uint32_t GS_SIM_KNOWN_FLAGS = GS_SIM_NO_PDL | GS_SIM_NO_GRID_STRIDE | GS_SIM_TILE_DESC_GLOBAL |
-                                        GS_SIM_TILE_DESC_TMA;
+                                        GS_SIM_TILE_DESC_TMA | GS_SIM_TILE_DESC_RESIDENT;
 
 static gs_status check_opts(const gs_sim_opts* o, const char* fn) {
     if (o->lanes == 0 || o->lanes % 64) return fail(GS_ERR_ARG, std::string(fn) + ": lanes must be a positive multiple of 64");

@@ -21,6 +21,7 @@ def main():
     ap.add_argument("--gates", default="5000,10000,20000,40000")
     ap.add_argument("--flags", default="0,16,32")
     ap.add_argument("--tile-words", type=int, default=0)
+    ap.add_argument("--tile-groups", type=int, default=0)
     args = ap.parse_args()
     lanes, cycles = args.lanes, 50
     depth = {5000: 24, 10000: 28, 20000: 32, 40000: 36, 100000: 40, 200000: 44, 400000: 48}
@@ -35,7 +36,8 @@ def main():
         for kernel, flags in [("lut", 0)] + [("tile", int(f)) for f in args.flags.split(",")]:
             try:
                 sim = gs.Sim(prog, lanes, kernel=kernel, flags=flags,
-                             tile_words=args.tile_words if kernel == "tile" else 0)
+                             tile_words=args.tile_words if kernel == "tile" else 0,
+                             tile_groups=args.tile_groups if kernel == "tile" else 0)
             except gs.GsError as e:
                 print(json.dumps({"gates": G, "kernel": kernel, "flags": flags, "error": str(e)}), flush=True)
                 continue
@@ -49,7 +51,8 @@ def main():
             torch.cuda.synchronize()
             s = e0.elapsed_time(e1) / 1e3
             print(json.dumps({"gates": G, "lanes": lanes, "levels": prog.info["n_levels"], "slots": slots,
-                              "kernel": kernel, "flags": flags, "sgc_per_s": G * lanes * cycles * 2 / s}), flush=True)
+                              "kernel": kernel, "flags": flags, "sgc_per_s": G * lanes * cycles * 2 / s,
+                              "launch": sim.launch}), flush=True)
             sim.close()
 
 

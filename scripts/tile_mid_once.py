@@ -1,0 +1,38 @@
+#!/usr/bin/env python
+"""Kernel T on a mid-size synthetic circuit in a fresh process (no other kernel before it): 3 warm-up
+and 5 timed steps of --cycles cycles; --gates G --flags F --tw TW --ng NG.  Also the ncu target."""
+import argparse
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--gates", type=int, default=5000)
+ap.add_argument("--flags", type=int, default=0)
+ap.add_argument("--tw", type=int, default=0)
+ap.add_argument("--ng", type=int, default=0)
+ap.add_argument("--cycles", type=int, default=10)
+a = ap.parse_args()
+import workloads
+import paper_conf_ipps_gavierrprs23_b200 as gs
+depth = {5000: 24, 10000: 28, 20000: 32, 40000: 36}
+nl = workloads.synthetic(a.gates, a.gates // 25, 64, 64, depth.get(a.gates, 40), seed=a.gates, name="m")
+prog = gs.Netlist.from_arrays(nl).compile()
+sim = gs.Sim(prog, 65536, kernel="tile", flags=a.flags, tile_words=a.tw, tile_groups=a.ng)
+import json
+import torch
+sim.bind_generated(1)
+for _ in range(3):
+    sim.step(a.cycles)
+sim.sync()
+e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+e0.record(sim.stream)
+for _ in range(5):
+    sim.step(a.cycles)
+e1.record(sim.stream)
+torch.cuda.synchronize()
+s = e0.elapsed_time(e1) / 1e3
+print(json.dumps({"gates": a.gates, "flags": a.flags, "sgc_per_s": a.gates * 65536 * a.cycles * 5 / s,
+                  "launch": sim.launch}))
