@@ -226,7 +226,8 @@ def run_reference(args):
     nl = cfg.netlist()
     G = int((nl.gate_k > 0).sum())
     threads = oracle.max_threads()
-    sample = np.linspace(0, cfg.lanes - 1, threads).astype(np.int64)
+    # 16 lanes per thread: the oracle advances lanes in 16-lane blocks, one block per thread
+    sample = np.linspace(0, cfg.lanes - 1, 16 * threads).astype(np.int64)
     cps = args.cycles_per_step or (cfg.cycles if cfg.shards > 1 else 100)
     # per step: every thread simulates one lane for c cycles from reset; size c so the whole
     # run is a few minutes

@@ -1,6 +1,7 @@
 #!/usr/bin/env python
-"""Kernel T on a mid-size synthetic circuit in a fresh process (no other kernel before it): 3 warm-up
-and 5 timed steps of --cycles cycles; --gates G --flags F --tw TW --ng NG.  Also the ncu target."""
+"""Kernel T on a mid-size synthetic circuit in a fresh process: ~1 s of warm-up steps (the GPU
+clock ramps from idle), then ~1 s of timed steps of --cycles cycles; --gates G --flags F --tw TW
+--ng NG.  Also an ncu target."""
 import argparse
 import os
 import sys
@@ -22,17 +23,26 @@ nl = workloads.synthetic(a.gates, a.gates // 25, 64, 64, depth.get(a.gates, 40),
 prog = gs.Netlist.from_arrays(nl).compile()
 sim = gs.Sim(prog, 65536, kernel="tile", flags=a.flags, tile_words=a.tw, tile_groups=a.ng)
 import json
+import time
 import torch
 sim.bind_generated(1)
-for _ in range(3):
+# warm the GPU up for ~1 s (clocks ramp from idle), then time ~1 s of steps
+t = time.time()
+while time.time() - t < 1.0:
     sim.step(a.cycles)
-sim.sync()
+    sim.sync()
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 e0.record(sim.stream)
-for _ in range(5):
+e1.record(sim.stream)
+e1.synchronize()
+n = 0
+e0.record(sim.stream)
+t = time.time()
+while time.time() - t < 1.0:
     sim.step(a.cycles)
+    n += 1
 e1.record(sim.stream)
 torch.cuda.synchronize()
 s = e0.elapsed_time(e1) / 1e3
-print(json.dumps({"gates": a.gates, "flags": a.flags, "sgc_per_s": a.gates * 65536 * a.cycles * 5 / s,
-                  "launch": sim.launch}))
+print(json.dumps({"gates": a.gates, "flags": a.flags, "sgc_per_s": a.gates * 65536 * a.cycles * n / s,
+                  "steps": n, "launch": sim.launch}))

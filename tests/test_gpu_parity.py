@@ -812,6 +812,13 @@ def test_auto_kernel_selection():
         prog = gs.Netlist.from_arrays(workloads.CONFIGS[name].netlist()).compile(lut_k=L)
         sim = gs.Sim(prog, lanes, kernel="auto")
         assert (sim.launches_per_cycle() == 1) == tile, name
+        li = sim.launch                                   # gs_sim_get_launch: the resolved plan
+        assert li["kernel"] == (gs.GS_KERNEL_TILE if tile else gs.GS_KERNEL_LUT), (name, li)
+        if tile:
+            assert li["tile_words"] in (4, 8, 16, 32, 64) and li["grid"] >= 1 and li["live_slots"] > 0
+            assert li["tile_groups"] in (1, 2, 4) and li["tile_desc"] in (0, 1, 2)
+        else:
+            assert li["lane_groups"] == sim.config["lane_groups"] >= 1
         sim.bind_generated(1)
         sim.step(2)
         ref = run_gpu(workloads.CONFIGS[name].netlist(), lanes, 2, "lut", seed=1, prog=prog)
