@@ -8,9 +8,10 @@ mkdir -p $OUT
 SAN="-fsanitize=address,undefined -fno-omit-frame-pointer -fno-sanitize-recover=undefined -g -O1"
 ARCH="-gencode arch=compute_100a,code=sm_100a"
 objs=""
+BID=$(python -c "import paper_conf_ipps_gavierrprs23_b200._build as b; print(b.build_id())")
 for f in paper_conf_ipps_gavierrprs23_b200/csrc/*.cpp; do
   o=$OUT/$(basename $f).o
-  g++ -std=c++17 -Iinclude -I/usr/local/cuda/include -fPIC $SAN -c $f -o $o
+  g++ -std=c++17 -Iinclude -I/usr/local/cuda/include -fPIC $SAN -DGS_BUILD_ID=\"$BID\" -c $f -o $o
   objs="$objs $o"
 done
 for f in paper_conf_ipps_gavierrprs23_b200/csrc/*.cu; do
