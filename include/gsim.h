@@ -349,7 +349,8 @@ typedef struct {
     int kernel;                   /* GS_KERNEL_* (AUTO resolved)                            */
     uint32_t lane_groups;         /* kernel A: concurrent lane groups                       */
     uint32_t tile_words, tile_groups, tile_desc;   /* kernel T: words per slot, thread groups
-                                     per CTA, descriptor source (0 global, 1 resident, 2 TMA) */
+                                     per CTA, descriptor source (0 global, 1 resident, 2 TMA;
+                                     | 4: narrow 8-byte descriptors, k <= 2 and no registers) */
     uint32_t grid;                /* kernels T / C: CTAs launched per step                  */
     uint32_t cluster_size, slab_lanes;             /* kernel C                                 */
     uint32_t live_slots;          /* kernel T: shared-memory slots per tile                 */

@@ -130,6 +130,10 @@ static_assert(sizeof(TileDesc) == 16, "TileDesc layout");
 struct TilePlan {
     uint32_t n_slots = 0, q0 = 0;
     std::vector<TileDesc> desc;         // [n_eval] exec order
+    // narrow 8-byte descriptors {in0 | in1 << 16, tt[15:0] | out << 16}, built when every gate
+    // has k <= 2, the program has no registers and no gate has k > 4 (C1, C2: half the
+    // descriptor bytes, so the table fits L1 or shared memory next to more slots)
+    std::vector<uint32_t> desc_n;       // [n_eval][2]
     std::vector<uint32_t> desc_hi;      // [n_eval][12] if any k > 4: in4|in5<<16, in6|in7<<16, 0, 0,
                                         //   then the 256-bit table as 8 words
     std::vector<uint32_t> po_slot;      // [n_po]

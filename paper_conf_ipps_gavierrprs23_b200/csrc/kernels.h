@@ -81,7 +81,8 @@ struct TileArgs {
                                       // (chunks of <= TILE_CHUNK gates when TMA-streamed)
     uint32_t n_eval, n_steps;
     uint32_t desc_smem;               // 0: descriptors read from global; 1: resident in shared
-                                      // memory; 2: TMA-streamed step by step (double buffer)
+                                      // memory; 2: TMA-streamed step by step (double buffer);
+                                      // | 4: narrow 8-byte descriptors (desc points at them)
     const uint32_t* po_slot;
     uint32_t n_po;
     const uint32_t* latch_src;
@@ -111,7 +112,7 @@ constexpr uint32_t STEP_N_MASK = 0xFFFFFFu;
 void tile_steps(const uint32_t* level_off, uint32_t n_levels, const GateAux* aux, uint32_t chunk,
                 std::vector<uint2>& out);
 size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_steps,
-                       int desc_mode);
+                       int desc_mode);   // desc_mode | 4: narrow descriptors
 cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_steps,
                        int desc_smem, uint32_t has_q, uint32_t* per_sm);
 cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s);

@@ -23,8 +23,10 @@ void tile_steps(const uint32_t* level_off, uint32_t n_levels, const GateAux* aux
 
 size_t tile_smem_bytes(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_eval, uint32_t n_steps,
                        int desc_mode) {
+    const size_t dbytes = (desc_mode & 4) ? 8 : 16;        // narrow descriptors: 8 bytes
+    desc_mode &= 3;
     size_t b = ((size_t)n_steps + 1) / 2 * 16;
-    if (desc_mode == 1) b += (size_t)n_eval * 16;
+    if (desc_mode == 1) b += ((size_t)n_eval * dbytes + 15) / 16 * 16;
     const size_t g = 32 + (desc_mode == 2 ? 2 * (size_t)TILE_CHUNK * 16 : 0) + ((size_t)n_slots + 64) * 4 * tw;
     return b + (size_t)ng * g;
 }

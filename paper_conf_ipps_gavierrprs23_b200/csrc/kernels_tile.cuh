@@ -17,6 +17,8 @@
 // lane signatures, outputs, registers and the trace are bit-identical.
 #pragma once
 
+#include <type_traits>
+
 #include <cuda_runtime.h>
 
 #include "device.cuh"
@@ -127,14 +129,18 @@ __device__ __forceinline__ void tile_gate(uint4* sl, uint32_t V, uint32_t v, uin
     }
 }
 
+// a descriptor as the 16-byte form (narrow descriptors: inputs 0-1, table and output slot)
+__device__ __forceinline__ uint4 as_desc4(const uint4& d) { return d; }
+__device__ __forceinline__ uint4 as_desc4(const uint2& d) { return make_uint4(d.x, 0u, d.y, 0u); }
+
 // All (gate, vector group) units of one step, every gate with fan-in K.
-template <int K, bool HASQ, int P, uint32_t VS, uint32_t VSH, uint32_t GT>
-__device__ __forceinline__ void tile_step(uint4* sl, uint32_t V, const uint4* dl, uint32_t g0, uint32_t n,
+template <int K, bool HASQ, int P, uint32_t VS, uint32_t VSH, uint32_t GT, typename DT>
+__device__ __forceinline__ void tile_step(uint4* sl, uint32_t V, const DT* dl, uint32_t g0, uint32_t n,
                                           uint32_t tid, const uint4* desc_hi, uint32_t q0, uint32_t R) {
 #pragma unroll 1
     for (uint32_t u = tid; u < n; u += GT) {
         const uint32_t gi = u >> VSH, v = u & (VS - 1);
-        tile_gate<K, HASQ, P>(sl, V, v, VS, dl[gi], desc_hi, g0 + gi, q0, R);
+        tile_gate<K, HASQ, P>(sl, V, v, VS, as_desc4(dl[gi]), desc_hi, g0 + gi, q0, R);
     }
 }
 
@@ -156,9 +162,13 @@ __device__ __forceinline__ void group_sync(uint32_t id, uint32_t nthreads) {
 // buffer while chunk t is evaluated).  Every step ends with the group barrier.  Everything
 // loop-invariant (Ctl fields, shared-memory addresses) is read once per launch, so a step
 // costs a handful of instructions besides its gates.
-template <int TW, bool HASQ, int NG, int DM>
+template <int TW, bool HASQ, int NG, int DMN>
 __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
-    // DM: descriptor mode (0 global, 1 resident, 2 TMA-streamed chunks)
+    // DM: descriptor mode (0 global, 1 resident, 2 TMA-streamed chunks); DMN | 4: narrow 8-byte
+    // descriptors (k <= 2, no registers)
+    constexpr int DM = DMN & 3;
+    constexpr bool NARROW = (DMN & 4) != 0;
+    using DT = typename std::conditional<NARROW, uint2, uint4>::type;
     constexpr uint32_t V = TW / 4;                       // uint4 per slot
     constexpr uint32_t P = V >= 4 ? TILE_VPT : 1;        // 16-byte vectors per thread and gate
     constexpr uint32_t VS = V / P;                       // threads per gate (vector stride)
@@ -171,9 +181,10 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     //                      (DM 2)] [slots: n_slots x V uint4] [MISR: 64 x V uint4]
     uint4* base = smem;
     if (DM == 1) {
-        const uint4* gd = reinterpret_cast<const uint4*>(a.desc);
-        for (uint32_t i = threadIdx.x; i < a.n_eval; i += blockDim.x) smem[i] = __ldg(gd + i);
-        base += a.n_eval;
+        const DT* gd = reinterpret_cast<const DT*>(a.desc);
+        DT* sd = reinterpret_cast<DT*>(smem);
+        for (uint32_t i = threadIdx.x; i < a.n_eval; i += blockDim.x) sd[i] = __ldg(gd + i);
+        base += ((size_t)a.n_eval * sizeof(DT) + 15) / 16;
     }
     uint2* steps = reinterpret_cast<uint2*>(base);
     for (uint32_t i = threadIdx.x; i < a.n_steps; i += blockDim.x) steps[i] = __ldg(a.steps + i);
@@ -185,7 +196,7 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     volatile uint32_t* tile_slot = reinterpret_cast<volatile uint32_t*>(greg + 1);
     uint4* dbuf = greg + 2;                                   // DM 2: [2][TILE_CHUNK]
     uint4* sl = greg + 2 + (DM == 2 ? 2 * TILE_CHUNK : 0);    // slots
-    const uint4* dsm = DM == 1 ? smem : reinterpret_cast<const uint4*>(a.desc);
+    const DT* dsm = DM == 1 ? reinterpret_cast<const DT*>(smem) : reinterpret_cast<const DT*>(a.desc);
     if (DM == 2 && tid == 0) {
         mbar_init(mbar, 1);
         mbar_init(mbar + 1, 1);
@@ -222,7 +233,8 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
     group_sync(bar, GT);                                  // every thread has read it before the next claim
     if (DM == 2 && tid == 0 && tile < a.n_tiles && n_steps) {
         const uint2 s0 = steps[0];
-        tma_load_1d(dbuf_s, a.desc + s0.x, (s0.y & STEP_N_MASK) * 16, mbar_s);
+        tma_load_1d(dbuf_s, reinterpret_cast<const DT*>(a.desc) + s0.x, (s0.y & STEP_N_MASK) * (uint32_t)sizeof(DT),
+                    mbar_s);
     }
     while (tile < a.n_tiles) {
         // claim the next tile now, so the descriptor stream knows whether to continue
@@ -264,16 +276,16 @@ __global__ void __launch_bounds__(TILE_CTA, 1) k_tile(TileArgs a) {
             for (uint32_t si = 0; si < n_steps; ++si) {
                 const uint2 st = steps[si];
                 const uint32_t sn_gates = st.y & STEP_N_MASK;
-                const uint4* dl = dsm + st.x;
+                const DT* dl = dsm + st.x;
                 if (DM == 2) {
                     const uint32_t b = step & 1;
                     if (tid == 0 && (si + 1 < n_steps || more)) {
                         const uint2 sn = steps[si + 1 < n_steps ? si + 1 : 0];
-                        tma_load_1d(dbuf_s + (b ^ 1) * (TILE_CHUNK * 16), a.desc + sn.x, (sn.y & STEP_N_MASK) * 16,
-                                    mbar_s + 8 * (b ^ 1));
+                        tma_load_1d(dbuf_s + (b ^ 1) * (TILE_CHUNK * 16), reinterpret_cast<const DT*>(a.desc) + sn.x,
+                                    (sn.y & STEP_N_MASK) * (uint32_t)sizeof(DT), mbar_s + 8 * (b ^ 1));
                     }
                     mbar_wait(mbar_s + 8 * b, (step >> 1) & 1);
-                    dl = dbuf + b * TILE_CHUNK;
+                    dl = reinterpret_cast<const DT*>(dbuf + b * TILE_CHUNK);
                     ++step;
                 }
                 // every gate of a step has the same fan-in k (steps are cut at k changes), so the

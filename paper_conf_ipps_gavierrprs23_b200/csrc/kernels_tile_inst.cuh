@@ -13,10 +13,21 @@
         case 2: CALL(TW, Q, G, 2); break;       \
         default: return cudaErrorInvalidValue;  \
     }
+/* programs without registers may also use narrow descriptors (mode | 4) */
+#define GS_TILE_DMN(TW, G, CALL)                \
+    switch (dm) {                               \
+        case 0: CALL(TW, false, G, 0); break;   \
+        case 1: CALL(TW, false, G, 1); break;   \
+        case 2: CALL(TW, false, G, 2); break;   \
+        case 4: CALL(TW, false, G, 4); break;   \
+        case 5: CALL(TW, false, G, 5); break;   \
+        case 6: CALL(TW, false, G, 6); break;   \
+        default: return cudaErrorInvalidValue;  \
+    }
 #define GS_TILE_QG(TW, CALL)                                                                        \
     switch ((has_q ? 8 : 0) + (ng == 1 ? 0 : ng == 2 ? 1 : ng == 4 ? 2 : 7)) {                      \
-        case 0: GS_TILE_DM(TW, false, 1, CALL) break; case 1: GS_TILE_DM(TW, false, 2, CALL) break; \
-        case 2: GS_TILE_DM(TW, false, 4, CALL) break; case 8: GS_TILE_DM(TW, true, 1, CALL) break;  \
+        case 0: GS_TILE_DMN(TW, 1, CALL) break; case 1: GS_TILE_DMN(TW, 2, CALL) break;             \
+        case 2: GS_TILE_DMN(TW, 4, CALL) break; case 8: GS_TILE_DM(TW, true, 1, CALL) break;        \
         case 9: GS_TILE_DM(TW, true, 2, CALL) break;  case 10: GS_TILE_DM(TW, true, 4, CALL) break; \
         default: return cudaErrorInvalidValue;                                                      \
     }

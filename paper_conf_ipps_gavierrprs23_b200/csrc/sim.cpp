@@ -32,6 +32,7 @@ struct Plans {
     uint32_t tw = 0;                  // kernel T: 32-bit words per slot
     uint32_t ng = 0;                  // kernel T: thread groups (tiles) per CTA
     int desc_smem = 0;                // kernel T: descriptors 0 global, 1 resident, 2 TMA-streamed
+                                      //   (| 4: narrow 8-byte descriptors)
     std::vector<uint2> steps;         // kernel T: level steps (chunks when TMA-streamed)
 };
 
@@ -69,6 +70,8 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
     // small descriptor table read through L1/L2, 3.18e13 (profiles/r02_kernelT_configs_C2.txt)
     const int forced = (o.flags & GS_SIM_TILE_DESC_GLOBAL) ? 0 : (o.flags & GS_SIM_TILE_DESC_TMA) ? 2
                        : (o.flags & GS_SIM_TILE_DESC_RESIDENT) ? 1 : -1;
+    const bool narrow = !pl.tile.desc_n.empty();              // 8-byte descriptors (tile.cpp)
+    const uint64_t table_bytes = (uint64_t)p.n_eval * (narrow ? 8 : 16);
     uint64_t best = 0;
     for (int ds : {1, 2, 0}) {
         if (forced >= 0 && ds != forced) continue;
@@ -78,19 +81,20 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
             for (uint32_t tw : {4u, 8u, 16u, 32u, 64u}) {
                 if (o.tile_words && tw != o.tile_words) continue;
                 if (o.lanes % (32ull * tw)) continue;
-                if (tile_smem_bytes(tw, ng, pl.tile.n_slots, p.n_eval, nsteps, ds) > TILE_SMEM_MAX) continue;
+                if (tile_smem_bytes(tw, ng, pl.tile.n_slots, p.n_eval, nsteps, ds | (narrow ? 4 : 0)) > TILE_SMEM_MAX)
+                    continue;
                 const uint64_t tiles = o.lanes / (32ull * tw);
                 const uint64_t slots = (uint64_t)ng * (uint64_t)sms;
                 const uint64_t waves = (tiles + slots - 1) / slots;
                 const uint64_t per_wave = o.lanes / waves;
                 // descriptor source weights (profiles/r02_kernelT_configs_C2.txt,
-                // r02_mid_size_kernelT.txt): a small table (<= 128 KB) read through L1/L2 beats the
-                // same table resident in shared memory (5k gates: 9.5e12 vs 5.1e12 at 512-lane
-                // tiles; C2 2 groups 3.4e13) — the descriptor reads stay off the shared-memory
-                // port the slots saturate; a large table is best TMA-streamed (10k gates)
-                const bool small_table = (uint64_t)p.n_eval * 16 <= 131072;
-                const uint64_t wgt = ds == 0 ? (small_table ? 40 : 28) : ds == 1 ? 36 : 32;
-                const uint64_t pref = ds == 0 && small_table ? 3 : ds == 1 ? 2 : ds == 2 ? 1 : 0;
+                // r02_mid_size_fresh_process.jsonl): resident >= a small table (<= 128 KB) read
+                // through L1/L2 (C2, narrow descriptors, 2 groups: 3.86e13 vs 3.65e13; 5k gates,
+                // 512-lane tiles: 6.31e12 vs 6.27e12) > TMA stream (3.21e13; 5.0e12) > a large
+                // table from L2 (10k gates: TMA 7.1e12 vs global 6.3e12)
+                const bool small_table = table_bytes <= 131072;
+                const uint64_t wgt = ds == 1 ? 40 : ds == 0 ? (small_table ? 38 : 28) : 32;
+                const uint64_t pref = ds == 1 ? 3 : ds == 0 && small_table ? 2 : ds == 2 ? 1 : 0;
                 // ties (e.g. every plan fits one wave): more SMs busy, then wider tiles (C1,
                 // 1,024 lanes: 8 tiles of 128 lanes 1.03e10 vs one 1,024-lane tile 7.8e9)
                 const uint64_t busy = std::min<uint64_t>((tiles + ng - 1) / ng, (uint64_t)sms);
@@ -102,6 +106,7 @@ gs_status make_plans(const Program& p, const gs_sim_opts& o, Plans& pl) {
     }
     if (!best) return fail(GS_ERR_ARG, "TILE: live state of a 128-lane tile exceeds shared memory (or lanes % 128)");
     pl.steps = pl.desc_smem == 2 ? st_chunk : st_level;
+    if (narrow) pl.desc_smem |= 4;
     return GS_OK;
 }
 
@@ -127,7 +132,8 @@ gs_sim_opts resolve_auto(const Program& p, const gs_sim_opts& o) {
     const std::string saved = gs_last_error();
     // (a large descriptor table read from global memory is slow: T only with resident or
     // TMA-streamed descriptors, or a table small enough to stay cache-resident)
-    if (p.n_eval == 0 || make_plans(p, r, pl) != GS_OK || (pl.desc_smem == 0 && (uint64_t)p.n_eval * 16 > 131072))
+    if (p.n_eval == 0 || make_plans(p, r, pl) != GS_OK ||
+        ((pl.desc_smem & 3) == 0 && (uint64_t)p.n_eval * ((pl.desc_smem & 4) ? 8 : 16) > 131072))
         r.kernel = GS_KERNEL_LUT;
     set_error(saved);
     return r;
@@ -162,7 +168,7 @@ Layout make_layout(const Program& p, const gs_sim_opts& o, const Plans& pl) {
     L.trace = take((size_t)o.trace_cycles * p.n_po * o.n_trace_words * 8);
     L.lane_sigs = take((size_t)o.lanes * 8);
     L.scratch = take((size_t)p.n_po * words * 8);
-    L.t_desc = take(t.desc.size() * sizeof(TileDesc));
+    L.t_desc = take(t.desc_n.empty() ? t.desc.size() * sizeof(TileDesc) : t.desc_n.size() * 4);
     L.t_desc_hi = take(t.desc_hi.size() * 4);   // 48 B per gate when any k > 4
     L.t_po = take(t.po_slot.size() * 4);
     L.t_lsrc = take(t.latch_src.size() * 4);
@@ -617,7 +623,8 @@ static gs_status sim_create(const gs_program* prog, const gs_sim_opts* opts_in, 
         {L.latch_dst, p.latch_dst.data(), p.latch_dst.size() * 4},
         {L.reg_init, p.reg_init.data(), p.reg_init.size()},
         {L.trace_slot, slot.data(), slot.size() * 4},
-        {L.t_desc, s->tile.desc.data(), s->tile.desc.size() * sizeof(TileDesc)},
+        {L.t_desc, s->tile.desc_n.empty() ? (const void*)s->tile.desc.data() : (const void*)s->tile.desc_n.data(),
+         s->tile.desc_n.empty() ? s->tile.desc.size() * sizeof(TileDesc) : s->tile.desc_n.size() * 4},
         {L.t_desc_hi, s->tile.desc_hi.data(), s->tile.desc_hi.size() * 4},
         {L.t_po, s->tile.po_slot.data(), s->tile.po_slot.size() * 4},
         {L.t_lsrc, s->tile.latch_src.data(), s->tile.latch_src.size() * 4},

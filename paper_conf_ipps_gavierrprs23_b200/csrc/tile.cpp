@@ -95,6 +95,13 @@ gs_status tile_plan(const Program& p, TilePlan& t) {
             }
         }
     }
+    if (p.max_k <= 2 && p.n_reg == 0 && !p.any_wide) {
+        t.desc_n.resize((size_t)G * 2);
+        for (uint32_t g = 0; g < G; ++g) {
+            t.desc_n[2 * (size_t)g] = t.desc[g].in01;
+            t.desc_n[2 * (size_t)g + 1] = t.desc[g].tt;
+        }
+    }
     for (uint32_t r : p.po_rows) t.po_slot.push_back(slot_of(r));
     for (size_t i = 0; i < p.latch_src.size(); ++i) {
         t.latch_src.push_back(slot_of(p.latch_src[i]));

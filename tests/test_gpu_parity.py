@@ -816,7 +816,8 @@ def test_auto_kernel_selection():
         assert li["kernel"] == (gs.GS_KERNEL_TILE if tile else gs.GS_KERNEL_LUT), (name, li)
         if tile:
             assert li["tile_words"] in (4, 8, 16, 32, 64) and li["grid"] >= 1 and li["live_slots"] > 0
-            assert li["tile_groups"] in (1, 2, 4) and li["tile_desc"] in (0, 1, 2)
+            assert li["tile_groups"] in (1, 2, 4) and li["tile_desc"] & 3 in (0, 1, 2)
+            assert bool(li["tile_desc"] & 4) == (name in ("C1", "C2") and L == 0)   # narrow: k <= 2, no regs
         else:
             assert li["lane_groups"] == sim.config["lane_groups"] >= 1
         sim.bind_generated(1)
