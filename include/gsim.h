@@ -389,6 +389,8 @@ typedef struct {
     uint64_t grid_stride_launches;  /* kernel A level launches (host launch decisions; with lane
                                        groups one per captured graph) whose grid was capped at
                                        the resident CTA capacity, grid-striding over the level */
+    uint64_t multi_gate_launches;   /* kernel A level launches (counted likewise) whose warp
+                                       units hold several gates (rows < 16,384 lanes) */
 } gs_profile;
 gs_status gs_sim_profile_step(gs_sim* sim, uint32_t ncycles, gs_profile* out);
 

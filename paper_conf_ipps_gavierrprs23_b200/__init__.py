@@ -99,7 +99,7 @@ class gs_launch_info(C.Structure):
 class gs_profile(C.Structure):
     _fields_ = [("level_ms", C.c_double), ("total_ms", C.c_double), ("level_launches", C.c_uint64),
                 ("total_launches", C.c_uint64), ("level_bytes", C.c_double),
-                ("grid_stride_launches", C.c_uint64)]
+                ("grid_stride_launches", C.c_uint64), ("multi_gate_launches", C.c_uint64)]
 
 
 # ------------------------------------------------------------------ loading

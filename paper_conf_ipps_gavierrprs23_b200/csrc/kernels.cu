@@ -180,11 +180,55 @@ __device__ __forceinline__ void lut_gate_u(const LevelArgs& a, uint32_t gate, ui
     }
 }
 
+// One gate x U*32 vectors of any fan-in (the body of a kernel A warp unit).
+template <int U>
+__device__ __forceinline__ void lut_gate_any(const LevelArgs& a, uint32_t gate, uint4 in, uint4 au, uint32_t v0) {
+    const uint64_t tt = ((uint64_t)au.y << 32) | au.x;
+    const uint32_t qdst = au.z, k = au.w & 0xFFu;
+    switch (k) {
+        case 1: lut_gate_u<1, U>(a, gate, in, v0, tt, qdst); break;
+        case 2: lut_gate_u<2, U>(a, gate, in, v0, tt, qdst); break;
+        case 3: lut_gate_u<3, U>(a, gate, in, v0, tt, qdst); break;
+        case 4: lut_gate_u<4, U>(a, gate, in, v0, tt, qdst); break;
+        case 5: lut_gate_u<5, 1>(a, gate, in, v0, tt, qdst);
+                if (U > 1) lut_gate_u<5, 1>(a, gate, in, v0 + 32, tt, qdst);
+                if (U > 2) { lut_gate_u<5, 1>(a, gate, in, v0 + 64, tt, qdst);
+                             lut_gate_u<5, 1>(a, gate, in, v0 + 96, tt, qdst); }
+                if (U > 4)
+                    for (int u = 4; u < U; ++u) lut_gate_u<5, 1>(a, gate, in, v0 + 32 * u, tt, qdst);
+                break;
+        case 6: lut_gate_u<6, 1>(a, gate, in, v0, tt, qdst);
+                if (U > 1) lut_gate_u<6, 1>(a, gate, in, v0 + 32, tt, qdst);
+                if (U > 2) { lut_gate_u<6, 1>(a, gate, in, v0 + 64, tt, qdst);
+                             lut_gate_u<6, 1>(a, gate, in, v0 + 96, tt, qdst); }
+                if (U > 4)
+                    for (int u = 4; u < U; ++u) lut_gate_u<6, 1>(a, gate, in, v0 + 32 * u, tt, qdst);
+                break;
+        case 7:
+#pragma unroll 1
+                for (int u = 0; u < U; ++u) lut_gate_big<7, uint4>(a, gate, in, v0 + 32 * u, qdst);
+                break;
+        default:
+#pragma unroll 1
+                for (int u = 0; u < U; ++u) lut_gate_big<8, uint4>(a, gate, in, v0 + 32 * u, qdst);
+                break;
+    }
+}
+
 // Grid-stride over warp units (gate, chunk of U*32 vectors): the grid is sized to the
 // resident capacity (148 SMs x CTAs per SM, a.grid_blocks), so no level ends with a
 // partially filled wave of CTAs.
 #ifndef GS_U1_MINB
 #define GS_U1_MINB 4
+#endif
+#ifndef GS_LUT_GP
+#define GS_LUT_GP 1
+#endif
+#ifndef GS_GP_MINB
+#define GS_GP_MINB 3
+#endif
+#ifndef GS_GP_VPT                 // gates x vectors per thread of a multi-gate warp unit
+#define GS_GP_VPT 4
 #endif
 template <int U>
 __global__ void __launch_bounds__(256, U > 4 ? 2 : U == 1 ? GS_U1_MINB : 4)
@@ -196,39 +240,80 @@ __global__ void __launch_bounds__(256, U > 4 ? 2 : U == 1 ? GS_U1_MINB : 4)
     for (uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; warp < total; warp += stride) {
         const uint32_t gi = warp >> cpg_shift;
         const uint32_t chunk = warp & ((1u << cpg_shift) - 1);
-        const uint32_t v0 = vec0 + chunk * 32 * U + lane;
         const uint32_t gate = a.g0 + gi;
-        const uint4 in = __ldg(a.din + gate);
-        const uint4 au = __ldg(reinterpret_cast<const uint4*>(a.aux) + gate);
-        const uint64_t tt = ((uint64_t)au.y << 32) | au.x;
-        const uint32_t qdst = au.z, k = au.w & 0xFFu;
-        switch (k) {
-            case 1: lut_gate_u<1, U>(a, gate, in, v0, tt, qdst); break;
-            case 2: lut_gate_u<2, U>(a, gate, in, v0, tt, qdst); break;
-            case 3: lut_gate_u<3, U>(a, gate, in, v0, tt, qdst); break;
-            case 4: lut_gate_u<4, U>(a, gate, in, v0, tt, qdst); break;
-            case 5: lut_gate_u<5, 1>(a, gate, in, v0, tt, qdst);
-                    if (U > 1) lut_gate_u<5, 1>(a, gate, in, v0 + 32, tt, qdst);
-                    if (U > 2) { lut_gate_u<5, 1>(a, gate, in, v0 + 64, tt, qdst);
-                                 lut_gate_u<5, 1>(a, gate, in, v0 + 96, tt, qdst); }
-                    if (U > 4)
-                        for (int u = 4; u < U; ++u) lut_gate_u<5, 1>(a, gate, in, v0 + 32 * u, tt, qdst);
-                    break;
-            case 6: lut_gate_u<6, 1>(a, gate, in, v0, tt, qdst);
-                    if (U > 1) lut_gate_u<6, 1>(a, gate, in, v0 + 32, tt, qdst);
-                    if (U > 2) { lut_gate_u<6, 1>(a, gate, in, v0 + 64, tt, qdst);
-                                 lut_gate_u<6, 1>(a, gate, in, v0 + 96, tt, qdst); }
-                    if (U > 4)
-                        for (int u = 4; u < U; ++u) lut_gate_u<6, 1>(a, gate, in, v0 + 32 * u, tt, qdst);
-                    break;
-            case 7:
-#pragma unroll 1
-                    for (int u = 0; u < U; ++u) lut_gate_big<7, uint4>(a, gate, in, v0 + 32 * u, qdst);
-                    break;
-            default:
-#pragma unroll 1
-                    for (int u = 0; u < U; ++u) lut_gate_big<8, uint4>(a, gate, in, v0 + 32 * u, qdst);
-                    break;
+        lut_gate_any<U>(a, gate, __ldg(a.din + gate), __ldg(reinterpret_cast<const uint4*>(a.aux) + gate),
+                        vec0 + chunk * 32 * U + lane);
+    }
+}
+
+// Short rows (< 4 x 32 vectors per lane group, i.e. < 16,384 lanes): a warp unit is GP
+// consecutive gates x U*32 vectors, with all GP*U*K input loads issued before any is used,
+// so a thread keeps as many bytes in flight as on 2 KB rows (GP*U = 4).  Gates are k-grouped
+// inside a level, so the GP gates share k except at a k-group edge (then one at a time).
+template <int K, int U, int GP>
+__device__ __forceinline__ void lut_gates_gp(const LevelArgs& a, uint32_t gate0, const uint4 (&in)[GP],
+                                             const uint4 (&au)[GP], uint32_t v0) {
+    uint4 x[GP][U][K];
+#pragma unroll
+    for (int g = 0; g < GP; ++g) {
+        const uint32_t r[4] = {in[g].x, in[g].y, in[g].z, in[g].w};
+#pragma unroll
+        for (int i = 0; i < K; ++i) {
+            const uint4* src = reinterpret_cast<const uint4*>(a.state + (uint64_t)resolve(r[i], a.qcur) * a.stride) + v0;
+#pragma unroll
+            for (int u = 0; u < U; ++u) x[g][u][i] = __ldg(src + u * 32);
+        }
+    }
+#pragma unroll
+    for (int g = 0; g < GP; ++g) {
+        const uint64_t tt = ((uint64_t)au[g].y << 32) | au[g].x;
+        const uint32_t qdst = au[g].z;
+        uint4* dst = reinterpret_cast<uint4*>(a.state + (uint64_t)(a.row_gate0 + gate0 + g) * a.stride) + v0;
+        const bool latch = qdst != 0xFFFFFFFFu;
+        uint4* qd = reinterpret_cast<uint4*>(a.state + (uint64_t)((latch ? qdst : 0u) + a.qnext) * a.stride) + v0;
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const uint4 y = lut_eval4<K>(tt, x[g][u]);
+            dst[u * 32] = y;
+            if (latch) qd[u * 32] = y;
+        }
+    }
+}
+
+template <int U, int GP>
+__global__ void __launch_bounds__(256, GS_GP_MINB) k_level_lut_gp(LevelArgs a, uint32_t cpg_shift, uint32_t vec0) {
+    pdl_entry();
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t total = ((a.ng + GP - 1) / GP) << cpg_shift;
+    const uint32_t stride = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; warp < total; warp += stride) {
+        const uint32_t gi0 = (warp >> cpg_shift) * GP;
+        const uint32_t chunk = warp & ((1u << cpg_shift) - 1);
+        const uint32_t v0 = vec0 + chunk * 32 * U + lane;
+        const uint32_t n = min((uint32_t)GP, a.ng - gi0);
+        const uint32_t gate0 = a.g0 + gi0;
+        uint4 in[GP], au[GP];
+#pragma unroll
+        for (int g = 0; g < GP; ++g) {
+            const uint32_t gate = gate0 + min((uint32_t)g, n - 1);
+            in[g] = __ldg(a.din + gate);
+            au[g] = __ldg(reinterpret_cast<const uint4*>(a.aux) + gate);
+        }
+        const uint32_t k = au[0].w & 0xFFu;
+        bool uni = n == GP;
+#pragma unroll
+        for (int g = 1; g < GP; ++g) uni = uni && (au[g].w & 0xFFu) == k;
+        if (uni && k >= 1 && k <= 4) {
+            switch (k) {
+                case 1: lut_gates_gp<1, U, GP>(a, gate0, in, au, v0); break;
+                case 2: lut_gates_gp<2, U, GP>(a, gate0, in, au, v0); break;
+                case 3: lut_gates_gp<3, U, GP>(a, gate0, in, au, v0); break;
+                default: lut_gates_gp<4, U, GP>(a, gate0, in, au, v0); break;
+            }
+        } else {
+#pragma unroll
+            for (int g = 0; g < GP; ++g)
+                if ((uint32_t)g < n) lut_gate_any<U>(a, gate0 + g, in[g], au[g], v0);
         }
     }
 }
@@ -268,6 +353,26 @@ cudaError_t launch_level_lut(const LevelArgs& a, cudaStream_t s, uint32_t* grid_
                 blocks = cap;
                 if (grid_stride) *grid_stride = 1;
             }
+#if GS_LUT_GP
+            // short rows: GP = 4 / U gates per warp unit when the level still fills a wave
+            // of resident warps
+            if (!a.unroll && U < 4 && cpg == 1) {
+                const uint32_t GP = GS_GP_VPT / U;
+                const uint64_t units = (uint64_t)((a.ng + GP - 1) / GP);
+                const uint32_t gcap = a.grid_blocks / 4 * GS_GP_MINB;   // resident CTAs
+                if (units >= (gcap ? (uint64_t)gcap * 8 : (uint64_t)a.min_warps)) {
+                    uint32_t gblocks = (uint32_t)((units * 32 + 255) / 256);
+                    if (grid_stride) *grid_stride = 0;
+                    if (gcap && gblocks > gcap && gblocks <= 4 * gcap) {
+                        gblocks = gcap;
+                        if (grid_stride) *grid_stride = 1;
+                    }
+                    if (grid_stride) *grid_stride |= 2;
+                    if (U == 2) return launch_k(k_level_lut_gp<2, GS_GP_VPT / 2>, gblocks, s, a.pdl, a, 0u, a.vec0);
+                    return launch_k(k_level_lut_gp<1, GS_GP_VPT>, gblocks, s, a.pdl, a, 0u, a.vec0);
+                }
+            }
+#endif
             if (U == 8) return launch_k(k_level_lut_wide<8>, blocks, s, a.pdl, a, sh, a.vec0);
             if (U == 4) return launch_k(k_level_lut_wide<4>, blocks, s, a.pdl, a, sh, a.vec0);
             if (U == 2) return launch_k(k_level_lut_wide<2>, blocks, s, a.pdl, a, sh, a.vec0);

@@ -117,8 +117,8 @@ cudaError_t tile_setup(uint32_t tw, uint32_t ng, uint32_t n_slots, uint32_t n_ev
                        int desc_smem, uint32_t has_q, uint32_t* per_sm);
 cudaError_t launch_tile(const TileArgs& a, uint32_t tw, uint32_t ng, uint32_t grid, cudaStream_t s);
 
-// *grid_stride (may be NULL) is set to 1 when the launch's grid was capped at the resident
-// capacity (the grid-stride branch), else 0
+// *grid_stride (may be NULL): bit 0 set when the launch's grid was capped at the resident
+// capacity (the grid-stride branch), bit 1 when its warp units hold several gates
 // Kernel C (kernels_cluster.cu): a thread-block cluster owns a lane slab and walks every
 // level of every cycle of a step for it, cluster barrier between levels.
 struct ClusterArgs {

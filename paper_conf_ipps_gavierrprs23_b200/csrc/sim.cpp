@@ -217,6 +217,7 @@ struct gs_sim {
     std::vector<cudaStream_t> gstream;  // [groups - 1] branch streams (group 0: the caller's)
     std::vector<cudaEvent_t> gev;       // [0] fork, [1 .. groups - 1] joins
     uint64_t grid_stride_launches = 0;  // level launches whose grid was capped at residency
+    uint64_t multi_gate_launches = 0;   // level launches with several gates per warp unit
     uint32_t cluster_size = 0, clusters = 0, slab_vec = 0, n_slabs = 0;   // kernel C
 
     Ctl* ctl() const { return reinterpret_cast<Ctl*>(ws + L.ctl); }
@@ -299,7 +300,8 @@ static cudaError_t level_launch(gs_sim* s, uint32_t l, uint32_t parity, cudaStre
             break;
         default: e = launch_level_lut(a, st, &gs_flag); break;
     }
-    s->grid_stride_launches += gs_flag;
+    s->grid_stride_launches += gs_flag & 1u;
+    s->multi_gate_launches += (gs_flag >> 1) & 1u;
     return e;
 }
 
@@ -1012,7 +1014,7 @@ static gs_status sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
     double level_ms = 0, total_ms = 0, level_bytes = 0;
     uint64_t lvl_launches = 0, launches = 0;
     const uint64_t per = launches_per_cycle(s);
-    const uint64_t gs0 = s->grid_stride_launches;
+    const uint64_t gs0 = s->grid_stride_launches, mg0 = s->multi_gate_launches;
     // concurrent lane groups: the branches only overlap as they do in gs_sim_step when the
     // cycle is replayed as its graph, so profile a graph of the cycle with timing-event
     // nodes at the fork and the join (eager launches of G x levels kernels would measure
@@ -1069,6 +1071,7 @@ static gs_status sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
     // launch decisions of the host side: with lane groups they were taken once per captured
     // graph (per parity), eagerly once per level launch otherwise
     out->grid_stride_launches = s->grid_stride_launches - gs0;
+    out->multi_gate_launches = s->multi_gate_launches - mg0;
     clear_error();
     return GS_OK;
 }

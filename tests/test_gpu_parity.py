@@ -930,6 +930,33 @@ def test_grid_stride_branch_every_lane_vs_oracle(gates, groups, depth):
     assert np.array_equal(sigs, o["sig"])
 
 
+@pytest.mark.parametrize("lanes,groups,lut_k", [(4096, 1, 0), (8192, 1, 0), (8192, 2, 0), (4096, 1, 6)])
+def test_multi_gate_warp_units_every_lane_vs_oracle(lanes, groups, lut_k):
+    """Kernel A on short rows (4,096 lanes per lane group: 4 gates x 1 vector per thread;
+    8,192 in one group: 2 gates x 2 vectors): wide levels (~50k gates) with k-group edges
+    inside a warp unit, levels whose width is not a multiple of the unit, fused latches, and
+    (lut_k = 6, cone-collapsed) k = 5, 6 gates on the one-gate-at-a-time branch: every lane
+    vs the oracle of the original netlist, and the branch provably taken."""
+    nl = workloads.synthetic(200000, 8000, 32, 48, 4, seed=70 + lanes // 4096 + groups, name="gp")
+    prog = gs.Netlist.from_arrays(nl).compile(lut_k=lut_k)
+    if lut_k:
+        assert sum(prog.info["k_hist"][5:]) > 0
+    cycles = 3
+    sim = gs.Sim(prog, lanes, kernel="lut", lane_groups=groups)
+    assert sim.config["lane_groups"] == groups
+    sim.bind_generated(7)
+    sim.step(cycles - 1)
+    pr = sim.profile_step(1)
+    assert pr["multi_gate_launches"] > 0, pr
+    sim.sync()
+    out, regs, sigs = sim.read_outputs(), sim.read_registers(), sim.read_lane_signatures()
+    sim.close()
+    o = oracle.simulate(nl, np.arange(lanes), cycles, seed=7, want=("last", "regs", "sig"))
+    assert np.array_equal(gs.unpack_lanes(out).T, o["last"])
+    assert np.array_equal(gs.unpack_lanes(regs).T, o["regs"])
+    assert np.array_equal(sigs, o["sig"])
+
+
 # ------------------------------------------------------------------ seeded fuzzing
 def _fuzz_netlist(rng, case):
     """Random sequential netlist: sizes, fan-in mix (k = 0..6, repeated inputs allowed),
