@@ -61,7 +61,11 @@ def parse():
     ap.add_argument("--lanes", type=int, default=0, help="override lanes per GPU (unsharded configs)")
     ap.add_argument("--kernel", default="lut", choices=["lut", "poly", "ab", "tile", "cluster", "auto"])
     ap.add_argument("--cluster-size", type=int, default=0, help="kernel C: CTAs per cluster (0 = auto)")
-    ap.add_argument("--slab-lanes", type=int, default=0, help="kernel C: lanes per slab (0 = auto)")
+    ap.add_argument("--slab-lanes", type=int, default=0,
+                    help="kernel C: lanes per slab (0 = auto); kernel A: lanes per slab of the segmented "
+                         "slab schedule (0 = off)")
+    ap.add_argument("--slab-min-gates", type=int, default=0,
+                    help="kernel A slab schedule: narrowest level run per slab (0 = library default)")
     ap.add_argument("--levels", default="auto", choices=["auto", "balanced", "asap", "alap"],
                     help="level assignment (auto: the workload's measured best, DESIGN.md §6)")
     ap.add_argument("--no-balance", action="store_true", help="= --levels asap")
@@ -337,7 +341,8 @@ def main():
     sim = gs.Sim(prog, lanes, lane_offset=lane_offset, kernel=args.kernel, device=local, stream=stream,
                  lut_unroll=args.lut_unroll, pdl=not args.no_pdl, tile_words=args.tile_words,
                  tile_groups=args.tile_groups, lane_groups=args.lane_groups, flags=flags,
-                 cluster_size=args.cluster_size, slab_lanes=args.slab_lanes)
+                 cluster_size=args.cluster_size, slab_lanes=args.slab_lanes,
+                 slab_min_gates=args.slab_min_gates)
     sim.bind_generated(cfg.stim_seed)
     launches_per_cycle = sim.launches_per_cycle()
 
@@ -398,6 +403,8 @@ def main():
         per_launch_bytes = pr["level_bytes"] / max(pr["level_launches"], 1)
         groups = sim.config["lane_groups"]
         key = f"{cfg.name}:{lanes}:{args.kernel}:G{groups}"
+        if args.kernel == "lut" and sim.launch.get("slab_lanes"):
+            key += f":S{sim.launch['slab_lanes']}"
         tr, tr_src = insitu_traffic(key, gs.build_id(), info["program_hash"])
         ms_cycle = ms_max / (args.steps * cycles_per_rank_step)
         dram = None

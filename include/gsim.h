@@ -271,7 +271,18 @@ typedef struct {
     uint32_t cluster_size;        /* CLUSTER: CTAs per thread-block cluster (1, 2, 4, 8 or 16;
                                      0 = auto)                                             */
     uint32_t slab_lanes;          /* CLUSTER: lanes per slab, a multiple of 128 dividing lanes
-                                     (0 = auto)                                            */
+                                     (0 = auto).
+                                     LUT: lanes per slab of the segmented schedule (0 = off):
+                                     every run of consecutive levels at least slab_min_gates
+                                     wide executes slab after slab, each slab through all
+                                     levels of the run, so a level's rows of the slab are
+                                     still in L2 when the run's next levels read them; the
+                                     other levels run over all lanes (of the lane group:
+                                     each concurrent group runs its own slab schedule).  A
+                                     multiple of 4096 dividing the lanes of a group; with
+                                     lane_groups 0 the schedule runs as one group.         */
+    uint32_t slab_min_gates;      /* LUT segmented schedule: narrowest level that runs per
+                                     slab (0 = 32768 gates)                                */
 } gs_sim_opts;
 /* flags: launch the per-cycle kernels WITHOUT programmatic dependent launch (by default a
  * level kernel may become resident while its predecessor drains; A/B measurement only). */

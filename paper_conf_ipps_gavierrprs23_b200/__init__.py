@@ -78,7 +78,7 @@ class gs_sim_opts(C.Structure):
                 ("trace_words", C.c_void_p), ("trace_cycles", C.c_uint32), ("use_graphs", C.c_int),
                 ("lut_unroll", C.c_uint32), ("flags", C.c_uint32), ("tile_words", C.c_uint32),
                 ("tile_groups", C.c_uint32), ("lane_groups", C.c_uint32), ("cluster_size", C.c_uint32),
-                ("slab_lanes", C.c_uint32)]
+                ("slab_lanes", C.c_uint32), ("slab_min_gates", C.c_uint32)]
 
 
 class gs_signature(C.Structure):
@@ -328,7 +328,7 @@ class Sim:
                  device: int = 0, stream=None, trace_words=(), trace_cycles: int = 0,
                  use_graphs: bool = True, lut_unroll: int = 0, pdl: bool = True,
                  tile_words: int = 0, tile_groups: int = 0, flags: int = 0, lane_groups: int = 0,
-                 cluster_size: int = 0, slab_lanes: int = 0):
+                 cluster_size: int = 0, slab_lanes: int = 0, slab_min_gates: int = 0):
         import torch
         self.program = program
         self.lanes, self.words = int(lanes), int(lanes) // 64
@@ -340,7 +340,7 @@ class Sim:
                         _p(self._tw) if len(self._tw) else None, int(trace_cycles),
                         1 if use_graphs else 0, int(lut_unroll),
                         (0 if pdl else GS_SIM_NO_PDL) | int(flags), int(tile_words), int(tile_groups),
-                        int(lane_groups), int(cluster_size), int(slab_lanes))
+                        int(lane_groups), int(cluster_size), int(slab_lanes), int(slab_min_gates))
         nbytes = C.c_size_t()
         _call("gs_sim_workspace_bytes", program.h, C.byref(o), C.byref(nbytes))
         self.workspace = torch.empty(int(nbytes.value) + 256, dtype=torch.uint8, device=self.device)

@@ -219,6 +219,10 @@ struct gs_sim {
     uint64_t grid_stride_launches = 0;  // level launches whose grid was capped at residency
     uint64_t multi_gate_launches = 0;   // level launches with several gates per warp unit
     uint32_t cluster_size = 0, clusters = 0, slab_vec = 0, n_slabs = 0;   // kernel C
+    // kernel A segmented slab schedule: slabs of lut_slab_vec 16-byte vectors (lut_slabs per
+    // lane group); levels with slabbed[l] != 0 run slab-major in runs of consecutive such levels
+    uint32_t lut_slabs = 1, lut_slab_vec = 0;
+    std::vector<uint8_t> slabbed;
 
     Ctl* ctl() const { return reinterpret_cast<Ctl*>(ws + L.ctl); }
     uint8_t* state() const { return ws + L.state; }
@@ -282,13 +286,13 @@ static EndArgs end_args(const gs_sim* s, uint32_t parity) {
     return e;
 }
 
-static cudaError_t level_launch(gs_sim* s, uint32_t l, uint32_t parity, cudaStream_t st, uint32_t group = 0) {
+// vec0 / vslab: the lane range of the launch in 16-byte vectors (vslab 0 = the whole row)
+static cudaError_t level_launch(gs_sim* s, uint32_t l, uint32_t parity, cudaStream_t st, uint32_t vec0 = 0,
+                                uint32_t vslab = 0) {
     LevelArgs a = level_args(s, l, parity);
     a.unroll = s->opts.lut_unroll;
-    if (s->groups > 1) {
-        a.vslab = (s->words / 2) / s->groups;
-        a.vec0 = group * a.vslab;
-    }
+    a.vec0 = vec0;
+    a.vslab = vslab;
     uint32_t gs_flag = 0;
     cudaError_t e = cudaSuccess;
     switch (s->opts.kernel) {
@@ -379,6 +383,31 @@ static cudaError_t cluster_launch(const gs_sim* s, uint32_t ncycles, cudaStream_
     return launch_cluster(a, s->clusters, s->cluster_size, st);
 }
 
+// The level chain of one cycle over the lane range [v0, v0 + vlen) (16-byte vectors; vlen 0
+// = the whole row).  With the segmented slab schedule a run of consecutive wide levels goes
+// slab after slab (each slab through every level of the run) and the other levels over the
+// whole range; levels only read earlier levels of the same lanes, so any slab order is valid.
+static cudaError_t level_chain(gs_sim* s, uint32_t parity, cudaStream_t st, uint32_t v0, uint32_t vlen) {
+    const Program& p = *s->prog;
+    const uint32_t nslab = s->lut_slab_vec ? (vlen ? vlen : s->words / 2) / s->lut_slab_vec : 1;
+    cudaError_t e = cudaSuccess;
+    for (uint32_t l = 0; l < p.n_levels;) {
+        if (nslab <= 1 || !s->slabbed[l]) {
+            if ((e = level_launch(s, l, parity, st, v0, vlen)) != cudaSuccess) return e;
+            ++l;
+            continue;
+        }
+        uint32_t m = l;
+        while (m < p.n_levels && s->slabbed[m]) ++m;
+        for (uint32_t j = 0; j < nslab; ++j)
+            for (uint32_t ll = l; ll < m; ++ll)
+                if ((e = level_launch(s, ll, parity, st, v0 + j * s->lut_slab_vec, s->lut_slab_vec)) != cudaSuccess)
+                    return e;
+        l = m;
+    }
+    return e;
+}
+
 // evs (profiling): timing events around every level launch (one group), or around the
 // concurrent level region (lane groups); ext = the launches are being captured, record the
 // events as graph nodes
@@ -393,15 +422,21 @@ static cudaError_t cycle_launches(gs_sim* s, uint32_t parity, cudaStream_t st,
         // before the end-of-cycle kernel; the branches share nothing but the stimulus rows
         if (evs) cudaEventRecordWithFlags((*evs)[0], st, ext ? cudaEventRecordExternal : 0u);
         if ((e = cudaEventRecord(s->gev[0], st)) != cudaSuccess) return e;
+        const uint32_t vs = (s->words / 2) / s->groups;
         for (uint32_t br = 0; br < s->groups; ++br) {
             cudaStream_t b = br ? s->gstream[br - 1] : st;
             if (br && (e = cudaStreamWaitEvent(b, s->gev[0], 0)) != cudaSuccess) return e;
-            for (uint32_t l = 0; l < p.n_levels; ++l)
-                if ((e = level_launch(s, l, parity, b, br)) != cudaSuccess) return e;
+            if ((e = level_chain(s, parity, b, br * vs, vs)) != cudaSuccess) return e;
             if (br && (e = cudaEventRecord(s->gev[br], b)) != cudaSuccess) return e;
         }
         for (uint32_t br = 1; br < s->groups; ++br)
             if ((e = cudaStreamWaitEvent(st, s->gev[br], 0)) != cudaSuccess) return e;
+        if (evs) cudaEventRecordWithFlags((*evs)[1], st, ext ? cudaEventRecordExternal : 0u);
+        return launch_end_cycle(end_args(s, parity), st);
+    }
+    if (s->lut_slabs > 1) {
+        if (evs) cudaEventRecordWithFlags((*evs)[0], st, ext ? cudaEventRecordExternal : 0u);
+        if ((e = level_chain(s, parity, st, 0, 0)) != cudaSuccess) return e;
         if (evs) cudaEventRecordWithFlags((*evs)[1], st, ext ? cudaEventRecordExternal : 0u);
         return launch_end_cycle(end_args(s, parity), st);
     }
@@ -540,8 +575,12 @@ static gs_status sim_create(const gs_program* prog, const gs_sim_opts* opts_in, 
     if (gs_status st = make_plans(p, *opts, pls)) return st;
     Layout L = make_layout(p, *opts, pls);
     if (bytes < L.total) return fail(GS_ERR_BUFFER_TOO_SMALL, "gs_sim_create: workspace smaller than gs_sim_workspace_bytes");
+    const bool lut_slab = opts->kernel == GS_KERNEL_LUT && opts->slab_lanes;
     uint32_t groups = opts->lane_groups;
-    if (groups == 0) groups = auto_lane_groups(p, *opts);
+    if (groups == 0) groups = lut_slab ? 1 : auto_lane_groups(p, *opts);
+    if (lut_slab && (opts->slab_lanes % 4096 || (opts->lanes / groups) % opts->slab_lanes || opts->lanes % groups))
+        return fail(GS_ERR_ARG, "gs_sim_create: LUT slab_lanes must be a multiple of 4096 dividing the lanes "
+                                "of a lane group");
     if (groups > 1) {
         const uint32_t vrow = words / 2;
         if (opts->kernel != GS_KERNEL_LUT || words % 2 || vrow % groups || (vrow / groups) % 32)
@@ -569,6 +608,13 @@ static gs_status sim_create(const gs_program* prog, const gs_sim_opts* opts_in, 
     s->tile_steps = pls.steps;
     s->pdl = (opts->flags & GS_SIM_NO_PDL) ? 0u : 1u;
     s->groups = groups;
+    if (lut_slab && opts->slab_lanes < opts->lanes / groups) {
+        s->lut_slabs = (uint32_t)(opts->lanes / groups / opts->slab_lanes);
+        s->lut_slab_vec = opts->slab_lanes / 128;
+        const uint32_t wmin = opts->slab_min_gates ? opts->slab_min_gates : 32768u;
+        s->slabbed.assign(p.n_levels, 0);
+        for (uint32_t l = 0; l < p.n_levels; ++l) s->slabbed[l] = p.level_off[l + 1] - p.level_off[l] >= wmin;
+    }
     {
         int sms = 148;
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, opts->device);
@@ -945,9 +991,19 @@ static uint64_t launches_per_cycle(const gs_sim* s) {
         return 1;                                          // per gs_sim_step call, not per cycle
     uint64_t lv = 0;
     for (uint32_t l = 0; l < p.n_levels; ++l)
-        if (p.level_off[l + 1] > p.level_off[l]) lv++;
+        if (p.level_off[l + 1] > p.level_off[l]) lv += s->lut_slabs > 1 && s->slabbed[l] ? s->lut_slabs : 1;
     const uint64_t per_level = s->opts.kernel == GS_KERNEL_AB ? 2 : 1;
     return (p.n_pi ? 1 : 0) + lv * per_level * s->groups + 1;
+}
+
+// level launches of one cycle (lane groups and the slab schedule included)
+static uint64_t level_launches_per_cycle(const gs_sim* s) {
+    const Program& p = *s->prog;
+    uint64_t n = 0;
+    for (uint32_t l = 0; l < p.n_levels; ++l)
+        if (p.level_off[l + 1] > p.level_off[l])
+            n += (uint64_t)s->groups * (s->lut_slabs > 1 && s->slabbed[l] ? s->lut_slabs : 1);
+    return n;
 }
 
 static gs_status sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
@@ -1033,7 +1089,8 @@ static gs_status sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
     };
     for (uint32_t i = 0; i < n; ++i) {
         const uint32_t parity = (uint32_t)(s->cycle & 1);
-        if (s->groups > 1) {
+        const bool region = s->groups > 1 || s->lut_slabs > 1;
+        if (region) {
             CU(prof_graph(parity));
             CU(cudaEventRecord(e0, s->stream));
             CU(cudaGraphLaunch(px[parity], s->stream));
@@ -1047,11 +1104,11 @@ static gs_status sim_profile_step(gs_sim* s, uint32_t n, gs_profile* out) {
         float ms = 0;
         cudaEventElapsedTime(&ms, e0, e1);
         total_ms += ms;
-        if (s->groups > 1) {           // concurrent branches cover every level
+        if (region) {                  // concurrent branches / slab runs cover every level
             cudaEventElapsedTime(&ms, evs[0], evs[1]);
             level_ms += ms;
             level_bytes += all_bytes;
-            for (uint32_t l = 0; l < p.n_levels; ++l) lvl_launches += p.level_off[l + 1] > p.level_off[l] ? s->groups : 0;
+            lvl_launches += level_launches_per_cycle(s);
         } else {
             for (uint32_t l = 0; l < p.n_levels; ++l) {
                 if (p.level_off[l + 1] == p.level_off[l]) continue;
@@ -1158,7 +1215,8 @@ gs_status gs_sim_get_launch(const gs_sim* s, gs_launch_info* out) {
         out->grid = s->opts.kernel == GS_KERNEL_TILE ? s->tile_grid
                     : s->opts.kernel == GS_KERNEL_CLUSTER ? s->clusters * s->cluster_size : 0;
         out->cluster_size = s->cluster_size;
-        out->slab_lanes = s->slab_vec * 128;
+        out->slab_lanes = s->opts.kernel == GS_KERNEL_CLUSTER ? s->slab_vec * 128
+                          : s->lut_slabs > 1 ? s->lut_slab_vec * 128 : 0;
         out->live_slots = s->opts.kernel == GS_KERNEL_TILE ? s->tile.n_slots : 0;
         clear_error();
         return GS_OK;

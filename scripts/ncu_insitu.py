@@ -62,6 +62,8 @@ def main():
     t_ns = statistics.median(v["gpu__time_duration.sum"] for v in vals)
     hit = statistics.median(v["lts__t_sector_hit_rate.pct"] for v in vals)
     key = f"{cfg['workload'].split(':')[0]}:{cfg['lanes_per_sub_batch']}:{cfg['kernel']}:G{cfg['lane_groups']}"
+    if cfg["kernel"] == "lut" and cfg.get("launch", {}).get("slab_lanes"):
+        key += f":S{cfg['launch']['slab_lanes']}"     # kernel A segmented slab schedule
     entry = {"dram_bytes_per_cycle": rd + wr, "read_bytes": rd, "write_bytes": wr, "l2_hit_pct": hit,
              "ncu_graph_us": t_ns / 1e3, "graphs": len(vals), "build_id": cfg["build_id"],
              "program_hash": cfg["program_hash"], "bench_args": " ".join(bargs),

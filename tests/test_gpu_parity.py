@@ -957,6 +957,46 @@ def test_multi_gate_warp_units_every_lane_vs_oracle(lanes, groups, lut_k):
     assert np.array_equal(sigs, o["sig"])
 
 
+@pytest.mark.parametrize("slab,min_gates,balance,groups",
+                         [(4096, 10000, False, 1), (8192, 1, True, 1), (4096, 1, False, 1), (4096, 10000, False, 2)])
+def test_slab_schedule_every_lane_vs_oracle(slab, min_gates, balance, groups):
+    """Kernel A's segmented slab schedule: runs of levels >= min_gates wide go slab after slab
+    (4,096-lane slabs take the multi-gate units), the other levels over all lanes of the lane
+    group (16,384 lanes, 1 or 2 concurrent groups); every lane vs the oracle, and the same
+    lane_sig_sum as the plain schedule."""
+    nl = workloads.synthetic(200000, 8000, 32, 48, 4, seed=80 + slab // 4096, name="slab")
+    prog = compile_nl(nl, balance)
+    lanes, cycles = 16384, 3
+    sim = gs.Sim(prog, lanes, kernel="lut", slab_lanes=slab, slab_min_gates=min_gates, lane_groups=groups)
+    assert sim.launch["slab_lanes"] == slab and sim.config["lane_groups"] == groups
+    widths = prog.level_widths()
+    wide = int((widths >= min_gates).sum())
+    assert 0 < wide
+    per_cycle = sim.launches_per_cycle()
+    assert per_cycle == 2 + groups * ((len(widths) - wide) + wide * (lanes // groups // slab))
+    sim.bind_generated(8)
+    sim.step(cycles - 1)
+    pr = sim.profile_step(1)
+    assert pr["level_launches"] == per_cycle - 2
+    sim.sync()
+    out, regs, sigs = sim.read_outputs(), sim.read_registers(), sim.read_lane_signatures()
+    sig = sim.signature()
+    sim.close()
+    o = oracle.simulate(nl, np.arange(lanes), cycles, seed=8, want=("last", "regs", "sig"))
+    assert np.array_equal(gs.unpack_lanes(out).T, o["last"])
+    assert np.array_equal(gs.unpack_lanes(regs).T, o["regs"])
+    assert np.array_equal(sigs, o["sig"])
+    assert sig["lane_sig_sum"] == run_gpu(nl, lanes, cycles, seed=8, prog=prog)["signature"]["lane_sig_sum"]
+
+
+def test_slab_schedule_bad_shapes_rejected():
+    nl = workloads.synthetic(3000, 100, 16, 48, 4, seed=81, name="slabbad")
+    prog = compile_nl(nl)
+    for kw in (dict(slab_lanes=2048), dict(slab_lanes=12288), dict(slab_lanes=8192, lane_groups=4)):
+        with pytest.raises(gs.GsError):
+            gs.Sim(prog, 16384, kernel="lut", **kw)
+
+
 # ------------------------------------------------------------------ seeded fuzzing
 def _fuzz_netlist(rng, case):
     """Random sequential netlist: sizes, fan-in mix (k = 0..6, repeated inputs allowed),
