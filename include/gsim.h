@@ -363,7 +363,8 @@ typedef struct {
                                      per CTA, descriptor source (0 global, 1 resident, 2 TMA;
                                      | 4: narrow 8-byte descriptors, k <= 2 and no registers) */
     uint32_t grid;                /* kernels T / C: CTAs launched per step                  */
-    uint32_t cluster_size, slab_lanes;             /* kernel C                                 */
+    uint32_t cluster_size, slab_lanes;             /* kernel C; slab_lanes also kernel A's slab
+                                     schedule (0 = off)                                    */
     uint32_t live_slots;          /* kernel T: shared-memory slots per tile                 */
 } gs_launch_info;
 gs_status gs_sim_get_launch(const gs_sim* sim, gs_launch_info* out);
