@@ -33,6 +33,12 @@ __device__ __forceinline__ void pdl_entry() {
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 
+// L1 prefetch of a line of program constants (gate descriptors), issued before pdl_entry()
+// so its latency overlaps the previous kernel's drain
+__device__ __forceinline__ void prefetch_l1(const void* p) {
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
+}
+
 template <typename... KArgs, typename... Args>
 static cudaError_t launch_k(void (*kern)(KArgs...), uint32_t blocks, cudaStream_t s, uint32_t pdl,
                             Args... args) {
