@@ -416,7 +416,7 @@ def main():
                     "note": "actual DRAM bytes of one cycle (in-situ ncu graph capture of this build and "
                             "program) / this run's device time per cycle"}
         lvl_per_cycle = pr["level_launches"] / max(ncyc, 1)
-        roof = {"bound": "hbm", "kernel": "k_level_lut_wide<4>" if args.kernel in ("lut", "auto") else args.kernel,
+        roof = {"bound": "hbm", "kernel": "k_level_lut_wide<4, false>" if args.kernel in ("lut", "auto") else args.kernel,
                 "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s", "frac": achieved / pk["hbm_gbs"],
                 "frac_basis": "algorithmic gather-model bytes (k reads + 1 write + fused latch per gate-row) "
                               "/ measured HBM copy peak; L2 hits let it exceed the DRAM fraction, which is "
